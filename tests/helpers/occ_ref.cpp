@@ -1,0 +1,39 @@
+// Test helper (not product, not oracle): NVIDIA's header-only occupancy calculator
+// (/usr/local/cuda/include/cuda_occupancy.h), used as an independent pin for the
+// oracle's O1 calculator.  Reads lines "T regs smem_static smem_dyn" on stdin and
+// prints the CTAs/SM that cudaOccMaxActiveBlocksPerMultiprocessor reports for a
+// B200 (cc 10.0) with the MAX_SHARED carveout and the dynamic-smem opt-in set.
+#include <cuda_occupancy.h>
+#include <cstdio>
+
+int main() {
+    cudaOccDeviceProp prop;
+    prop.computeMajor = 10;
+    prop.computeMinor = 0;
+    prop.maxThreadsPerBlock = 1024;
+    prop.maxThreadsPerMultiprocessor = 2048;
+    prop.regsPerBlock = 65536;
+    prop.regsPerMultiprocessor = 65536;
+    prop.warpSize = 32;
+    prop.sharedMemPerBlock = 49152;
+    prop.sharedMemPerMultiprocessor = 233472;
+    prop.numSms = 148;
+    prop.sharedMemPerBlockOptin = 232448;
+    prop.reservedSharedMemPerBlock = 1024;
+    int T, regs, sst, sdyn;
+    while (std::scanf("%d %d %d %d", &T, &regs, &sst, &sdyn) == 4) {
+        cudaOccFuncAttributes attr;
+        attr.maxThreadsPerBlock = 1024;
+        attr.numRegs = regs;
+        attr.sharedSizeBytes = (size_t)sst;
+        attr.partitionedGCConfig = PARTITIONED_GC_OFF;
+        attr.shmemLimitConfig = FUNC_SHMEM_LIMIT_OPTIN;
+        attr.maxDynamicSharedSizeBytes = 232448 - sst;
+        cudaOccDeviceState state;
+        state.carveoutConfig = SHAREDMEM_CARVEOUT_MAX_SHARED;
+        cudaOccResult res;
+        cudaOccError e = cudaOccMaxActiveBlocksPerMultiprocessor(&res, &prop, &attr, &state, T, (size_t)sdyn);
+        std::printf("%d\n", e == CUDA_OCC_SUCCESS ? res.activeBlocksPerMultiprocessor : -1);
+    }
+    return 0;
+}

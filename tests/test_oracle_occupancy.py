@@ -1,0 +1,95 @@
+"""Pins for oracle O1 (occupancy calculator + levels) -- PAPER.md Eq. (1).
+
+The oracle is pinned to things other than itself:
+  * SURVEY.md Appendix A hand-worked tables (B200, cc 10.0);
+  * NVIDIA's header-only cudaOccMaxActiveBlocksPerMultiprocessor (an independent
+    implementation, compiled from cuda_occupancy.h by tests/helpers/occ_ref.cpp);
+  * the Kepler GTX680 case behind Fig. 1 (P:L91 best at 50 %, P:L713 platform,
+    Table 2 P:L733 imageDenoising 63 registers).
+"""
+import itertools
+
+import pytest
+
+from oracle import occupancy as O
+
+# regs/thread -> CTAs/SM at T = 64, 128, 256.
+APPENDIX_A = {
+    32: (32, 16, 8), 40: (24, 12, 6), 48: (20, 10, 5), 56: (18, 9, 4), 64: (16, 8, 4),
+    72: (14, 7, 3), 80: (12, 6, 3), 88: (10, 5, 2), 96: (10, 5, 2), 104: (8, 4, 2),
+    128: (8, 4, 2), 136: (6, 3, 1), 168: (6, 3, 1), 176: (4, 2, 1), 255: (4, 2, 1),
+}
+# Appendix A: dynamic bytes pinning exactly k CTAs/SM at T=64, no static smem.
+APPENDIX_A_PAD = {1: 115840, 2: 76928, 3: 57472, 4: 45696, 8: 24960, 12: 17024, 16: 12800,
+                  24: 8320, 31: 6400, 32: 0}
+
+
+@pytest.mark.parametrize("regs", sorted(APPENDIX_A))
+def test_appendix_a_register_table(regs):
+    for T, want in zip((64, 128, 256), APPENDIX_A[regs]):
+        assert O.ctas_per_sm(O.B200, T, regs) == want, (T, regs)
+
+
+@pytest.mark.parametrize("k", sorted(APPENDIX_A_PAD))
+def test_appendix_a_pad_table(k):
+    pad = O.pad_for(O.B200, 64, 32, 0, 0, k)
+    assert pad == APPENDIX_A_PAD[k]
+    assert O.ctas_per_sm(O.B200, 64, 32, 0, pad) == k
+    if pad > 0:  # minimal: 128 bytes less admits k+1
+        assert O.ctas_per_sm(O.B200, 64, 32, 0, pad - 128) == k + 1
+
+
+def test_against_nvidia_header_grid(occ_ref):
+    cases = []
+    for T in (32, 64, 96, 128, 160, 256, 384, 512, 1024):
+        for regs in (16, 24, 32, 37, 39, 40, 48, 56, 63, 64, 72, 80, 96, 128, 168, 200, 255):
+            for sst, sdyn in ((0, 0), (0, 4096), (2048, 10000), (8192, 0), (0, 45000), (0, 100000),
+                              (1024, 226000)):
+                cases.append((T, regs, sst, sdyn))
+    want = occ_ref(cases)
+    got = [O.ctas_per_sm(O.B200, *c) for c in cases]
+    bad = [(c, g, w) for c, g, w in zip(cases, got, want) if g != w]
+    assert not bad, bad[:10]
+
+
+@pytest.mark.parametrize("T,natural,need", [(64, 39, 0), (128, 255, 0), (128, 39, 8704), (256, 20, 0),
+                                            (128, 200, 30000), (256, 96, 2048), (64, 255, 4096)])
+def test_every_level_realises_k_per_nvidia_header(occ_ref, T, natural, need):
+    lv = O.levels(O.B200, T, natural, 0, need)
+    assert [l.ctas_per_sm for l in lv] == sorted({l.ctas_per_sm for l in lv})
+    cases = [(T, natural if l.reg_cap == 0 else l.reg_cap, 0, need + l.smem_pad_bytes) for l in lv]
+    assert occ_ref(cases) == [l.ctas_per_sm for l in lv]
+    # k_max is reached and every k below it is feasible (reading R-A10)
+    assert [l.ctas_per_sm for l in lv] == list(range(1, lv[-1].ctas_per_sm + 1))
+
+
+def test_register_ladder_255_regs_T128():
+    lv = {l.ctas_per_sm: l for l in O.levels(O.B200, 128, 255)}
+    rungs = {k: l.reg_cap for k, l in lv.items() if l.smem_pad_bytes == 0}
+    assert rungs == {2: 0, 3: 168, 4: 128, 5: 96, 6: 80, 7: 72, 8: 64, 9: 56, 10: 48, 12: 40, 16: 32}
+    assert lv[1].reg_cap == 0 and lv[1].smem_pad_bytes > 0
+    assert lv[11].reg_cap == 40 and lv[11].smem_pad_bytes > 0
+    assert O.original_level_index(list(lv.values())) == 1
+
+
+def test_kepler_gtx680_fig1_sanity():
+    # imageDenoising 63 regs (Table 2) at 256 threads -> 4 CTAs = 32 warps = 50 % (Fig. 1 best).
+    assert O.ctas_per_sm(O.GTX680, 256, 63) == 4
+    assert O.occupancy(O.GTX680, 256, 4) == 0.5
+    assert O.ctas_per_sm(O.GTX680, 64, 63) == 16  # 16-CTA Kepler limit binds at 8x8 CTAs
+    caps = {32: 1.0, 40: 0.75, 48: 0.625, 56: 0.5}
+    for r, occ in caps.items():
+        assert O.occupancy(O.GTX680, 256, O.ctas_per_sm(O.GTX680, 256, r)) == occ
+    # 0.875 is unreachable by register caps (absent from Fig. 1's axis)
+    reach = {O.occupancy(O.GTX680, 256, O.ctas_per_sm(O.GTX680, 256, r)) for r in range(16, 64)}
+    assert 0.875 not in reach
+
+
+def test_limiter_mask_and_eq1_upper_bound():
+    # Eq. (1) without granularity is an upper bound of the calculator's answer.
+    for T, regs, smem in itertools.product((64, 128, 256), (24, 40, 64, 128, 255), (0, 8192, 40000)):
+        k = O.ctas_per_sm(O.B200, T, regs, 0, smem)
+        eq1_threads = min(65536 / regs, 233472 / ((smem + 1024) / T))
+        assert k * T <= eq1_threads + 1e-9
+        m = O.limiter_mask(O.B200, T, regs, 0, smem)
+        assert m != 0
