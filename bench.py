@@ -1,0 +1,403 @@
+#!/usr/bin/env python3
+"""bench.py -- Orion occupancy-tuned hot path on B200 (BASELINE.json metric).
+
+One "step" = one application iteration of the whole hot path on one synthetic
+frame: orion_tune_step (Fig. 9 dynamic selection over the Fig. 8 ladder of the
+occupancy variants orion_build_variants produced from orion_levels) launching
+the NLM imageDenoising kernel on a 2048x2048 RGBA frame (config C2,
+BASELINE.json configs[1]).  Variants are built and every level is swept
+(orion_sweep, the exhaustive brute-force reference) before the timed region.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--workload c1|c2|c3|c4] [--no-cpu-baseline]
+
+Multi-GPU (torchrun, one process per GPU): weak scaling -- every rank tunes and
+runs its own C2 frames (no data-path collective); time = max over ranks.
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "tuned Mpix/s vs max-occupancy build; tuner regret vs exhaustive level sweep"
+
+# Workloads (BASELINE.json configs).  algorithmic FP32-pipe instructions per output unit
+# of the formulation each kernel implements, and HBM bytes per unit.
+WORKLOADS = {
+    "c1": dict(kernel="knn_f4", W=64, H=64, sigma=0.2, unit="Mpix/s", name="imageDenoising KNN 64x64 RGBA r=3",
+               insts=49 * 15 + 10, bytes=32),
+    "c2": dict(kernel="nlm_f4", W=2048, H=2048, sigma=0.13, unit="Mpix/s", name="imageDenoising NLM 2048x2048 RGBA",
+               insts=49 * 24 + 10, bytes=32),
+    "c4": dict(kernel="nlm_f4_regheavy", W=4096, H=4096, sigma=0.13, unit="Mpix/s",
+               name="register-heavy NLM 4096x4096 RGBA, maxrregcount caps", insts=49 * (49 * 6 + 9) + 10, bytes=32),
+    "c3": dict(kernel="hotspot_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
+               insts=12, bytes=12),
+}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi-equivalent sampling (NVML) of SM clock + throttle reasons during the timed region."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clock_setting"}
+
+    def __init__(self, index: int, period: float = 0.02):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self.period = period
+        self.stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = str(e)
+            self.max_mhz = None
+
+    def _run(self):
+        while not self.stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self.stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None, "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons - {"gpu_idle"}), "samples": len(self.samples)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# ---------------------------------------------------------------------------------------------
+def cpu_baseline_nlm(kind: str, W: int, H: int, sigma: float, budget_s: float):
+    """The oracle (C, double, single thread) timed on a bounded row band of the same frame."""
+    import numpy as np
+    import oracle
+    import synth
+    rows_per = 2 if kind == "nlm" else 16
+    y0 = H // 2
+    img = synth.noisy_rgba(W, H, seed=1, sigma=sigma, row_begin=y0 - 6, row_end=y0 + 6 + 4096)
+    t0 = time.perf_counter()
+    n = 0
+    y = y0
+    while True:
+        oracle.denoise(kind, img, height=H, row0=y0 - 6, y_begin=y, y_end=min(H, y + rows_per))
+        n += min(H, y + rows_per) - y
+        y += rows_per
+        dt = time.perf_counter() - t0
+        if dt >= budget_s or y >= H:
+            break
+    return n * W, dt, f"{n} rows x {W} px of the C2 frame (rows {y0}..{y0 + n}), oracle/denoise.c, double"
+
+
+def cpu_baseline_hotspot(W: int, steps: int, budget_s: float):
+    import oracle
+    import synth
+    rows = 64
+    t0a, pw = synth.thermal_inputs(W, rows, seed=1)
+    t0 = time.perf_counter()
+    n = 0
+    while True:
+        oracle.hotspot(t0a, pw, steps, precision="f64")
+        n += 1
+        dt = time.perf_counter() - t0
+        if dt >= budget_s:
+            break
+    return n * rows * W * steps, dt, f"{n} x ({rows} x {W} cells x {steps} steps), oracle/stencil.c f64"
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, timed on bounded samples (rank 0 only)."""
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return
+    wl = WORKLOADS[args.workload]
+    K, Wm = args.steps, args.warmup
+    per_step = max(0.2, min(2.0, 150.0 / max(1, K + Wm)))
+    times, units = [], []
+    for s in range(Wm + K):
+        if wl["kernel"] == "hotspot_f32":
+            u, dt, sample = cpu_baseline_hotspot(wl["W"], 1, per_step)
+        else:
+            u, dt, sample = cpu_baseline_nlm("knn" if wl["kernel"].startswith("knn") else "nlm", wl["W"], wl["H"],
+                                             wl.get("sigma", 0.13), per_step)
+        if s >= Wm:
+            times.append(dt)
+            units.append(u)
+    value = sum(units) / sum(times) / 1e6
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": wl["unit"], "n_gpus": world,
+            "steps": K, "warmup": Wm, "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": wl["name"], "impl": "CPU oracle (plain C, double), single thread"},
+            "cpu_baseline": {"value": value, "unit": wl["unit"], "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": wl["unit"], "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------------------------
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_middleware_hayeslcsz16_b200 import orion as O
+
+    world, rank, local = dist_env()
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py: no CUDA device (the product has no CPU path)")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    sp = stream.cuda_stream
+    wl = WORKLOADS[args.workload]
+    kernel, W, H = wl["kernel"], wl["W"], wl["H"]
+    is_stencil = kernel == "hotspot_f32"
+
+    # ---- multi-version binary: probe -> levels -> build (offline, untimed) ----------------
+    t_build = time.perf_counter()
+    variants, res = O.build_all_levels(local, kernel)
+    t_build = time.perf_counter() - t_build
+    nlev = len(variants)
+    lv = [variants.level(i) for i in range(nlev)]
+    infos = [variants.info(i) for i in range(nlev)]
+    orig = next(i for i, l in enumerate(variants.planned) if l.reg_cap == 0 and l.smem_pad_bytes == 0)
+    kmax = nlev - 1
+
+    # ---- inputs resident in HBM: a pool of frames larger than L2 -------------------------
+    frame_bytes = W * H * (4 if is_stencil else 16)
+    nframes = max(2, math.ceil(2 * 126e6 / (2 * frame_bytes)) + 1)
+    if is_stencil:
+        nframes = 1
+        t_a = torch.empty((H, W), device=dev)
+        t_b = torch.empty((H, W), device=dev)
+        pw = torch.empty((H, W), device=dev)
+        O.generate_thermal(local, t_a.data_ptr(), pw.data_ptr(), W, H, seed=1 + rank, stream=sp)
+        state = {"a": t_a, "b": t_b}
+
+        def step_args(s):
+            a = O.hotspot_args(state["a"].data_ptr(), state["b"].data_ptr(), pw.data_ptr(), W, H)
+            state["a"], state["b"] = state["b"], state["a"]
+            return a
+    else:
+        srcs = [torch.empty((H, W, 4), device=dev) for _ in range(nframes)]
+        dsts = [torch.empty((H, W, 4), device=dev) for _ in range(nframes)]
+        for f, t in enumerate(srcs):
+            O.generate_rgba(local, t.data_ptr(), W, H, seed=1 + f + 97 * rank, sigma=wl["sigma"], stream=sp)
+
+        def step_args(s):
+            f = s % nframes
+            return O.denoise_args(kernel, srcs[f].data_ptr(), dsts[f].data_ptr(), W, H)
+    torch.cuda.synchronize()
+
+    # ---- exhaustive sweep (brute-force reference, Fig. 11 Orion-Max/Min) ------------------
+    sweep_args = step_args(0)
+    if is_stencil:
+        state["a"], state["b"] = t_a, t_b
+        sweep_args = O.hotspot_args(t_a.data_ptr(), t_b.data_ptr(), pw.data_ptr(), W, H)
+    ms = variants.sweep(sweep_args, sp, rounds=args.rounds)
+    best = min(range(nlev), key=lambda i: ms[i])
+    worst = max(range(nlev), key=lambda i: ms[i])
+
+    # ---- the tuned loop: warmup (includes Fig. 9 exploration) then K timed steps ----------
+    cfg = O.default_cfg()
+    tuner = O.Tuner(variants, cfg)
+    direction, ladder = tuner.ladder()
+    if is_stencil:
+        state["a"], state["b"] = t_a, t_b
+    step = 0
+    explore_ms = []
+    for _ in range(args.warmup):
+        r = tuner.step(step_args(step), sp)
+        if r.phase == 0:
+            explore_ms.append(r.ms)
+        step += 1
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    n_launch0 = O.launch_count()
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            tuner.step(step_args(step), sp)
+            step += 1
+        e1.record(stream)
+        torch.cuda.synchronize()
+    launches = O.launch_count() - n_launch0
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    total_ms = e0.elapsed_time(e1)
+    if world > 1:
+        t = torch.tensor([total_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    final, iters_to_final = tuner.final()
+    units_per_step = W * H
+    value = world * units_per_step * args.steps / (total_ms * 1e-3) / 1e6
+    ms_step = total_ms / args.steps
+    t_final = ms[final] if final >= 0 else float("nan")
+
+    # ---- end to end through the C ABI with pinned host buffers ---------------------------
+    e2e = None
+    if not is_stencil:
+        host_in = srcs[0].cpu().pin_memory()
+        host_out = torch.empty((H, W, 4)).pin_memory()
+        ha = O.denoise_args(kernel, host_in.data_ptr(), host_out.data_ptr(), W, H)
+        n_e2e = max(3, min(args.steps, 50))
+        tuner.step_host(ha, srcs[0].data_ptr(), dsts[0].data_ptr(), stream=sp)   # warm
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        hi = ho = 0
+        for _ in range(n_e2e):
+            _, hi, ho = tuner.step_host(ha, srcs[0].data_ptr(), dsts[0].data_ptr(), stream=sp)
+        dt = time.perf_counter() - t0
+        if world > 1:
+            t = torch.tensor([dt], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dt = float(t.item())
+        e2e = {"value": world * W * H * n_e2e / dt / 1e6, "unit": wl["unit"], "h2d_bytes_per_step": hi,
+               "d2h_bytes_per_step": ho, "steps": n_e2e}
+    else:
+        e2e = {"value": None, "unit": wl["unit"], "note": "stencil grid stays resident across its 100 iterations"}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    # ---- roofline of the dominant kernel ----------------------------------------------------
+    peaks, peak_kind = load_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    kernel_ms = ms_step  # one launch per steady-state step; the stream holds only our kernel
+    if is_stencil:
+        achieved = wl["bytes"] * units_per_step / (kernel_ms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "peak_kind": peak_kind + " (copy bandwidth)"}
+    else:
+        peak = 148 * 128 * sm_max * 1e6 / 1e12
+        achieved = wl["insts"] * units_per_step / (kernel_ms * 1e-3) / 1e12
+        roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tinst/s (FP32 pipe lane-ops)",
+                "frac": achieved / peak,
+                "peak_kind": f"derived: 148 SM x 128 FP32 lanes x {sm_max:.0f} MHz (sm_max_mhz, {peak_kind})",
+                "hbm_frac": wl["bytes"] * units_per_step / (kernel_ms * 1e-3) / 1e9 / peaks["hbm_gbs"]}
+    roof["traffic"] = None
+    prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if os.path.exists(prof):
+        try:
+            with open(prof) as f:
+                pj = json.load(f)
+            ent = pj.get(kernel) or {}
+            roof["traffic"] = ent.get("dram_bytes_per_launch")
+        except Exception:
+            pass
+    roof["kernel"] = kernel
+    roof["algorithmic_per_unit"] = wl["insts"] if not is_stencil else wl["bytes"]
+
+    # ---- CPU baseline (the oracle), rank 0, N=1 only ------------------------------------------
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        if is_stencil:
+            u, dt, sample = cpu_baseline_hotspot(W, 1, args.cpu_seconds)
+        else:
+            u, dt, sample = cpu_baseline_nlm("knn" if kernel.startswith("knn") else "nlm", W, H, wl["sigma"],
+                                             args.cpu_seconds)
+        cpu = {"value": u / dt / 1e6, "unit": wl["unit"], "cores": 1, "kind": "oracle", "sample": sample}
+
+    lvl_rows = [{"k": lv[i].ctas_per_sm, "occ": lv[i].occupancy_permille / 1000, "reg_cap": lv[i].reg_cap,
+                 "regs": infos[i].regs, "pad": lv[i].smem_pad_bytes, "spill_st": infos[i].spill_store,
+                 "ms": round(ms[i], 5)} for i in range(nlev)]
+    line = {
+        "metric": METRIC, "value": value, "unit": wl["unit"], "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": wl["name"], "kernel": kernel, "block_threads": res.block_threads,
+                   "width": W, "height": H, "frames_in_pool": nframes,
+                   "l2": "inputs larger than L2: rotating pool of frames" if not is_stencil else
+                         "grid 768 MiB > L2 (126 MB)",
+                   "parallelism": f"dp{world} (independent frames per GPU)"},
+        "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
+        "tuner": {"direction": "increasing" if direction == 1 else "decreasing", "ladder_k": [lv[i].ctas_per_sm
+                  for i in ladder], "final_k": lv[final].ctas_per_sm if final >= 0 else None,
+                  "final_occupancy": lv[final].occupancy_permille / 1000 if final >= 0 else None,
+                  "iterations_to_final": iters_to_final, "explore_ms": explore_ms},
+        "sweep": {"rounds": args.rounds, "levels": lvl_rows, "best_k": lv[best].ctas_per_sm, "ms_best": ms[best],
+                  "worst_k": lv[worst].ctas_per_sm, "ms_worst": ms[worst], "maxocc_k": lv[kmax].ctas_per_sm,
+                  "ms_maxocc": ms[kmax], "nvcc_default_k": lv[orig].ctas_per_sm, "ms_nvcc_default": ms[orig]},
+        "regret": t_final / ms[best] - 1.0,
+        "vs_maxocc": ms[kmax] / t_final,
+        "vs_nvcc_default": ms[orig] / t_final,
+        "build_seconds": round(t_build, 2),
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=300)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", choices=sorted(WORKLOADS), default="c2")
+    ap.add_argument("--rounds", type=int, default=11, help="interleaved rounds of the exhaustive sweep")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        ap.error("--warmup must be >= 3")
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

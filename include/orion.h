@@ -1,0 +1,250 @@
+/*
+ * orion.h -- the C ABI of liborion, the B200-native (sm_100a) occupancy-tuned hot
+ * path of "Orion: A Framework for GPU Occupancy Tuning" (Hayes et al., Middleware'16).
+ *
+ * Citations: P:L<n> = PAPER.md line n (section / figure / equation given beside it).
+ * The boundary follows the paper's two questions (§3, P:L133-P:L137 and P:L175):
+ *   (1) "how to generate the code given any occupancy level"
+ *         -> orion_levels + orion_build_variants (+ orion_launch to realise a level);
+ *   (2) "how to choose the best code version out of all the code versions"
+ *         -> orion_tuner_create + orion_tune_step (two-level selection, Fig. 3).
+ *
+ * Conventions (every function):
+ *   - Returns orion_status: ORION_OK (0) or a negative error code.  Errors are never
+ *     fatal; orion_last_error() returns a thread-local message (driver string, ptxas log).
+ *   - Ownership: the CALLER owns all image / grid buffers (device pointers, e.g. torch
+ *     tensors' data_ptr()) and the CUDA stream (a CUstream / cudaStream_t passed as
+ *     void*; NULL = the legacy default stream).  The LIBRARY owns compiled cubins,
+ *     CUmodules, CUDA events and tuner state; each has a create/destroy pair.
+ *   - No device allocation happens inside orion_launch / orion_tune_step.
+ *   - Handles are not thread-safe: use one per stream / rank.
+ *   - Every device entry point uses the CUDA primary context of the given device (the
+ *     same context PyTorch uses); host-only entry points never touch the GPU.
+ *   - Image layout: float4 RGBA (x,y,z,w = r,g,b,a) in [0,1], row-major, pitch = width
+ *     pixels; stencil grids: float32, row-major, pitch = width.
+ */
+#ifndef ORION_H
+#define ORION_H
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int orion_status;
+enum {
+    ORION_OK = 0,
+    ORION_E_INVALID = -1,             /* bad argument (NULL, out-of-range, unknown kernel id)      */
+    ORION_E_CAPACITY = -2,            /* output array too small; *n_out holds the size needed      */
+    ORION_E_INFEASIBLE = -3,          /* requested occupancy level cannot be realised               */
+    ORION_E_COMPILE = -4,             /* ptxas (nvPTXCompiler) failed; log in orion_last_error()   */
+    ORION_E_CUDA = -5,                /* CUDA driver error (or no driver / no GPU)                  */
+    ORION_E_OCCUPANCY_MISMATCH = -6,  /* realised CTAs/SM (driver occupancy API) != the level's k   */
+    ORION_E_STATE = -7                /* call not valid in the object's current state               */
+};
+
+/* Limiter bits of orion_level.limiter (which limits equal the realised CTA count). */
+enum { ORION_LIM_REGS = 1, ORION_LIM_SMEM = 2, ORION_LIM_WARPS = 4, ORION_LIM_BLOCKS = 8 };
+
+/* Device resource limits -- the inputs of Eq. (1) (P:L121-P:L127: Nreg, Nsmem, Smax) plus
+ * the allocation granularities the "NVIDIA occupancy calculator" [19] applies. */
+typedef struct {
+    int cc_major, cc_minor, sm_count, warp_size;
+    int regs_per_sm, regs_per_block, max_regs_per_thread, reg_alloc_unit, num_subpartitions;
+    int max_threads_per_sm, max_threads_per_block, max_blocks_per_sm;
+    int smem_per_sm, smem_per_block_optin, smem_reserved_per_block, smem_alloc_unit;
+} orion_device_limits;
+
+/* A kernel's resource usage at its natural ("original") build: Vreg and Vsmem of Eq. (1). */
+typedef struct {
+    int block_threads;      /* T, threads per CTA                                        */
+    int regs_per_thread;    /* natural (uncapped) ptxas register count = MAXLIVE proxy   */
+    int static_smem_bytes;  /* __shared__ arrays                                         */
+    int dyn_smem_bytes;     /* the kernel's own dynamic shared-memory need (its tile)    */
+    int min_reg_cap;        /* lowest register cap allowed (default 16)                  */
+} orion_kernel_resources;
+
+/* One occupancy level: k = ctas_per_sm resident CTAs per SM. */
+typedef struct {
+    int ctas_per_sm;         /* k                                                          */
+    int warps_per_sm;        /* k * ceil(T/32)                                             */
+    int occupancy_permille;  /* floor(1000 * warps / max warps per SM)                     */
+    int reg_cap;             /* ptxas --maxrregcount for this level; 0 = uncapped (natural) */
+    int smem_pad_bytes;      /* extra dynamic shared memory that caps residency at k */
+    int limiter;             /* ORION_LIM_* bits                                            */
+} orion_level;
+
+/* ---- occupancy levels (question 1; host-only, pure) -------------------------------------- */
+
+/* Nominal B200 (cc 10.0, 148 SMs) limits, for planning without a GPU. */
+orion_status orion_b200_limits(orion_device_limits *out);
+
+/* Limits of CUDA device `device`, read from the driver (cuDeviceGetAttribute). */
+orion_status orion_query_limits(int device, orion_device_limits *out);
+
+/* Eq. (1) evaluated with the calculator's granularities (P:L125-P:L127): CTAs/SM of a
+ * kernel with T threads, `regs` registers/thread, `smem_static` + `smem_dyn` bytes/CTA,
+ * and the shared-memory carveout pinned at the device maximum.  *limiter gets ORION_LIM_*
+ * bits (may be NULL). */
+orion_status orion_ctas_per_sm(const orion_device_limits *dev, int block_threads, int regs,
+                               int smem_static, int smem_dyn, int *ctas, int *limiter);
+
+/* All feasible occupancy levels k = 1..k_max of a kernel ("generate code at all
+ * occupancy levels"), ascending k.  Level k is realised by a register cap R_k (0 = natural
+ * if the natural count already admits k; else the largest multiple of 8 below it that
+ * admits k) and, where the registers admit more than k, dynamic shared-memory
+ * padding.  Pure function of its inputs.  Capacity protocol: capacity too small
+ * -> ORION_E_CAPACITY with *n_out = the number needed.  `out` may be NULL if capacity = 0. */
+orion_status orion_levels(const orion_device_limits *dev, const orion_kernel_resources *res,
+                          orion_level *out, int capacity, int *n_out);
+
+/* ---- code generation (question 1; host-only, no GPU needed) ------------------------------ */
+
+/* Kernel ids: "knn_f4", "nlm_f4", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32".
+ * block_threads = 0 selects the kernel's default CTA size.  Fills the natural resources
+ * (compiles the kernel's PTX once, uncapped, with the embedded ptxas). */
+orion_status orion_kernel_probe(const char *kernel_id, int block_threads, orion_kernel_resources *out);
+
+/* Compile the kernel at register cap `reg_cap` (0 = uncapped) and report what ptxas did:
+ * registers used, spill store / load bytes, local (stack) bytes per thread. */
+orion_status orion_compile_info(const char *kernel_id, int block_threads, int reg_cap, int *regs,
+                                int *spill_store_bytes, int *spill_load_bytes, int *local_bytes);
+
+/* ---- multi-version binary (question 1; device) -------------------------------------------- */
+
+typedef struct orion_variants orion_variants;   /* opaque, library-owned */
+
+/* Build one sm_100a variant per level (the paper's "multi-version binary"):
+ * the kernel's PTX is compiled once (at library build time) and assembled by ptxas once
+ * per distinct register cap; every variant is loaded on `device`, its padding recomputed
+ * from the ACTUAL register count, the carveout pinned when padding is used, and its
+ * realised CTAs/SM checked with cuOccupancyMaxActiveBlocksPerMultiprocessor
+ * (-> ORION_E_OCCUPANCY_MISMATCH).  Every variant is launched once (warm-up, defeats lazy
+ * loading) only when orion_launch is first called with it. */
+orion_status orion_build_variants(int device, const char *kernel_id, int block_threads,
+                                  const orion_level *levels, int n, orion_variants **out);
+orion_status orion_variants_count(const orion_variants *v, int *n);
+/* The realised level (pad recomputed from actual registers) of variant `level_idx`. */
+orion_status orion_variant_level(const orion_variants *v, int level_idx, orion_level *out);
+orion_status orion_variant_info(const orion_variants *v, int level_idx, int *regs, int *spill_store_bytes,
+                                int *spill_load_bytes, int *local_bytes, int *verified_ctas_per_sm);
+/* The kernel's natural resources (what orion_kernel_probe returned when building). */
+orion_status orion_variants_resources(const orion_variants *v, orion_kernel_resources *out);
+void orion_variants_destroy(orion_variants *v);
+
+/* ---- launching one iteration ------------------------------------------------------------ */
+
+/* One launch of the kernel = one application iteration.
+ *  denoisers: src = float4 rows [src_row_begin, src_row_end); dst = float4 rows
+ *             [dst_row_begin, ...); output rows [row_begin, row_end) are computed.  src must
+ *             hold every row the window + patch reach after clamping to [0, height) (halo:
+ *             3 rows KNN, 6 rows NLM).  fparam[0] = Noise (1/h^2), fparam[1] = lerpC,
+ *             fparam[2] = weight threshold, fparam[3] = lerp threshold (fraction of the 49
+ *             window taps), as in the SDK imageDenoising sample (reading R-O2).
+ *  hotspot:   src = T (float), aux = power (same rows as src), dst = T'; fparam[0..4] =
+ *             sdc (step/Cap), rx = 1/Rx, ry = 1/Ry, rz = 1/Rz, amb (reading R-O3/R-A15).
+ *             src must hold rows row_begin-1 .. row_end (clamped). */
+typedef struct {
+    const void *src;
+    void *dst;
+    const void *aux;
+    int width, height;
+    int row_begin, row_end;
+    int src_row_begin, src_row_end;
+    int dst_row_begin;
+    float fparam[8];
+} orion_args;
+
+/* Launch variant `level_idx` (realising its occupancy level) on `stream` (async). */
+orion_status orion_launch(orion_variants *v, int level_idx, const orion_args *a, void *stream);
+
+/* Exhaustive occupancy sweep (Fig. 11's Orion-Min / Orion-Max methodology, P:L747-P:L755):
+ * `rounds` rounds, each launching every level once in round-robin order (interleaving
+ * cancels clock drift), each launch timed with a CUDA event pair on `stream`; writes the
+ * median ms per level into ms_median[n levels].  Synchronises the stream. */
+orion_status orion_sweep(orion_variants *v, const orion_args *a, void *stream, int rounds, float *ms_median);
+
+/* ---- runtime adaptation (question 2) ------------------------------------------------------ */
+
+enum { ORION_DIR_DECREASING = -1, ORION_DIR_INCREASING = 1 };
+enum { ORION_SELECT_FASTEST = 0, ORION_SELECT_LOWEST_WITHIN_TOL = 1 };
+
+typedef struct {
+    int maxlive_threshold;        /* Fig. 8 line 01: MAXLIVE >= 32 -> increasing (P:L645-P:L647)   */
+    int samples_per_level;        /* timed launches per explored level (paper: 1)                  */
+    int select_mode;              /* ORION_SELECT_* (reading R-A4)                        */
+    int allow_direction_switch;   /* P:L689 fail-safe: switch direction if the original is final
+                                     (default 1, reading R-A12)                           */
+    float slowdown_tol;           /* Fig. 9 "Slowdown > .02?"                              */
+    float worse_eps;              /* Fig. 9 "Worse runtime?" margin (paper: 0)                      */
+    int expected_iterations;      /* canTune (Fig. 8 line 05): 0 = unknown (assume enough)          */
+} orion_tuner_cfg;
+
+orion_status orion_tuner_default_cfg(orion_tuner_cfg *cfg);
+
+typedef struct orion_tuner orion_tuner;   /* opaque, library-owned (holds CUDA events) */
+
+/* Fig. 8 (P:L589-P:L603) applied to the variants' levels: direction from MAXLIVE (the
+ * natural register count), ladder = original + conservative..max (increasing) or
+ * original, original-1, .. 1 by padding (decreasing), with the opposite direction kept
+ * as the fail-safe. */
+orion_status orion_tuner_create(orion_variants *v, const orion_tuner_cfg *cfg, orion_tuner **out);
+
+typedef struct {
+    int iteration;        /* 0-based iteration index                                        */
+    int level_idx;        /* variant launched this iteration                                 */
+    int phase;            /* 0 = exploring (timed, synchronised), 1 = final (no host sync)   */
+    int final_level_idx;  /* -1 until the final kernel is set                                */
+    float ms;             /* measured kernel ms while exploring, else -1                     */
+} orion_step_report;
+
+/* One application iteration under Fig. 9 (P:L605-P:L643, P:L651-P:L653, P:L687-P:L689):
+ * first iteration runs the original; then the next ladder level while runtimes do not
+ * degrade ("Worse runtime?" when increasing, "Slowdown > .02?" vs the best when
+ * decreasing); then the final kernel every iteration.  Exploration iterations record a
+ * CUDA event pair and synchronise on it; final iterations only enqueue the launch. */
+orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, orion_step_report *out);
+
+/* Same iteration end to end from HOST buffers: copies a->src (host, pinned for async)
+ * into dev_src, runs orion_tune_step with device pointers, copies dev_dst back into
+ * a->dst (host) -- all on `stream`, then synchronises it.  dev_src / dev_dst are
+ * caller-owned device buffers at least as large as the host regions (and dev_aux for the
+ * stencil power map).  Byte counts copied are returned in *h2d_bytes / *d2h_bytes. */
+orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev_src, void *dev_dst,
+                                  void *dev_aux, void *stream, orion_step_report *out,
+                                  long long *h2d_bytes, long long *d2h_bytes);
+
+/* Current ladder: *direction, ladder level indices (ladder[0] = original) -> out[]. */
+orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, int capacity, int *n_out);
+orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final);
+void orion_tuner_destroy(orion_tuner *t);
+
+/* Host-only replay of Fig. 8 + Fig. 9 on a synthetic per-level runtime table (no GPU):
+ * levels[n] as from orion_levels, natural_regs = MAXLIVE proxy, ms_of_level[n] = the runtime
+ * each level would take; runs `iterations` iterations writing the level index run at each
+ * into ran[iterations], and the final level / the iteration it was set at. */
+orion_status orion_tuner_replay(const orion_tuner_cfg *cfg, const orion_level *levels, int n, int natural_regs,
+                                const float *ms_of_level, int iterations, int *ran, int *final_level_idx,
+                                int *final_iteration);
+
+/* ---- synthetic inputs on the device (the generator's GPU twin; no method arithmetic) ---- */
+
+/* Rows [row_begin, row_end) of the W x H seeded noisy RGBA image into dst (pitch W). */
+orion_status orion_generate_rgba(int device, void *dst, int width, int height, int row_begin, int row_end,
+                                 unsigned seed, float sigma, void *stream);
+/* Thermal T0 and power map (W x H) into t0 / power. */
+orion_status orion_generate_thermal(int device, void *t0, void *power, int width, int height, unsigned seed,
+                                    void *stream);
+/* Write `bytes` of `buf` (a device scratch buffer larger than L2) to evict the L2. */
+orion_status orion_flush_l2(int device, void *buf, long long bytes, void *stream);
+
+/* ---- diagnostics -------------------------------------------------------------------------- */
+const char *orion_status_str(orion_status s);
+const char *orion_last_error(void);
+/* Number of kernel launches liborion has enqueued in this process (all kernels). */
+long long orion_launch_count(void);
+const char *orion_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ORION_H */

@@ -1,0 +1,61 @@
+// common.cuh -- helpers shared by the Orion sm_100a kernels (product code).
+//
+// Every kernel is compiled ONCE to PTX (nvcc -arch=compute_100a -fmad=false) and
+// then assembled by liborion once per register cap (orion_build_variants), so the
+// value path must not depend on ptxas' register allocation: all floating-point
+// arithmetic is explicit (.rn mul/add/fma, no contraction freedom) and therefore
+// bit-identical across every occupancy variant (SURVEY §7 hard part 2).
+#pragma once
+#include <stdint.h>
+#include "../orion_kargs.h"
+
+#define ORION_DEVICE __device__ __forceinline__
+
+ORION_DEVICE int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
+
+// Squared RGB distance, |a - b|^2 with a fixed operation order.
+ORION_DEVICE float dist2(float4 a, float4 b)
+{
+    float dx = __fsub_rn(a.x, b.x), dy = __fsub_rn(a.y, b.y), dz = __fsub_rn(a.z, b.z);
+    return __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));
+}
+
+// Cooperative, coalesced load of a TW x TH float4 tile whose top-left corner is
+// global pixel (gx0, gy0), with clamp-to-edge addressing in GLOBAL coordinates
+// (so a row-sharded launch reads exactly what the full-image launch reads).
+template <int TW, int TH, int NT>
+ORION_DEVICE void load_tile_clamped(float4 *tile, const orion_kargs &a, int gx0, int gy0)
+{
+    const float4 *src = (const float4 *)a.src;
+    const int W = a.width, H = a.height;
+    const int tid = threadIdx.y * blockDim.x + threadIdx.x;
+    for (int idx = tid; idx < TW * TH; idx += NT) {
+        int ty = idx / TW;
+        int tx = idx - ty * TW;
+        int gx = clampi(gx0 + tx, 0, W - 1);
+        int gy = clampi(gy0 + ty, 0, H - 1);
+        tile[idx] = __ldg(src + (size_t)(gy - a.src_row_begin) * (size_t)W + gx);
+    }
+}
+
+// Final SDK imageDenoising blend: clr = acc/sw; out = clr + (c00 - clr) * q.
+ORION_DEVICE float4 lerp_out(float4 c00, float ax, float ay, float az, float sw, int cnt,
+                             const orion_kargs &a)
+{
+    const float lerpc = a.fparam[1];
+    const float q = (cnt >= a.iparam0) ? lerpc : __fsub_rn(1.0f, lerpc);
+    float cx = __fdiv_rn(ax, sw), cy = __fdiv_rn(ay, sw), cz = __fdiv_rn(az, sw);
+    float4 o;
+    o.x = __fmaf_rn(__fsub_rn(c00.x, cx), q, cx);
+    o.y = __fmaf_rn(__fsub_rn(c00.y, cy), q, cy);
+    o.z = __fmaf_rn(__fsub_rn(c00.z, cz), q, cz);
+    o.w = 0.0f;
+    return o;
+}
+
+
+// Same term evaluated at run time: (i*i + j*j) * (-log2(e)/49) with one rounding.
+ORION_DEVICE float geo_l2_rt(int i, int j)
+{
+    return __fmul_rn((float)(i * i + j * j), (float)(-1.4426950408889634 / 49.0));
+}

@@ -1,0 +1,66 @@
+// nlm_direct.cuh -- shared body of the direct-form NLM kernels (see nlm_direct.cu).
+#pragma once
+#include "common.cuh"
+
+#define NLM_R 3
+#define NLM_B 3
+#define NLM_H (NLM_R + NLM_B)
+#define NLM_A 49
+
+template <int BX, int BY, bool REGHEAVY>
+__device__ __forceinline__ void nlm_direct_body(const orion_kargs &a)
+{
+    constexpr int TW = BX + 2 * NLM_H;
+    constexpr int TH = BY + 2 * NLM_H;
+    extern __shared__ float4 tile[];
+    const int x0 = blockIdx.x * BX;
+    const int y0 = a.row_begin + blockIdx.y * BY;
+    load_tile_clamped<TW, TH, BX * BY>(tile, a, x0 - NLM_H, y0 - NLM_H);
+    __syncthreads();
+
+    const int tx = threadIdx.x + NLM_H, ty = threadIdx.y + NLM_H;   // centre in tile coords
+    const float nl2 = a.fparam[0];
+    const float wthr = a.fparam[2];
+    const float4 c00 = tile[ty * TW + tx];
+
+    float4 cp[REGHEAVY ? 2 * NLM_B + 1 : 1][REGHEAVY ? 2 * NLM_B + 1 : 1];
+    if (REGHEAVY) {
+#pragma unroll
+        for (int n = 0; n < 2 * NLM_B + 1; ++n)
+#pragma unroll
+            for (int m = 0; m < 2 * NLM_B + 1; ++m)
+                cp[REGHEAVY ? n : 0][REGHEAVY ? m : 0] = tile[(ty + n - NLM_B) * TW + tx + m - NLM_B];
+    }
+
+    float ax = 0.f, ay = 0.f, az = 0.f, sw = 0.f;
+    int cnt = 0;
+#pragma unroll 1
+    for (int i = -NLM_R; i <= NLM_R; ++i) {
+#pragma unroll (REGHEAVY ? 7 : 1)
+        for (int j = -NLM_R; j <= NLM_R; ++j) {
+            float d = 0.0f;
+#pragma unroll
+            for (int n = -NLM_B; n <= NLM_B; ++n) {
+#pragma unroll
+                for (int m = -NLM_B; m <= NLM_B; ++m) {
+                    const float4 s = tile[(ty + i + n) * TW + tx + j + m];
+                    const float4 c = REGHEAVY ? cp[REGHEAVY ? n + NLM_B : 0][REGHEAVY ? m + NLM_B : 0]
+                                              : tile[(ty + n) * TW + tx + m];
+                    d = __fadd_rn(d, dist2(s, c));
+                }
+            }
+            const float w = exp2f(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
+            const float4 cij = tile[(ty + i) * TW + tx + j];
+            ax = __fmaf_rn(w, cij.x, ax);
+            ay = __fmaf_rn(w, cij.y, ay);
+            az = __fmaf_rn(w, cij.z, az);
+            sw = __fadd_rn(sw, w);
+            cnt += (w > wthr);
+        }
+    }
+    const int x = x0 + threadIdx.x, y = y0 + threadIdx.y;
+    if (x < a.width && y < a.row_end)
+        ((float4 *)a.dst)[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] =
+            lerp_out(c00, ax, ay, az, sw, cnt, a);
+}
+

@@ -1,0 +1,19 @@
+/* orion_kargs.h -- the by-value parameter block every Orion kernel receives.
+ * Shared by the host launcher (g++) and the kernels (nvcc -> PTX); product-internal.
+ * Layout must stay identical on both sides (plain 4/8-byte fields, no padding surprises). */
+#ifndef ORION_KARGS_H
+#define ORION_KARGS_H
+
+typedef struct {
+    const void *src;      /* rows [src_row_begin, src_row_end) of a width-wide image, pitch = width */
+    void *dst;            /* rows [dst_row_begin, ...), pitch = width                               */
+    const void *aux;      /* stencil power map (same rows as src); NULL for the denoisers            */
+    int width, height;    /* global image size                                                      */
+    int row_begin, row_end;          /* output rows computed by this launch (global)                */
+    int src_row_begin, src_row_end;  /* rows held by src (global)                                   */
+    int dst_row_begin;               /* global row of dst's first row                               */
+    int iparam0;                     /* denoise: lerp count threshold (cnt >= iparam0 -> lerpC)     */
+    float fparam[8];                 /* denoise: -Noise*log2e, lerpC, wthr ; stencil: sdc,rx,ry,rz,amb */
+} orion_kargs;
+
+#endif

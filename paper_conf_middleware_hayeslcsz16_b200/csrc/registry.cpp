@@ -1,0 +1,230 @@
+// registry.cpp -- the kernel families liborion knows, and their code generation.
+//
+// The paper's compiler realises an occupancy level by re-allocating registers in SASS
+// (P:L213-P:L229, P:L697-P:L707).  On sm_100a ptxas owns register allocation, so a
+// level's register budget is realised the way NVIDIA's toolchain exposes it: each
+// kernel is compiled ONCE to PTX when the library is built (nvcc -arch=compute_100a
+// -fmad=false; the PTX is embedded in liborion.so), and `orion_build_variants`
+// assembles that PTX to an sm_100a cubin once per distinct register cap with the
+// embedded ptxas (nvPTXCompiler, --maxrregcount=R).  One PTX + explicit .rn arithmetic
+// => every variant computes bit-identical results; only resources differ.
+#include <nvPTXCompiler.h>
+
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <sstream>
+
+#include "orion_internal.h"
+
+// Generated at build time (build.py): the PTX of every kernel family, NUL-terminated.
+extern "C" const char liborion_ptx_knn[];
+extern "C" const char liborion_ptx_nlm_box[];
+extern "C" const char liborion_ptx_nlm_direct[];
+extern "C" const char liborion_ptx_nlm_regheavy[];
+extern "C" const char liborion_ptx_hotspot[];
+extern "C" const char liborion_ptx_gen[];
+
+namespace orion {
+
+static const char *module_ptx(const char *module)
+{
+    if (!std::strcmp(module, "knn")) return liborion_ptx_knn;
+    if (!std::strcmp(module, "nlm_box")) return liborion_ptx_nlm_box;
+    if (!std::strcmp(module, "nlm_direct")) return liborion_ptx_nlm_direct;
+    if (!std::strcmp(module, "nlm_regheavy")) return liborion_ptx_nlm_regheavy;
+    if (!std::strcmp(module, "hotspot")) return liborion_ptx_hotspot;
+    if (!std::strcmp(module, "gen")) return liborion_ptx_gen;
+    return nullptr;
+}
+
+// id, T, entry, module, bx, by, tile_w, tile_h, halo, kind, smem_tile, smem_bytes.  The first row of
+// each id is its default CTA size.
+static const KernelDef kKernels[] = {
+    {"knn_f4", 128, "orion_knn_f4_128", "knn", 32, 4, 32, 16, 3, K_KNN, 1, 0},
+    {"knn_f4", 256, "orion_knn_f4_256", "knn", 32, 8, 32, 32, 3, K_KNN, 1, 0},
+    {"knn_f4", 64, "orion_knn_f4_64", "knn", 8, 8, 8, 32, 3, K_KNN, 1, 0},
+    // nlm_box: 3 planar (120+12) x (16+12) fp32 planes + 16 x 128 floats of vertical sums
+    {"nlm_f4", 128, "orion_nlm_box_f4_128", "nlm_box", 128, 1, 120, 16, 6, K_NLM, 0,
+     3 * 132 * 28 * 4 + 16 * 128 * 4},
+    {"nlm_f4_direct", 128, "orion_nlm_direct_f4_128", "nlm_direct", 32, 4, 32, 4, 6, K_NLM, 1, 0},
+    {"nlm_f4_regheavy", 128, "orion_nlm_regheavy_f4_128", "nlm_regheavy", 32, 4, 32, 4, 6, K_NLM, 1, 0},
+    {"nlm_f4_regheavy", 64, "orion_nlm_regheavy_f4_64", "nlm_regheavy", 8, 8, 8, 8, 6, K_NLM, 1, 0},
+    {"hotspot_f32", 256, "orion_hotspot_f32_256", "hotspot", 32, 8, 32, 128, 1, K_STENCIL, 0, 0},
+    {"hotspot_f32", 128, "orion_hotspot_f32_128", "hotspot", 32, 4, 32, 64, 1, K_STENCIL, 0, 0},
+};
+
+const KernelDef *find_kernel(const char *id, int threads)
+{
+    if (!id) return nullptr;
+    for (const KernelDef &k : kKernels)
+        if (!std::strcmp(k.id, id) && (threads == 0 || threads == k.threads)) return &k;
+    return nullptr;
+}
+
+static void parse_ptxas_log(const std::string &log, CompiledVariant &cv)
+{
+    std::istringstream in(log);
+    std::string line;
+    while (std::getline(in, line)) {
+        int a, b, c;
+        const char *p;
+        if ((p = std::strstr(line.c_str(), "bytes stack frame")) != nullptr) {
+            if (std::sscanf(line.c_str() + line.find_first_of("0123456789"),
+                            "%d bytes stack frame, %d bytes spill stores, %d bytes spill loads", &a, &b, &c) == 3) {
+                cv.stack_bytes = a;
+                cv.spill_store = b;
+                cv.spill_load = c;
+            }
+        }
+        if ((p = std::strstr(line.c_str(), "Used ")) != nullptr) {
+            if (std::sscanf(p, "Used %d registers", &a) == 1) cv.regs = a;
+            const char *s = std::strstr(p, "bytes smem");
+            if (s) {
+                const char *q = s;
+                while (q > p && q[-1] == ' ') --q;
+                while (q > p && q[-1] >= '0' && q[-1] <= '9') --q;
+                cv.static_smem = std::atoi(q);
+            }
+        }
+    }
+}
+
+orion_status compile_variant(const KernelDef &def, int cap, std::shared_ptr<const CompiledVariant> *out)
+{
+    static std::mutex mu;
+    static std::map<std::pair<std::string, int>, std::shared_ptr<const CompiledVariant>> cache;
+    const auto key = std::make_pair(std::string(def.entry), cap);
+    {
+        std::lock_guard<std::mutex> g(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) {
+            *out = it->second;
+            return ORION_OK;
+        }
+    }
+    const char *ptx0 = module_ptx(def.module);
+    if (!ptx0) return fail(ORION_E_INVALID, std::string("no PTX module ") + def.module);
+    // The register budget of a level is a per-entry PTX performance directive: `.maxnreg R`
+    // is inserted after the entry's `.maxntid` (its __launch_bounds__, which would make
+    // ptxas ignore a global --maxrregcount).  Everything else in the PTX is untouched.
+    std::string ptx(ptx0);
+    if (cap > 0) {
+        const std::string ent = std::string(".entry ") + def.entry + "(";
+        size_t at = ptx.find(ent);
+        size_t mt = at == std::string::npos ? at : ptx.find(".maxntid", at);
+        size_t body = at == std::string::npos ? at : ptx.find("\n{", at);
+        if (mt == std::string::npos || body == std::string::npos || mt > body)
+            return fail(ORION_E_COMPILE, std::string("no .maxntid directive for ") + def.entry);
+        size_t eol = ptx.find('\n', mt);
+        ptx.insert(eol + 1, ".maxnreg " + std::to_string(cap) + "\n");
+    }
+    nvPTXCompilerHandle h = nullptr;
+    if (nvPTXCompilerCreate(&h, ptx.size(), ptx.c_str()) != NVPTXCOMPILE_SUCCESS)
+        return fail(ORION_E_COMPILE, "nvPTXCompilerCreate failed");
+    std::string entry = std::string("--entry=") + def.entry;
+    std::vector<const char *> opts = {"--gpu-name=sm_100a", "--verbose", "-O3", "--generate-line-info",
+                                      entry.c_str()};
+    nvPTXCompileResult r = nvPTXCompilerCompile(h, (int)opts.size(), opts.data());
+    auto cv = std::make_shared<CompiledVariant>();
+    size_t n = 0;
+    if (nvPTXCompilerGetInfoLogSize(h, &n) == NVPTXCOMPILE_SUCCESS && n) {
+        cv->log.resize(n);
+        nvPTXCompilerGetInfoLog(h, &cv->log[0]);
+    }
+    if (r != NVPTXCOMPILE_SUCCESS) {
+        std::string err;
+        if (nvPTXCompilerGetErrorLogSize(h, &n) == NVPTXCOMPILE_SUCCESS && n) {
+            err.resize(n);
+            nvPTXCompilerGetErrorLog(h, &err[0]);
+        }
+        nvPTXCompilerDestroy(&h);
+        return fail(ORION_E_COMPILE, std::string("ptxas failed for ") + def.entry + " cap " + std::to_string(cap) +
+                                         ": " + err);
+    }
+    if (nvPTXCompilerGetCompiledProgramSize(h, &n) != NVPTXCOMPILE_SUCCESS) {
+        nvPTXCompilerDestroy(&h);
+        return fail(ORION_E_COMPILE, "nvPTXCompilerGetCompiledProgramSize failed");
+    }
+    cv->cubin.resize(n);
+    nvPTXCompilerGetCompiledProgram(h, cv->cubin.data());
+    nvPTXCompilerDestroy(&h);
+    parse_ptxas_log(cv->log, *cv);
+    std::lock_guard<std::mutex> g(mu);
+    auto &slot = cache[key];
+    if (!slot) slot = cv;
+    *out = slot;
+    return ORION_OK;
+}
+
+orion_status load_aux_module(int device, const char *module, CUmodule *out)
+{
+    static std::mutex mu;
+    static std::map<std::pair<int, std::string>, CUmodule> mods;
+    ORION_TRY(ensure_context(device));
+    std::lock_guard<std::mutex> g(mu);
+    auto key = std::make_pair(device, std::string(module));
+    auto it = mods.find(key);
+    if (it != mods.end()) {
+        *out = it->second;
+        return ORION_OK;
+    }
+    const char *ptx = module_ptx(module);
+    if (!ptx) return fail(ORION_E_INVALID, std::string("no PTX module ") + module);
+    nvPTXCompilerHandle h = nullptr;
+    if (nvPTXCompilerCreate(&h, std::strlen(ptx), ptx) != NVPTXCOMPILE_SUCCESS)
+        return fail(ORION_E_COMPILE, "nvPTXCompilerCreate failed");
+    const char *opts[] = {"--gpu-name=sm_100a", "-O3"};
+    if (nvPTXCompilerCompile(h, 2, opts) != NVPTXCOMPILE_SUCCESS) {
+        nvPTXCompilerDestroy(&h);
+        return fail(ORION_E_COMPILE, std::string("ptxas failed for module ") + module);
+    }
+    size_t n = 0;
+    nvPTXCompilerGetCompiledProgramSize(h, &n);
+    std::vector<char> cubin(n);
+    nvPTXCompilerGetCompiledProgram(h, cubin.data());
+    nvPTXCompilerDestroy(&h);
+    CUmodule m;
+    ORION_CU(drv().cuModuleLoadData(&m, cubin.data()));
+    mods[key] = m;
+    *out = m;
+    return ORION_OK;
+}
+
+}  // namespace orion
+
+using namespace orion;
+
+extern "C" {
+
+orion_status orion_kernel_probe(const char *kernel_id, int block_threads, orion_kernel_resources *out)
+{
+    if (!out) return fail(ORION_E_INVALID, "orion_kernel_probe: NULL");
+    const KernelDef *def = find_kernel(kernel_id, block_threads);
+    if (!def) return fail(ORION_E_INVALID, std::string("unknown kernel ") + (kernel_id ? kernel_id : "(null)"));
+    std::shared_ptr<const CompiledVariant> cv;
+    ORION_TRY(compile_variant(*def, 0, &cv));
+    out->block_threads = def->threads;
+    out->regs_per_thread = cv->regs;
+    out->static_smem_bytes = cv->static_smem;
+    out->dyn_smem_bytes = def->dyn_need();
+    out->min_reg_cap = 16;
+    return ORION_OK;
+}
+
+orion_status orion_compile_info(const char *kernel_id, int block_threads, int reg_cap, int *regs, int *spill_st,
+                                int *spill_ld, int *local_bytes)
+{
+    const KernelDef *def = find_kernel(kernel_id, block_threads);
+    if (!def || reg_cap < 0 || reg_cap > 255) return fail(ORION_E_INVALID, "orion_compile_info: bad argument");
+    std::shared_ptr<const CompiledVariant> cv;
+    ORION_TRY(compile_variant(*def, reg_cap, &cv));
+    if (regs) *regs = cv->regs;
+    if (spill_st) *spill_st = cv->spill_store;
+    if (spill_ld) *spill_ld = cv->spill_load;
+    if (local_bytes) *local_bytes = cv->stack_bytes;
+    return ORION_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,328 @@
+// tuner.cpp -- Orion's two-level selection (Fig. 3):
+//   level 1, compile time: Fig. 8's occupancy update algorithm prunes the levels to a
+//            candidate ladder (P:L583-P:L603, P:L645-P:L649);
+//   level 2, run time:     Fig. 9's dynamic occupancy selection walks that ladder across
+//            the application's iterations and settles on a final kernel (P:L605-P:L643,
+//            P:L651-P:L653, P:L687-P:L689).
+//
+// Readings: MAXLIVE = the natural register count (R-A5); conservative = the
+// first register-cap rung above the original (R-A6); canTune = iterations >= |ladder|+2
+// (R-A7); "Slowdown > .02" is measured against the best so far (R-A3); the final kernel
+// is the fastest measured (ties -> lower occupancy, Principle 2 P:L181-P:L183) or, in
+// LOWEST_WITHIN_TOL mode, the lowest occupancy within slowdown_tol of the best (R-A4).
+#include <algorithm>
+#include <map>
+
+#include "orion_internal.h"
+
+using namespace orion;
+
+namespace {
+
+struct Fig9 {
+    orion_tuner_cfg cfg{};
+    std::vector<int> ks;        // CTAs/SM of every level (index = level idx)
+    int direction = ORION_DIR_INCREASING;
+    std::vector<int> ladder, other;
+    int cur = -1;               // ladder position last run (-1: nothing run yet)
+    float best = 0.0f;
+    int final_idx = -1, final_iter = -1;
+    bool switched = false;
+    int iter = 0;
+    std::map<int, float> tried; // level idx -> measured ms
+
+    // Fig. 8 (canTune branch): ladders from the level list and MAXLIVE.
+    void prune(const orion_level *lv, int n, int natural_regs)
+    {
+        ks.resize(n);
+        int orig = -1;
+        for (int i = 0; i < n; ++i) {
+            ks[i] = lv[i].ctas_per_sm;
+            if (lv[i].reg_cap == 0 && lv[i].smem_pad_bytes == 0) orig = i;
+        }
+        const int k0 = ks[orig];
+        std::vector<int> up, down;
+        for (int i = 0; i < n; ++i) {
+            if (lv[i].smem_pad_bytes == 0 && ks[i] > k0) up.push_back(i);   // register-cap rungs
+            if (ks[i] < k0) down.push_back(i);                              // padding levels
+        }
+        std::sort(up.begin(), up.end(), [&](int a, int b) { return ks[a] < ks[b]; });
+        std::sort(down.begin(), down.end(), [&](int a, int b) { return ks[a] > ks[b]; });
+        up.insert(up.begin(), orig);
+        down.insert(down.begin(), orig);
+        if (natural_regs >= cfg.maxlive_threshold) {       // Fig. 8 lines 01-02, 07-09
+            direction = ORION_DIR_INCREASING;
+            ladder = up;
+            other = down;                                   // fail-safe: pad down
+        } else {                                            // lines 03-04, 10-11
+            direction = ORION_DIR_DECREASING;
+            ladder = down;
+            other.assign(up.begin(), up.begin() + std::min<size_t>(2, up.size()));   // original + conservative
+        }
+        if (cfg.expected_iterations > 0 && cfg.expected_iterations < (int)ladder.size() + 2) {
+            final_idx = ladder[0];                          // !canTune: the safe original
+            final_iter = 0;
+        }
+    }
+
+    int select() const
+    {
+        float b = tried.begin()->second;
+        for (auto &kv : tried) b = std::min(b, kv.second);
+        int pick = -1;
+        for (auto &kv : tried) {
+            const int i = kv.first;
+            const float t = kv.second;
+            if (cfg.select_mode == ORION_SELECT_FASTEST) {
+                if (pick < 0 || t < tried.at(pick) || (t == tried.at(pick) && ks[i] < ks[pick])) pick = i;
+            } else if (t <= b * (1.0f + cfg.slowdown_tol)) {
+                if (pick < 0 || ks[i] < ks[pick] || (ks[i] == ks[pick] && t < tried.at(pick))) pick = i;
+            }
+        }
+        return pick;
+    }
+
+    // "Set final kernel" -- or, with the P:L689 augmentation, switch direction once when
+    // the original would be final.  Returns true if the final kernel is now set.
+    bool set_final()
+    {
+        const int f = select();
+        if (cfg.allow_direction_switch && !switched && f == ladder[0] && other.size() > 1) {
+            switched = true;
+            direction = -direction;
+            std::swap(ladder, other);
+            cur = 0;
+            return false;
+        }
+        final_idx = f;
+        final_iter = iter;
+        return true;
+    }
+
+    // Which level runs this iteration, and whether its time must be measured.
+    int choose(bool *measure)
+    {
+        *measure = false;
+        if (final_idx >= 0) return final_idx;                      // "Final kernel has been set?"
+        if (cur < 0) {                                             // "First iteration?"
+            *measure = true;
+            return ladder[0];
+        }
+        if (cur == (int)ladder.size() - 1 && set_final()) return final_idx;   // tried every occ
+        *measure = true;
+        return ladder[cur + 1];                                    // "Run next kernel"
+    }
+
+    // Feed back the measured time of the level chosen with measure = true.
+    void observe(int lvl, float ms)
+    {
+        if (cur < 0) {
+            tried[lvl] = ms;
+            best = ms;
+            cur = 0;
+            return;
+        }
+        const float prev = tried.at(ladder[cur]);
+        ++cur;
+        tried[lvl] = ms;
+        const bool stop = (direction == ORION_DIR_INCREASING) ? ms > prev * (1.0f + cfg.worse_eps)      // "Worse runtime?"
+                                                              : ms > best * (1.0f + cfg.slowdown_tol);  // "Slowdown > .02?"
+        best = std::min(best, ms);
+        if (stop) set_final();
+    }
+};
+
+orion_status check_cfg(const orion_tuner_cfg *c)
+{
+    if (!c || c->samples_per_level < 1 || c->slowdown_tol < 0.0f || c->worse_eps < 0.0f ||
+        (c->select_mode != ORION_SELECT_FASTEST && c->select_mode != ORION_SELECT_LOWEST_WITHIN_TOL))
+        return fail(ORION_E_INVALID, "bad tuner cfg");
+    return ORION_OK;
+}
+
+orion_status check_levels(const orion_level *lv, int n)
+{
+    if (!lv || n <= 0) return fail(ORION_E_INVALID, "no levels");
+    for (int i = 0; i < n; ++i)
+        if (lv[i].reg_cap == 0 && lv[i].smem_pad_bytes == 0) return ORION_OK;
+    return fail(ORION_E_INVALID, "levels lack the original (uncapped, unpadded) version");
+}
+
+}  // namespace
+
+struct orion_tuner {
+    orion_variants *v = nullptr;
+    Fig9 f;
+    CUevent e0 = nullptr, e1 = nullptr;
+    int pending_level = -1;      // level being sampled (samples_per_level > 1)
+    int samples = 0;
+    float sample_best = 0.0f;
+};
+
+extern "C" {
+
+orion_status orion_tuner_default_cfg(orion_tuner_cfg *c)
+{
+    if (!c) return fail(ORION_E_INVALID, "NULL cfg");
+    c->maxlive_threshold = 32;
+    c->samples_per_level = 1;
+    c->select_mode = ORION_SELECT_FASTEST;
+    c->allow_direction_switch = 1;   // P:L689 augmentation on by default (reading R-A12)
+    c->slowdown_tol = 0.02f;
+    c->worse_eps = 0.0f;
+    c->expected_iterations = 0;
+    return ORION_OK;
+}
+
+orion_status orion_tuner_replay(const orion_tuner_cfg *cfg, const orion_level *levels, int n, int natural_regs,
+                                const float *ms_of_level, int iterations, int *ran, int *final_level_idx,
+                                int *final_iteration)
+{
+    ORION_TRY(check_cfg(cfg));
+    ORION_TRY(check_levels(levels, n));
+    if (!ms_of_level || iterations < 0 || (iterations > 0 && !ran)) return fail(ORION_E_INVALID, "replay: bad argument");
+    Fig9 f;
+    f.cfg = *cfg;
+    f.prune(levels, n, natural_regs);
+    for (int it = 0; it < iterations; ++it) {
+        f.iter = it;
+        bool measure;
+        const int lvl = f.choose(&measure);
+        if (measure) f.observe(lvl, ms_of_level[lvl]);
+        ran[it] = lvl;
+    }
+    if (final_level_idx) *final_level_idx = f.final_idx;
+    if (final_iteration) *final_iteration = f.final_iter;
+    return ORION_OK;
+}
+
+orion_status orion_tuner_create(orion_variants *v, const orion_tuner_cfg *cfg, orion_tuner **out)
+{
+    if (!v || !out) return fail(ORION_E_INVALID, "orion_tuner_create: NULL");
+    ORION_TRY(check_cfg(cfg));
+    std::vector<orion_level> lv(v->vars.size());
+    for (size_t i = 0; i < lv.size(); ++i) lv[i] = v->vars[i].planned;
+    ORION_TRY(check_levels(lv.data(), (int)lv.size()));
+    ORION_TRY(ensure_context(v->device));
+    auto t = new orion_tuner();
+    t->v = v;
+    t->f.cfg = *cfg;
+    t->f.prune(lv.data(), (int)lv.size(), v->res.regs_per_thread);
+    const Driver &D = drv();
+    if (D.cuEventCreate(&t->e0, CU_EVENT_DEFAULT) != CUDA_SUCCESS ||
+        D.cuEventCreate(&t->e1, CU_EVENT_DEFAULT) != CUDA_SUCCESS) {
+        orion_tuner_destroy(t);
+        return fail(ORION_E_CUDA, "cuEventCreate");
+    }
+    *out = t;
+    return ORION_OK;
+}
+
+void orion_tuner_destroy(orion_tuner *t)
+{
+    if (!t) return;
+    if (drv().ok) {
+        if (t->e0) drv().cuEventDestroy(t->e0);
+        if (t->e1) drv().cuEventDestroy(t->e1);
+    }
+    delete t;
+}
+
+orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, orion_step_report *out)
+{
+    if (!t || !a) return fail(ORION_E_INVALID, "orion_tune_step: NULL");
+    Fig9 &f = t->f;
+    bool measure = false;
+    int lvl;
+    if (t->pending_level >= 0) {          // still sampling a level (samples_per_level > 1)
+        lvl = t->pending_level;
+        measure = true;
+    } else {
+        lvl = f.choose(&measure);
+    }
+    CUstream s = (CUstream)stream;
+    const Driver &D = drv();
+    float ms = -1.0f;
+    if (measure) {
+        ORION_CU(D.cuEventRecord(t->e0, s));
+        ORION_TRY(orion_launch(t->v, lvl, a, stream));
+        ORION_CU(D.cuEventRecord(t->e1, s));
+        ORION_CU(D.cuEventSynchronize(t->e1));
+        ORION_CU(D.cuEventElapsedTime(&ms, t->e0, t->e1));
+        const float m = (t->samples == 0) ? ms : std::min(t->sample_best, ms);
+        t->samples += 1;
+        t->sample_best = m;
+        if (t->samples >= f.cfg.samples_per_level) {
+            f.observe(lvl, m);            // best of the samples feeds Fig. 9
+            t->pending_level = -1;
+            t->samples = 0;
+        } else {
+            t->pending_level = lvl;
+        }
+    } else {
+        ORION_TRY(orion_launch(t->v, lvl, a, stream));
+    }
+    if (out) {
+        out->iteration = f.iter;
+        out->level_idx = lvl;
+        out->phase = measure ? 0 : 1;
+        out->final_level_idx = f.final_idx;
+        out->ms = ms;
+    }
+    f.iter += 1;
+    return ORION_OK;
+}
+
+orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev_src, void *dev_dst, void *dev_aux,
+                                  void *stream, orion_step_report *out, long long *h2d, long long *d2h)
+{
+    if (!t || !a || !dev_src || !dev_dst) return fail(ORION_E_INVALID, "orion_tune_step_host: NULL");
+    const KernelDef &def = *t->v->def;
+    const size_t elem = def.kind == K_STENCIL ? 4 : 16;
+    const size_t row = (size_t)a->width * elem;
+    const size_t in_bytes = (size_t)(a->src_row_end - a->src_row_begin) * row;
+    const size_t out_bytes = (size_t)(a->row_end - a->row_begin) * row;
+    if (a->src_row_end < a->src_row_begin || (def.kind == K_STENCIL && (!dev_aux || !a->aux)))
+        return fail(ORION_E_INVALID, "orion_tune_step_host: bad argument");
+    const Driver &D = drv();
+    CUstream s = (CUstream)stream;
+    ORION_TRY(ensure_context(t->v->device));
+    ORION_CU(D.cuMemcpyHtoDAsync((CUdeviceptr)dev_src, a->src, in_bytes, s));
+    size_t aux_bytes = 0;
+    if (def.kind == K_STENCIL) {
+        aux_bytes = in_bytes;
+        ORION_CU(D.cuMemcpyHtoDAsync((CUdeviceptr)dev_aux, a->aux, aux_bytes, s));
+    }
+    orion_args da = *a;
+    da.src = dev_src;
+    da.dst = dev_dst;
+    da.aux = dev_aux;
+    ORION_TRY(orion_tune_step(t, &da, stream, out));
+    const char *dptr = (const char *)dev_dst + (size_t)(a->row_begin - a->dst_row_begin) * row;
+    ORION_CU(D.cuMemcpyDtoHAsync((char *)a->dst + (size_t)(a->row_begin - a->dst_row_begin) * row,
+                                 (CUdeviceptr)dptr, out_bytes, s));
+    ORION_CU(D.cuStreamSynchronize(s));
+    if (h2d) *h2d = (long long)(in_bytes + aux_bytes);
+    if (d2h) *d2h = (long long)out_bytes;
+    return ORION_OK;
+}
+
+orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, int capacity, int *n_out)
+{
+    if (!t || !n_out || capacity < 0 || (capacity > 0 && !out)) return fail(ORION_E_INVALID, "orion_tuner_ladder");
+    if (direction) *direction = t->f.direction;
+    *n_out = (int)t->f.ladder.size();
+    if ((int)t->f.ladder.size() > capacity) return fail(ORION_E_CAPACITY, "orion_tuner_ladder: capacity");
+    std::copy(t->f.ladder.begin(), t->f.ladder.end(), out);
+    return ORION_OK;
+}
+
+orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final)
+{
+    if (!t) return fail(ORION_E_INVALID, "orion_tuner_final: NULL");
+    if (final_level_idx) *final_level_idx = t->f.final_idx;
+    if (iterations_to_final) *iterations_to_final = t->f.final_iter;
+    return ORION_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,323 @@
+// variants.cpp -- the multi-version binary (orion_build_variants), realising a level at
+// launch (orion_launch), the exhaustive sweep, and the synthetic-input generators.
+//
+// Realising occupancy level k on sm_100a (§3.2 P:L213-P:L229 realises it by
+// bounding registers and shared memory per thread; P:L649 lowers it "by dynamically
+// increasing shared memory usage per thread"):
+//   registers      -> the variant's cubin was assembled with --maxrregcount=R_k;
+//   shared memory  -> the launch requests the kernel's own need + pad_k bytes of dynamic
+//                     shared memory, pad_k recomputed from the ACTUAL register count, with
+//                     the shared-memory carveout pinned at 100 % whenever pad_k > 0 so the
+//                     per-SM budget the pad divides is the full 228 KB;
+//   verification   -> cuOccupancyMaxActiveBlocksPerMultiprocessor must report exactly k.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+
+#include "orion_internal.h"
+
+using namespace orion;
+
+namespace {
+
+int warps_of(const orion_device_limits &d, int T) { return (T + d.warp_size - 1) / d.warp_size; }
+
+// Translate the public argument block into the kernel's parameter block, checking that
+// the source slab holds every row the kernel reaches (clamped to the image).
+orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *k)
+{
+    if (!a) return fail(ORION_E_INVALID, "orion_launch: NULL args");
+    if (a->width <= 0 || a->height <= 0 || a->row_begin < 0 || a->row_end > a->height || a->row_begin > a->row_end)
+        return fail(ORION_E_INVALID, "orion_launch: bad image geometry");
+    if (a->row_begin == a->row_end) return ORION_OK;
+    if (!a->src || !a->dst || (def.kind == K_STENCIL && !a->aux))
+        return fail(ORION_E_INVALID, "orion_launch: NULL buffer");
+    const int need_lo = std::max(0, a->row_begin - def.halo);
+    const int need_hi = std::min(a->height, a->row_end + def.halo);
+    if (a->src_row_begin > need_lo || a->src_row_end < need_hi)
+        return fail(ORION_E_INVALID, "orion_launch: src rows do not cover the halo of the output rows");
+    if (a->dst_row_begin > a->row_begin) return fail(ORION_E_INVALID, "orion_launch: dst_row_begin > row_begin");
+    std::memset(k, 0, sizeof *k);
+    k->src = a->src;
+    k->dst = a->dst;
+    k->aux = a->aux;
+    k->width = a->width;
+    k->height = a->height;
+    k->row_begin = a->row_begin;
+    k->row_end = a->row_end;
+    k->src_row_begin = a->src_row_begin;
+    k->src_row_end = a->src_row_end;
+    k->dst_row_begin = a->dst_row_begin;
+    if (def.kind == K_STENCIL) {
+        for (int i = 0; i < 5; ++i) k->fparam[i] = a->fparam[i];
+    } else {
+        // SDK parameters -> kernel form: w = 2^(d * (-Noise log2 e) + geo); count threshold
+        // "cnt/A > lthr" on an integer count == cnt >= floor(lthr*A) + 1.
+        const double noise = a->fparam[0];
+        if (!(noise >= 0.0)) return fail(ORION_E_INVALID, "orion_launch: Noise must be >= 0");
+        k->fparam[0] = (float)(-noise * 1.4426950408889634);
+        k->fparam[1] = a->fparam[1];
+        k->fparam[2] = a->fparam[2];
+        k->iparam0 = (int)std::floor((double)a->fparam[3] * 49.0) + 1;
+    }
+    return ORION_OK;
+}
+
+orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const orion_kargs &k, CUstream s)
+{
+    const int rows = k.row_end - k.row_begin;
+    if (rows <= 0) return ORION_OK;
+    const unsigned gx = (unsigned)((k.width + def.tile_w - 1) / def.tile_w);
+    const unsigned gy = (unsigned)((rows + def.tile_h - 1) / def.tile_h);
+    void *params[] = {const_cast<orion_kargs *>(&k)};
+    ORION_CU(drv().cuLaunchKernel(fn, gx, gy, 1, (unsigned)def.bx, (unsigned)def.by, 1, (unsigned)dyn_bytes, s,
+                                  params, nullptr));
+    g_launches.fetch_add(1);
+    return ORION_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+orion_status orion_build_variants(int device, const char *kernel_id, int block_threads, const orion_level *levels,
+                                  int n, orion_variants **out)
+{
+    if (!out || !levels || n <= 0) return fail(ORION_E_INVALID, "orion_build_variants: bad argument");
+    *out = nullptr;
+    const KernelDef *def = find_kernel(kernel_id, block_threads);
+    if (!def) return fail(ORION_E_INVALID, std::string("unknown kernel ") + (kernel_id ? kernel_id : "(null)"));
+    ORION_TRY(ensure_context(device));
+    auto v = new orion_variants();
+    std::unique_ptr<orion_variants, void (*)(orion_variants *)> guard(v, orion_variants_destroy);
+    v->device = device;
+    v->def = def;
+    ORION_TRY(orion_query_limits(device, &v->dev));
+    ORION_TRY(orion_kernel_probe(kernel_id, def->threads, &v->res));
+    const Driver &D = drv();
+    const int T = def->threads;
+    const int need = def->dyn_need();
+    for (int i = 0; i < n; ++i) {
+        const orion_level &L = levels[i];
+        if (L.ctas_per_sm < 1 || L.reg_cap < 0 || L.reg_cap > 255)
+            return fail(ORION_E_INVALID, "orion_build_variants: bad level");
+        orion_variants::Var var;
+        var.planned = L;
+        ORION_TRY(compile_variant(*def, L.reg_cap, &var.cv));
+        ORION_CU(D.cuModuleLoadData(&var.mod, var.cv->cubin.data()));
+        v->vars.push_back(var);   // owns the module from here on (destroy unloads it)
+        orion_variants::Var &w = v->vars.back();
+        ORION_CU(D.cuModuleGetFunction(&w.fn, w.mod, def->entry));
+        int static_smem = 0;
+        ORION_CU(D.cuFuncGetAttribute(&w.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, w.fn));
+        ORION_CU(D.cuFuncGetAttribute(&w.local_bytes, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, w.fn));
+        ORION_CU(D.cuFuncGetAttribute(&static_smem, CU_FUNC_ATTRIBUTE_SHARED_SIZE_BYTES, w.fn));
+        const int pad = pad_for_level(v->dev, T, w.regs, static_smem, need, L.ctas_per_sm);
+        if (pad < 0)
+            return fail(ORION_E_INFEASIBLE, "level " + std::to_string(L.ctas_per_sm) + " CTAs/SM not realisable at " +
+                                                std::to_string(w.regs) + " registers");
+        w.dyn_bytes = need + pad;
+        ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, w.dyn_bytes));
+        if (pad > 0) ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100));
+        ORION_CU(D.cuOccupancyMaxActiveBlocksPerMultiprocessor(&w.verified, w.fn, T, (size_t)w.dyn_bytes));
+        if (w.verified != L.ctas_per_sm && pad == 0) {
+            // the driver picked a smaller carveout than the calculator assumes: pin it
+            ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100));
+            ORION_CU(D.cuOccupancyMaxActiveBlocksPerMultiprocessor(&w.verified, w.fn, T, (size_t)w.dyn_bytes));
+        }
+        if (w.verified != L.ctas_per_sm)
+            return fail(ORION_E_OCCUPANCY_MISMATCH, std::string(def->entry) + ": level " +
+                                                        std::to_string(L.ctas_per_sm) + " realised as " +
+                                                        std::to_string(w.verified) + " CTAs/SM");
+        w.realised = L;
+        w.realised.smem_pad_bytes = pad;
+        int limiter = 0;
+        ctas_per_sm(v->dev, T, w.regs, static_smem, w.dyn_bytes, &limiter);
+        w.realised.limiter = limiter;
+        w.realised.warps_per_sm = L.ctas_per_sm * warps_of(v->dev, T);
+        w.realised.occupancy_permille = w.realised.warps_per_sm * 1000 / (v->dev.max_threads_per_sm / v->dev.warp_size);
+    }
+    *out = guard.release();
+    return ORION_OK;
+}
+
+void orion_variants_destroy(orion_variants *v)
+{
+    if (!v) return;
+    if (drv().ok)
+        for (auto &w : v->vars)
+            if (w.mod) drv().cuModuleUnload(w.mod);
+    delete v;
+}
+
+orion_status orion_variants_count(const orion_variants *v, int *n)
+{
+    if (!v || !n) return fail(ORION_E_INVALID, "orion_variants_count: NULL");
+    *n = (int)v->vars.size();
+    return ORION_OK;
+}
+
+orion_status orion_variant_level(const orion_variants *v, int i, orion_level *out)
+{
+    if (!v || !out || i < 0 || i >= (int)v->vars.size()) return fail(ORION_E_INVALID, "orion_variant_level");
+    *out = v->vars[i].realised;
+    return ORION_OK;
+}
+
+orion_status orion_variant_info(const orion_variants *v, int i, int *regs, int *spill_st, int *spill_ld,
+                                int *local_bytes, int *verified)
+{
+    if (!v || i < 0 || i >= (int)v->vars.size()) return fail(ORION_E_INVALID, "orion_variant_info");
+    const auto &w = v->vars[i];
+    if (regs) *regs = w.regs;
+    if (spill_st) *spill_st = w.cv->spill_store;
+    if (spill_ld) *spill_ld = w.cv->spill_load;
+    if (local_bytes) *local_bytes = w.local_bytes;
+    if (verified) *verified = w.verified;
+    return ORION_OK;
+}
+
+orion_status orion_variants_resources(const orion_variants *v, orion_kernel_resources *out)
+{
+    if (!v || !out) return fail(ORION_E_INVALID, "orion_variants_resources: NULL");
+    *out = v->res;
+    return ORION_OK;
+}
+
+orion_status orion_launch(orion_variants *v, int i, const orion_args *a, void *stream)
+{
+    if (!v || i < 0 || i >= (int)v->vars.size()) return fail(ORION_E_INVALID, "orion_launch: bad variant");
+    orion_kargs k;
+    ORION_TRY(make_kargs(*v->def, a, &k));
+    if (a->row_begin == a->row_end) return ORION_OK;
+    ORION_TRY(ensure_context(v->device));
+    const auto &w = v->vars[i];
+    return launch_fn(*v->def, w.fn, w.dyn_bytes, k, (CUstream)stream);
+}
+
+orion_status orion_sweep(orion_variants *v, const orion_args *a, void *stream, int rounds, float *ms_median)
+{
+    if (!v || !a || rounds <= 0 || !ms_median) return fail(ORION_E_INVALID, "orion_sweep: bad argument");
+    orion_kargs k;
+    ORION_TRY(make_kargs(*v->def, a, &k));
+    ORION_TRY(ensure_context(v->device));
+    const Driver &D = drv();
+    const int n = (int)v->vars.size();
+    CUstream s = (CUstream)stream;
+    // warm every variant once (module lazy loading, instruction cache)
+    for (int i = 0; i < n; ++i) ORION_TRY(launch_fn(*v->def, v->vars[i].fn, v->vars[i].dyn_bytes, k, s));
+    std::vector<CUevent> ev((size_t)2 * n * rounds, nullptr);
+    orion_status st = ORION_OK;
+    for (auto &e : ev)
+        if (D.cuEventCreate(&e, CU_EVENT_DEFAULT) != CUDA_SUCCESS) {
+            st = fail(ORION_E_CUDA, "cuEventCreate");
+            break;
+        }
+    if (st == ORION_OK) {
+        for (int r = 0; r < rounds && st == ORION_OK; ++r)
+            for (int q = 0; q < n && st == ORION_OK; ++q) {
+                const int i = (q + r) % n;   // rotate the start so no level is always first
+                const size_t e = (size_t)2 * (r * n + i);
+                if (D.cuEventRecord(ev[e], s) != CUDA_SUCCESS) st = fail(ORION_E_CUDA, "cuEventRecord");
+                if (st == ORION_OK) st = launch_fn(*v->def, v->vars[i].fn, v->vars[i].dyn_bytes, k, s);
+                if (st == ORION_OK && D.cuEventRecord(ev[e + 1], s) != CUDA_SUCCESS)
+                    st = fail(ORION_E_CUDA, "cuEventRecord");
+            }
+        if (st == ORION_OK && D.cuStreamSynchronize(s) != CUDA_SUCCESS) st = fail(ORION_E_CUDA, "cuStreamSynchronize");
+        if (st == ORION_OK) {
+            std::vector<float> t(rounds);
+            for (int i = 0; i < n && st == ORION_OK; ++i) {
+                for (int r = 0; r < rounds; ++r) {
+                    const size_t e = (size_t)2 * (r * n + i);
+                    if (D.cuEventElapsedTime(&t[r], ev[e], ev[e + 1]) != CUDA_SUCCESS) {
+                        st = fail(ORION_E_CUDA, "cuEventElapsedTime");
+                        break;
+                    }
+                }
+                std::sort(t.begin(), t.end());
+                ms_median[i] = (rounds % 2) ? t[rounds / 2] : 0.5f * (t[rounds / 2 - 1] + t[rounds / 2]);
+            }
+        }
+    }
+    for (auto &e : ev)
+        if (e) D.cuEventDestroy(e);
+    return st;
+}
+
+// ---- synthetic inputs -------------------------------------------------------------------
+// The device twin of synth/ (a separate implementation of the same counter-based
+// generator; no method arithmetic).  Box geometry is drawn here on the host.
+struct orion_boxes { int x0[12], y0[12], w[12], h[12]; float r[12], g[12], b[12]; };
+
+static uint64_t splitmix64_host(uint64_t x)
+{
+    uint64_t z = x + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+orion_status orion_generate_rgba(int device, void *dst, int W, int H, int row_begin, int row_end, unsigned seed,
+                                 float sigma, void *stream)
+{
+    if (!dst || W <= 0 || H <= 0 || row_begin < 0 || row_end > H || row_begin > row_end || seed >= (1u << 24))
+        return fail(ORION_E_INVALID, "orion_generate_rgba: bad argument");
+    if (row_begin == row_end) return ORION_OK;
+    CUmodule m;
+    ORION_TRY(load_aux_module(device, "gen", &m));
+    CUfunction f;
+    ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_gen_rgba"));
+    orion_boxes bx;
+    for (int b = 0; b < 12; ++b) {
+        uint64_t h[5];
+        for (int k = 0; k < 5; ++k)
+            h[k] = splitmix64_host(((uint64_t)seed << 40) | (1ull << 39) | (uint64_t)(b * 8 + k));
+        bx.x0[b] = (int)(h[0] % (uint64_t)W);
+        bx.y0[b] = (int)(h[1] % (uint64_t)H);
+        bx.w[b] = 1 + (int)(h[2] % (uint64_t)std::max(1, W / 4));
+        bx.h[b] = 1 + (int)(h[3] % (uint64_t)std::max(1, H / 4));
+        bx.r[b] = (float)(((h[4] >> 0) % 820 + 102) / 1024.0);
+        bx.g[b] = (float)(((h[4] >> 16) % 820 + 102) / 1024.0);
+        bx.b[b] = (float)(((h[4] >> 32) % 820 + 102) / 1024.0);
+    }
+    const float s = (float)(std::sqrt(3.0) * (double)sigma);
+    unsigned long long sd = seed;
+    void *params[] = {&dst, &W, &H, &row_begin, &row_end, &sd, (void *)&s, &bx};
+    ORION_CU(drv().cuLaunchKernel(f, (unsigned)((W + 255) / 256), (unsigned)(row_end - row_begin), 1, 256, 1, 1, 0,
+                                  (CUstream)stream, params, nullptr));
+    g_launches.fetch_add(1);
+    return ORION_OK;
+}
+
+orion_status orion_generate_thermal(int device, void *t0, void *pw, int W, int H, unsigned seed, void *stream)
+{
+    if (!t0 || !pw || W <= 0 || H <= 0 || seed >= (1u << 24))
+        return fail(ORION_E_INVALID, "orion_generate_thermal: bad argument");
+    CUmodule m;
+    ORION_TRY(load_aux_module(device, "gen", &m));
+    CUfunction f;
+    ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_gen_thermal"));
+    unsigned long long sd = seed;
+    void *params[] = {&t0, &pw, &W, &H, &sd};
+    ORION_CU(drv().cuLaunchKernel(f, (unsigned)((W + 255) / 256), (unsigned)H, 1, 256, 1, 1, 0, (CUstream)stream,
+                                  params, nullptr));
+    g_launches.fetch_add(1);
+    return ORION_OK;
+}
+
+orion_status orion_flush_l2(int device, void *buf, long long bytes, void *stream)
+{
+    if (!buf || bytes < 16) return fail(ORION_E_INVALID, "orion_flush_l2: bad argument");
+    CUmodule m;
+    ORION_TRY(load_aux_module(device, "gen", &m));
+    CUfunction f;
+    ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_l2_flush"));
+    size_t n = (size_t)(bytes / 16);
+    float val = 0.0f;
+    void *params[] = {&buf, &n, &val};
+    ORION_CU(drv().cuLaunchKernel(f, 148 * 8, 1, 1, 256, 1, 1, 0, (CUstream)stream, params, nullptr));
+    g_launches.fetch_add(1);
+    return ORION_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,407 @@
+"""Thin ctypes binding of liborion (include/orion.h) -- argument marshalling only.
+
+Every step of the hot path runs inside liborion.so and its sm_100a kernels; this
+module only converts Python values to the C structs and raises ``OrionError`` on a
+negative status.  There is no fallback: if liborion.so is missing the import of
+``lib()`` raises, and on a machine without a GPU the device entry points return
+ORION_E_CUDA (host-only entry points -- levels, probe, replay -- still work).
+
+Device buffers are passed as integer device pointers (e.g. ``tensor.data_ptr()``) and
+streams as integer CUstream handles (``torch.cuda.current_stream().cuda_stream``).
+"""
+from __future__ import annotations
+
+import ctypes
+import math
+import os
+import threading
+from dataclasses import dataclass
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liborion.so")
+
+ORION_OK = 0
+STATUS = {0: "ORION_OK", -1: "ORION_E_INVALID", -2: "ORION_E_CAPACITY", -3: "ORION_E_INFEASIBLE",
+          -4: "ORION_E_COMPILE", -5: "ORION_E_CUDA", -6: "ORION_E_OCCUPANCY_MISMATCH", -7: "ORION_E_STATE"}
+LIM_REGS, LIM_SMEM, LIM_WARPS, LIM_BLOCKS = 1, 2, 4, 8
+DIR_DECREASING, DIR_INCREASING = -1, 1
+SELECT_FASTEST, SELECT_LOWEST_WITHIN_TOL = 0, 1
+
+# SDK imageDenoising parameters (reading R-O2): Noise = 1/h^2, lerpC, weight
+# threshold, lerp threshold (fraction of the 49 window taps).
+KNN_PARAMS = (1.0 / (0.32 * 0.32), 0.2, 0.02, 0.79)
+NLM_PARAMS = (1.0 / (1.45 * 1.45), 0.2, 0.10, 0.10)
+HALO = {"knn_f4": 3, "nlm_f4": 6, "nlm_f4_direct": 6, "nlm_f4_regheavy": 6, "hotspot_f32": 1}
+KERNELS = ("knn_f4", "nlm_f4", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32")
+
+
+class OrionError(RuntimeError):
+    def __init__(self, status: int, where: str, msg: str):
+        super().__init__(f"{where}: {STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class DeviceLimits(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int) for n in (
+        "cc_major", "cc_minor", "sm_count", "warp_size", "regs_per_sm", "regs_per_block",
+        "max_regs_per_thread", "reg_alloc_unit", "num_subpartitions", "max_threads_per_sm",
+        "max_threads_per_block", "max_blocks_per_sm", "smem_per_sm", "smem_per_block_optin",
+        "smem_reserved_per_block", "smem_alloc_unit")]
+
+
+class KernelResources(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int) for n in (
+        "block_threads", "regs_per_thread", "static_smem_bytes", "dyn_smem_bytes", "min_reg_cap")]
+
+
+class Level(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int) for n in (
+        "ctas_per_sm", "warps_per_sm", "occupancy_permille", "reg_cap", "smem_pad_bytes", "limiter")]
+
+    def as_tuple(self):
+        return tuple(getattr(self, n) for n, _ in self._fields_)
+
+    def __repr__(self):
+        return ("Level(k=%d, warps=%d, occ=%.3f, cap=%d, pad=%d, lim=%d)"
+                % (self.ctas_per_sm, self.warps_per_sm, self.occupancy_permille / 1000.0,
+                   self.reg_cap, self.smem_pad_bytes, self.limiter))
+
+
+class Args(ctypes.Structure):
+    _fields_ = [("src", ctypes.c_void_p), ("dst", ctypes.c_void_p), ("aux", ctypes.c_void_p),
+                ("width", ctypes.c_int), ("height", ctypes.c_int),
+                ("row_begin", ctypes.c_int), ("row_end", ctypes.c_int),
+                ("src_row_begin", ctypes.c_int), ("src_row_end", ctypes.c_int),
+                ("dst_row_begin", ctypes.c_int), ("fparam", ctypes.c_float * 8)]
+
+
+class TunerCfg(ctypes.Structure):
+    _fields_ = [("maxlive_threshold", ctypes.c_int), ("samples_per_level", ctypes.c_int),
+                ("select_mode", ctypes.c_int), ("allow_direction_switch", ctypes.c_int),
+                ("slowdown_tol", ctypes.c_float), ("worse_eps", ctypes.c_float),
+                ("expected_iterations", ctypes.c_int)]
+
+
+class StepReport(ctypes.Structure):
+    _fields_ = [("iteration", ctypes.c_int), ("level_idx", ctypes.c_int), ("phase", ctypes.c_int),
+                ("final_level_idx", ctypes.c_int), ("ms", ctypes.c_float)]
+
+
+_lock = threading.Lock()
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load liborion.so (building it first if it is missing and nvcc is available)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            if not os.path.exists(LIB_PATH):
+                from . import build as _build
+                _build.build()
+            L = ctypes.CDLL(LIB_PATH)
+            P, I, V = ctypes.POINTER, ctypes.c_int, ctypes.c_void_p
+            sig = {
+                "orion_b200_limits": [P(DeviceLimits)],
+                "orion_query_limits": [I, P(DeviceLimits)],
+                "orion_ctas_per_sm": [P(DeviceLimits), I, I, I, I, P(I), P(I)],
+                "orion_levels": [P(DeviceLimits), P(KernelResources), P(Level), I, P(I)],
+                "orion_kernel_probe": [ctypes.c_char_p, I, P(KernelResources)],
+                "orion_compile_info": [ctypes.c_char_p, I, I, P(I), P(I), P(I), P(I)],
+                "orion_build_variants": [I, ctypes.c_char_p, I, P(Level), I, P(V)],
+                "orion_variants_count": [V, P(I)],
+                "orion_variant_level": [V, I, P(Level)],
+                "orion_variant_info": [V, I, P(I), P(I), P(I), P(I), P(I)],
+                "orion_variants_resources": [V, P(KernelResources)],
+                "orion_launch": [V, I, P(Args), V],
+                "orion_sweep": [V, P(Args), V, I, P(ctypes.c_float)],
+                "orion_tuner_default_cfg": [P(TunerCfg)],
+                "orion_tuner_create": [V, P(TunerCfg), P(V)],
+                "orion_tune_step": [V, P(Args), V, P(StepReport)],
+                "orion_tune_step_host": [V, P(Args), V, V, V, V, P(StepReport), P(ctypes.c_longlong),
+                                         P(ctypes.c_longlong)],
+                "orion_tuner_ladder": [V, P(I), P(I), I, P(I)],
+                "orion_tuner_final": [V, P(I), P(I)],
+                "orion_tuner_replay": [P(TunerCfg), P(Level), I, I, P(ctypes.c_float), I, P(I), P(I), P(I)],
+                "orion_generate_rgba": [I, V, I, I, I, I, ctypes.c_uint, ctypes.c_float, V],
+                "orion_generate_thermal": [I, V, V, I, I, ctypes.c_uint, V],
+                "orion_flush_l2": [I, V, ctypes.c_longlong, V],
+            }
+            for name, args in sig.items():
+                f = getattr(L, name)
+                f.argtypes = args
+                f.restype = ctypes.c_int
+            for name in ("orion_variants_destroy", "orion_tuner_destroy"):
+                getattr(L, name).argtypes = [V]
+                getattr(L, name).restype = None
+            L.orion_status_str.restype = ctypes.c_char_p
+            L.orion_status_str.argtypes = [I]
+            L.orion_last_error.restype = ctypes.c_char_p
+            L.orion_last_error.argtypes = []
+            L.orion_launch_count.restype = ctypes.c_longlong
+            L.orion_version.restype = ctypes.c_char_p
+            _lib = L
+    return _lib
+
+
+def _check(status: int, where: str):
+    if status != ORION_OK:
+        raise OrionError(status, where, lib().orion_last_error().decode(errors="replace"))
+
+
+def _s(stream) -> ctypes.c_void_p:
+    return ctypes.c_void_p(int(stream) if stream else 0)
+
+
+# ---- levels (host-only) -------------------------------------------------------------------
+def b200_limits() -> DeviceLimits:
+    d = DeviceLimits()
+    _check(lib().orion_b200_limits(ctypes.byref(d)), "orion_b200_limits")
+    return d
+
+
+def query_limits(device: int = 0) -> DeviceLimits:
+    d = DeviceLimits()
+    _check(lib().orion_query_limits(device, ctypes.byref(d)), "orion_query_limits")
+    return d
+
+
+def ctas_per_sm(dev: DeviceLimits, T: int, regs: int, smem_static: int = 0, smem_dyn: int = 0):
+    c, lim = ctypes.c_int(), ctypes.c_int()
+    _check(lib().orion_ctas_per_sm(ctypes.byref(dev), T, regs, smem_static, smem_dyn, ctypes.byref(c),
+                                   ctypes.byref(lim)), "orion_ctas_per_sm")
+    return c.value, lim.value
+
+
+def resources(block_threads: int, regs: int, static_smem: int = 0, dyn_smem: int = 0,
+              min_reg_cap: int = 16) -> KernelResources:
+    return KernelResources(block_threads, regs, static_smem, dyn_smem, min_reg_cap)
+
+
+def levels(dev: DeviceLimits, res: KernelResources) -> list[Level]:
+    n = ctypes.c_int()
+    st = lib().orion_levels(ctypes.byref(dev), ctypes.byref(res), None, 0, ctypes.byref(n))
+    if st not in (ORION_OK, -2):
+        _check(st, "orion_levels")
+    arr = (Level * max(1, n.value))()
+    _check(lib().orion_levels(ctypes.byref(dev), ctypes.byref(res), arr, n.value, ctypes.byref(n)), "orion_levels")
+    return [arr[i] for i in range(n.value)]
+
+
+def kernel_probe(kernel_id: str, block_threads: int = 0) -> KernelResources:
+    r = KernelResources()
+    _check(lib().orion_kernel_probe(kernel_id.encode(), block_threads, ctypes.byref(r)), "orion_kernel_probe")
+    return r
+
+
+def compile_info(kernel_id: str, block_threads: int, reg_cap: int) -> dict:
+    v = [ctypes.c_int() for _ in range(4)]
+    _check(lib().orion_compile_info(kernel_id.encode(), block_threads, reg_cap, *[ctypes.byref(x) for x in v]),
+           "orion_compile_info")
+    return dict(regs=v[0].value, spill_store=v[1].value, spill_load=v[2].value, local_bytes=v[3].value)
+
+
+# ---- launch arguments ----------------------------------------------------------------------
+def denoise_args(kernel_id: str, src: int, dst: int, width: int, height: int, row_begin: int = 0,
+                 row_end: int | None = None, src_row_begin: int = 0, src_row_end: int | None = None,
+                 dst_row_begin: int | None = None, params=None) -> Args:
+    row_end = height if row_end is None else row_end
+    src_row_end = height if src_row_end is None else src_row_end
+    dst_row_begin = row_begin if dst_row_begin is None else dst_row_begin
+    p = params or (KNN_PARAMS if kernel_id.startswith("knn") else NLM_PARAMS)
+    a = Args(src, dst, None, width, height, row_begin, row_end, src_row_begin, src_row_end, dst_row_begin)
+    for i, x in enumerate(p):
+        a.fparam[i] = x
+    return a
+
+
+def hotspot_constants(cell: float = 0.016 / 512) -> tuple:
+    """Rodinia hotspot coefficients at a fixed cell size (reading R-A15):
+    (sdc = step/Cap, rx = 1/Rx, ry = 1/Ry, rz = 1/Rz, amb)."""
+    t_chip, k_si, spec_heat, factor_chip, max_pd, precision = 0.0005, 100.0, 1.75e6, 0.5, 3.0e6, 0.001
+    cap = factor_chip * spec_heat * t_chip * cell * cell
+    r_x = cell / (2.0 * k_si * t_chip * cell)
+    r_y = cell / (2.0 * k_si * t_chip * cell)
+    r_z = t_chip / (k_si * cell * cell)
+    step = precision / (max_pd / (factor_chip * t_chip * spec_heat))
+    return (step / cap, 1.0 / r_x, 1.0 / r_y, 1.0 / r_z, 80.0)
+
+
+def hotspot_args(t_in: int, t_out: int, power: int, width: int, height: int, row_begin: int = 0,
+                 row_end: int | None = None, consts=None) -> Args:
+    row_end = height if row_end is None else row_end
+    a = Args(t_in, t_out, power, width, height, row_begin, row_end, 0, height, 0)
+    for i, x in enumerate(consts or hotspot_constants()):
+        a.fparam[i] = x
+    return a
+
+
+# ---- the multi-version binary --------------------------------------------------------------
+@dataclass
+class VariantInfo:
+    level: Level
+    regs: int
+    spill_store: int
+    spill_load: int
+    local_bytes: int
+    verified_ctas: int
+
+
+class Variants:
+    """orion_build_variants handle: one sm_100a variant per occupancy level."""
+
+    def __init__(self, device: int, kernel_id: str, lv: list[Level], block_threads: int = 0):
+        self.kernel_id = kernel_id
+        self.device = device
+        arr = (Level * len(lv))(*lv)
+        h = ctypes.c_void_p()
+        _check(lib().orion_build_variants(device, kernel_id.encode(), block_threads, arr, len(lv), ctypes.byref(h)),
+               "orion_build_variants")
+        self.h = h
+        self.planned = list(lv)
+
+    def __len__(self):
+        n = ctypes.c_int()
+        _check(lib().orion_variants_count(self.h, ctypes.byref(n)), "orion_variants_count")
+        return n.value
+
+    def level(self, i: int) -> Level:
+        L = Level()
+        _check(lib().orion_variant_level(self.h, i, ctypes.byref(L)), "orion_variant_level")
+        return L
+
+    def info(self, i: int) -> VariantInfo:
+        v = [ctypes.c_int() for _ in range(5)]
+        _check(lib().orion_variant_info(self.h, i, *[ctypes.byref(x) for x in v]), "orion_variant_info")
+        return VariantInfo(self.level(i), *[x.value for x in v])
+
+    def resources(self) -> KernelResources:
+        r = KernelResources()
+        _check(lib().orion_variants_resources(self.h, ctypes.byref(r)), "orion_variants_resources")
+        return r
+
+    def launch(self, i: int, args: Args, stream=None):
+        _check(lib().orion_launch(self.h, i, ctypes.byref(args), _s(stream)), "orion_launch")
+
+    def sweep(self, args: Args, stream=None, rounds: int = 5) -> list[float]:
+        ms = (ctypes.c_float * len(self))()
+        _check(lib().orion_sweep(self.h, ctypes.byref(args), _s(stream), rounds, ms), "orion_sweep")
+        return list(ms)
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().orion_variants_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def build_all_levels(device: int, kernel_id: str, block_threads: int = 0, dev: DeviceLimits | None = None):
+    """Convenience: probe -> orion_levels -> orion_build_variants (every feasible level)."""
+    res = kernel_probe(kernel_id, block_threads)
+    dev = dev or query_limits(device)
+    lv = levels(dev, res)
+    return Variants(device, kernel_id, lv, block_threads), res
+
+
+def default_cfg(**kw) -> TunerCfg:
+    c = TunerCfg()
+    _check(lib().orion_tuner_default_cfg(ctypes.byref(c)), "orion_tuner_default_cfg")
+    for k, v in kw.items():
+        setattr(c, k, v)
+    return c
+
+
+class Tuner:
+    """orion_tuner handle: Fig. 8 ladder + Fig. 9 walk across iterations."""
+
+    def __init__(self, variants: Variants, cfg: TunerCfg | None = None):
+        self.variants = variants
+        h = ctypes.c_void_p()
+        _check(lib().orion_tuner_create(variants.h, ctypes.byref(cfg or default_cfg()), ctypes.byref(h)),
+               "orion_tuner_create")
+        self.h = h
+
+    def step(self, args: Args, stream=None) -> StepReport:
+        r = StepReport()
+        _check(lib().orion_tune_step(self.h, ctypes.byref(args), _s(stream), ctypes.byref(r)), "orion_tune_step")
+        return r
+
+    def step_host(self, args: Args, dev_src: int, dev_dst: int, dev_aux: int | None = None, stream=None):
+        r = StepReport()
+        hi, ho = ctypes.c_longlong(), ctypes.c_longlong()
+        _check(lib().orion_tune_step_host(self.h, ctypes.byref(args), ctypes.c_void_p(dev_src),
+                                          ctypes.c_void_p(dev_dst), ctypes.c_void_p(dev_aux or 0), _s(stream),
+                                          ctypes.byref(r), ctypes.byref(hi), ctypes.byref(ho)),
+               "orion_tune_step_host")
+        return r, hi.value, ho.value
+
+    def ladder(self):
+        d, n = ctypes.c_int(), ctypes.c_int()
+        buf = (ctypes.c_int * 64)()
+        _check(lib().orion_tuner_ladder(self.h, ctypes.byref(d), buf, 64, ctypes.byref(n)), "orion_tuner_ladder")
+        return d.value, [buf[i] for i in range(n.value)]
+
+    def final(self):
+        f, it = ctypes.c_int(), ctypes.c_int()
+        _check(lib().orion_tuner_final(self.h, ctypes.byref(f), ctypes.byref(it)), "orion_tuner_final")
+        return f.value, it.value
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().orion_tuner_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def tuner_replay(cfg: TunerCfg, lv: list[Level], natural_regs: int, ms_of_level, iterations: int):
+    n = len(lv)
+    arr = (Level * n)(*lv)
+    ms = (ctypes.c_float * n)(*[float(x) for x in ms_of_level])
+    ran = (ctypes.c_int * max(1, iterations))()
+    f, fi = ctypes.c_int(), ctypes.c_int()
+    _check(lib().orion_tuner_replay(ctypes.byref(cfg), arr, n, natural_regs, ms, iterations, ran, ctypes.byref(f),
+                                    ctypes.byref(fi)), "orion_tuner_replay")
+    return [ran[i] for i in range(iterations)], f.value, fi.value
+
+
+# ---- synthetic inputs (device generator) ----------------------------------------------------
+def generate_rgba(device: int, dst: int, width: int, height: int, row_begin: int = 0, row_end: int | None = None,
+                  seed: int = 1, sigma: float = 0.13, stream=None):
+    row_end = height if row_end is None else row_end
+    _check(lib().orion_generate_rgba(device, ctypes.c_void_p(dst), width, height, row_begin, row_end, seed,
+                                     sigma, _s(stream)), "orion_generate_rgba")
+
+
+def generate_thermal(device: int, t0: int, power: int, width: int, height: int, seed: int = 1, stream=None):
+    _check(lib().orion_generate_thermal(device, ctypes.c_void_p(t0), ctypes.c_void_p(power), width, height, seed,
+                                        _s(stream)), "orion_generate_thermal")
+
+
+def flush_l2(device: int, buf: int, nbytes: int, stream=None):
+    _check(lib().orion_flush_l2(device, ctypes.c_void_p(buf), nbytes, _s(stream)), "orion_flush_l2")
+
+
+def launch_count() -> int:
+    return lib().orion_launch_count()
+
+
+def version() -> str:
+    return lib().orion_version().decode()
+
+
+def occupancy(level: Level) -> float:
+    return level.occupancy_permille / 1000.0
+
+
+__all__ = [n for n in dir() if not n.startswith("_") and n not in ("annotations", "ctypes", "math", "os",
+                                                                      "threading", "dataclass")]

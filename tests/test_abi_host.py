@@ -1,0 +1,143 @@
+"""The C-ABI library on the CPU: it loads, exports every symbol include/orion.h declares,
+and its host-only entry points agree with the oracle:
+
+* orion_levels / orion_ctas_per_sm  == oracle O1, field by field (bit-exact integers);
+* orion_tuner_replay (the product's Fig. 8 + Fig. 9 state machine) == oracle O4's decision
+  sequence on the SURVEY O4 vectors and on random runtime tables;
+* the embedded ptxas honours every register cap (regs <= cap) -- the realisation of a level.
+No compute call runs here (no GPU).
+"""
+import itertools
+import os
+import random
+import re
+
+import pytest
+from hypothesis import given, settings, strategies as st
+
+from oracle import occupancy as OC
+from oracle import tuner as OT
+from paper_conf_middleware_hayeslcsz16_b200 import orion as O
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    txt = open(os.path.join(ROOT, "include", "orion.h")).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(orion_[a-z0-9_]+)\s*\(", txt)))
+
+
+def test_library_exports_every_declared_symbol():
+    lib = O.lib()
+    syms = header_symbols()
+    assert len(syms) >= 29
+    missing = [s for s in syms if not hasattr(lib, s)]
+    assert not missing, missing
+    assert O.version().startswith("liborion")
+
+
+def _to_oracle_dev(d: O.DeviceLimits) -> OC.Device:
+    return OC.Device(**{n: getattr(d, n) for n, _ in O.DeviceLimits._fields_})
+
+
+def test_b200_limits_match_oracle_device():
+    assert _to_oracle_dev(O.b200_limits()) == OC.B200
+
+
+def test_ctas_per_sm_matches_oracle_grid():
+    d = O.b200_limits()
+    for T, r, s, dyn in itertools.product((32, 64, 96, 128, 256, 512, 1024), (16, 24, 32, 40, 56, 64, 96, 128, 200, 255),
+                                          (0, 4096), (0, 3000, 45000, 120000, 231424)):
+        k, lim = O.ctas_per_sm(d, T, r, s, dyn)
+        assert k == OC.ctas_per_sm(OC.B200, T, r, s, dyn), (T, r, s, dyn)
+        assert lim == OC.limiter_mask(OC.B200, T, r, s, dyn), (T, r, s, dyn)
+
+
+@pytest.mark.parametrize("T", [64, 128, 256, 512])
+@pytest.mark.parametrize("natural", [16, 24, 32, 37, 39, 46, 56, 63, 64, 72, 96, 128, 168, 200, 241, 255])
+@pytest.mark.parametrize("smem", [(0, 0), (0, 13376), (1024, 8192), (0, 52544), (0, 100000)])
+def test_levels_bit_exact_vs_oracle(T, natural, smem):
+    d = O.b200_limits()
+    got = [l.as_tuple() for l in O.levels(d, O.resources(T, natural, smem[0], smem[1]))]
+    want = [(l.ctas_per_sm, l.warps_per_sm, l.occupancy_permille, l.reg_cap, l.smem_pad_bytes, l.limiter)
+            for l in OC.levels(OC.B200, T, natural, smem[0], smem[1])]
+    assert got == want
+
+
+def test_levels_capacity_protocol():
+    import ctypes
+    d = O.b200_limits()
+    res = O.resources(128, 255)
+    n = ctypes.c_int()
+    arr = (O.Level * 3)()
+    st_ = O.lib().orion_levels(ctypes.byref(d), ctypes.byref(res), arr, 3, ctypes.byref(n))
+    assert st_ == -2 and n.value == 16
+    bad = O.resources(0, 40)
+    assert O.lib().orion_levels(ctypes.byref(d), ctypes.byref(bad), arr, 3, ctypes.byref(n)) == -1
+    assert "bad kernel resources" in O.lib().orion_last_error().decode()
+
+
+def _o_levels(T, natural, need=0):
+    ol = OC.levels(OC.B200, T, natural, 0, need)
+    return ol, [O.Level(*[getattr(l, f) for f, _ in O.Level._fields_]) for l in ol]
+
+
+def _replay_both(T, natural, need, ms, iters, **cfgkw):
+    ol, pl = _o_levels(T, natural, need)
+    ocfg = OT.TunerCfg(**{k: v for k, v in cfgkw.items()})
+    pcfg = O.default_cfg(**{k: (int(v) if isinstance(v, bool) else v) for k, v in cfgkw.items()})
+    tr = OT.replay(ol, natural, ocfg, ms, iters)
+    ran, fin, fit = O.tuner_replay(pcfg, pl, natural, ms, iters)
+    return tr, ran, fin, fit
+
+
+@pytest.mark.parametrize("T,natural,need,ladder_ms,mode", [
+    (128, 56, 0, [1.00, 1.30, 1.80, 2.60], 0),                 # V1
+    (128, 56, 0, [1.00, 0.90, 0.85, 0.95], 0),                 # V2
+    (256, 20, 45000, [1.000, 1.005, 1.010, 1.015, 1.030], 0),  # V3 FASTEST
+    (256, 20, 45000, [1.000, 1.005, 1.010, 1.015, 1.030], 1),  # V3 LOWEST_WITHIN_TOL
+    (128, 48, 0, [1.0, 0.9, 0.8], 0),                          # V4
+    (128, 40, 0, [1.0, 1.0], 0),                               # V5
+])
+def test_replay_vectors_match_oracle(T, natural, need, ladder_ms, mode):
+    ol, _ = _o_levels(T, natural, need)
+    _, ladder, _ = OT.candidates(ol, natural, OT.TunerCfg())
+    ms = [9.5] * len(ol)
+    for i, t in zip(ladder, ladder_ms):
+        ms[i] = t
+    tr, ran, fin, fit = _replay_both(T, natural, need, ms, 10, select_mode=mode, allow_direction_switch=False)
+    assert ran == tr.ran and fin == tr.final and fit == tr.final_iteration
+
+
+@settings(max_examples=200, deadline=None)
+@given(st.sampled_from([(128, 255, 0), (128, 56, 0), (256, 20, 0), (256, 46, 0), (128, 128, 52544), (64, 39, 13376)]),
+       st.integers(0, 2**31 - 1), st.sampled_from([0, 1]), st.booleans(), st.integers(0, 20))
+def test_replay_random_tables_match_oracle(shape, seed, mode, switch, expected):
+    T, natural, need = shape
+    ol, _ = _o_levels(T, natural, need)
+    rng = random.Random(seed)
+    ms = [round(rng.uniform(0.5, 2.0), 3) for _ in ol]
+    tr, ran, fin, fit = _replay_both(T, natural, need, ms, 25, select_mode=mode, allow_direction_switch=switch,
+                                     expected_iterations=expected)
+    assert ran == tr.ran
+    assert fin == (tr.final if tr.final is not None else -1)
+    assert fit == (tr.final_iteration if tr.final_iteration is not None else -1)
+
+
+@pytest.mark.parametrize("kernel", ["knn_f4", "nlm_f4", "nlm_f4_regheavy", "hotspot_f32"])
+def test_embedded_ptxas_honours_register_caps(kernel):
+    res = O.kernel_probe(kernel)
+    assert res.regs_per_thread > 0 and res.block_threads in (64, 128, 256)
+    for l in O.levels(O.b200_limits(), res):
+        if l.reg_cap:
+            info = O.compile_info(kernel, res.block_threads, l.reg_cap)
+            assert info["regs"] <= l.reg_cap
+
+
+def test_device_entry_points_fail_cleanly_without_gpu():
+    if os.path.exists("/dev/nvidia0"):
+        pytest.skip("a GPU is present")
+    with pytest.raises(O.OrionError) as e:
+        O.query_limits(0)
+    assert e.value.status == -5
