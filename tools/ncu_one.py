@@ -1,0 +1,38 @@
+"""Launch ONE kernel variant once on a synthetic frame (for ncu --set full captures).
+
+usage: python tools/ncu_one.py KERNEL LEVEL W H [THREADS] [REPEAT]
+  LEVEL = index into the level list (-1 = max occupancy, 'orig' = natural build)
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
+
+kernel, lev, W, H = sys.argv[1], sys.argv[2], int(sys.argv[3]), int(sys.argv[4])
+threads = int(sys.argv[5]) if len(sys.argv) > 5 else 0
+repeat = int(sys.argv[6]) if len(sys.argv) > 6 else 1
+torch.cuda.set_device(0)
+sp = torch.cuda.current_stream().cuda_stream
+v, res = O.build_all_levels(0, kernel, threads)
+if lev == "orig":
+    li = next(i for i, l in enumerate(v.planned) if l.reg_cap == 0 and l.smem_pad_bytes == 0)
+else:
+    li = int(lev) % len(v)
+if kernel == "hotspot_f32":
+    a = torch.empty((H, W), device="cuda")
+    b = torch.empty((H, W), device="cuda")
+    p = torch.empty((H, W), device="cuda")
+    O.generate_thermal(0, a.data_ptr(), p.data_ptr(), W, H, stream=sp)
+    args = O.hotspot_args(a.data_ptr(), b.data_ptr(), p.data_ptr(), W, H)
+else:
+    a = torch.empty((H, W, 4), device="cuda")
+    b = torch.empty((H, W, 4), device="cuda")
+    O.generate_rgba(0, a.data_ptr(), W, H, sigma=0.13, stream=sp)
+    args = O.denoise_args(kernel, a.data_ptr(), b.data_ptr(), W, H)
+for _ in range(repeat):
+    v.launch(li, args, sp)
+torch.cuda.synchronize()
+print("launched", kernel, "level", li, v.level(li), v.info(li))
