@@ -6,14 +6,24 @@
 // rounding per operation, no contraction):
 //   t2 = T+T; a = ((S+N)-t2)*ry; b = ((E+W)-t2)*rx; c = (amb-T)*rz; T' = T + (((P+a)+b)+c)*sdc
 //
-// HBM-bound (12 algorithmic bytes per cell-step).  Each warp owns 32 consecutive
-// columns and walks a strip of RY rows top to bottom, keeping N / T / S in
-// registers (every row of T is read once from DRAM per strip); E and W come from
-// the neighbouring lanes by shuffle, lanes 0/31 fetch their outer neighbour (an
-// L1/L2 hit, the same line the neighbouring warp loads).  The loads of the next
-// rows are software-prefetched RY_PF rows ahead to keep enough bytes in flight --
-// and the warps resident per SM (the occupancy level Orion tunes) supply the rest.
+// HBM-bound: 12 algorithmic bytes per cell-step (read T and P, write T').  Each warp
+// owns 128 consecutive columns (4 per lane, 16-byte vector loads and stores) and walks
+// a strip of RY rows top to bottom keeping N / T / S in registers, so every row of T is
+// read from DRAM once per strip; W and E of the lane's 4 cells come from the
+// neighbouring lanes by shuffle, lanes 0/31 fetch their outer neighbour (an L1/L2 hit:
+// the neighbouring warp reads that line).  Grids whose width is not a multiple of 4
+// (rows not 16-byte aligned) take a scalar path with the same arithmetic.
 #include "common.cuh"
+
+ORION_DEVICE float hs_cell(float T, float N, float S, float E, float Wv, float P, const float (&c)[5])
+{
+    const float t2 = __fadd_rn(T, T);
+    const float av = __fmul_rn(__fsub_rn(__fadd_rn(S, N), t2), c[2]);
+    const float bv = __fmul_rn(__fsub_rn(__fadd_rn(E, Wv), t2), c[1]);
+    const float cv = __fmul_rn(__fsub_rn(c[4], T), c[3]);
+    const float acc = __fadd_rn(__fadd_rn(__fadd_rn(P, av), bv), cv);
+    return __fadd_rn(T, __fmul_rn(acc, c[0]));
+}
 
 template <int BY, int RY>
 __device__ __forceinline__ void hotspot_body(const orion_kargs &a)
@@ -23,40 +33,66 @@ __device__ __forceinline__ void hotspot_body(const orion_kargs &a)
     float *tout = (float *)a.dst;
     const int W = a.width, H = a.height;
     const int lane = threadIdx.x;
-    const int xr = blockIdx.x * 32 + lane;
-    const int x = min(xr, W - 1);
     const int ys = a.row_begin + (blockIdx.y * BY + threadIdx.y) * RY;
     if (ys >= a.row_end) return;
     const int ye = min(ys + RY, a.row_end);
-    const float sdc = a.fparam[0], rx = a.fparam[1], ry = a.fparam[2], rz = a.fparam[3], amb = a.fparam[4];
-    const int xl = max(blockIdx.x * 32 - 1, 0);                 // lane 0's west neighbour
-    const int xh = min(blockIdx.x * 32 + 32, W - 1);            // lane 31's east neighbour
-    const int sb = a.src_row_begin;
-#define ROWP(y) (tin + (size_t)((y) - sb) * (size_t)W)
-    float N = __ldg(ROWP(max(ys - 1, 0)) + x);
-    float T = __ldg(ROWP(ys) + x);
-    for (int y = ys; y < ye; ++y) {
-        const float S = __ldg(ROWP(min(y + 1, H - 1)) + x);
-        const float P = __ldg(pw + (size_t)(y - sb) * (size_t)W + x);
-        float Wv = __shfl_up_sync(0xffffffffu, T, 1);
-        float Ev = __shfl_down_sync(0xffffffffu, T, 1);
-        if (lane == 0) Wv = (xr == 0) ? T : __ldg(ROWP(y) + xl);
-        if (lane == 31) Ev = __ldg(ROWP(y) + xh);
-        if (xr >= W - 1) Ev = T;                                  // clamp at the east edge
-        const float t2 = __fadd_rn(T, T);
-        const float av = __fmul_rn(__fsub_rn(__fadd_rn(S, N), t2), ry);
-        const float bv = __fmul_rn(__fsub_rn(__fadd_rn(Ev, Wv), t2), rx);
-        const float cv = __fmul_rn(__fsub_rn(amb, T), rz);
-        const float acc = __fadd_rn(__fadd_rn(__fadd_rn(P, av), bv), cv);
-        const float o = __fadd_rn(T, __fmul_rn(acc, sdc));
-        if (xr < W) tout[(size_t)(y - a.dst_row_begin) * (size_t)W + xr] = o;
-        N = T;
-        T = S;
+    const float c[5] = {a.fparam[0], a.fparam[1], a.fparam[2], a.fparam[3], a.fparam[4]};
+    const size_t sb = (size_t)a.src_row_begin, db = (size_t)a.dst_row_begin;
+    if ((W & 3) == 0) {
+        // ---- vector path: lane owns columns cx .. cx+3 ------------------------------------
+        const int cx = (blockIdx.x * 32 + lane) * 4;
+        const int cxl = min(cx, W - 4);                         // clamped (lanes past the edge)
+        const int base = blockIdx.x * 128;
+#define ROW4(y) (reinterpret_cast<const float4 *>(tin + ((size_t)(y) - sb) * (size_t)W + cxl))
+        float4 N = __ldg(ROW4(max(ys - 1, 0)));
+        float4 T = __ldg(ROW4(ys));
+#pragma unroll 4
+        for (int y = ys; y < ye; ++y) {
+            const float4 S = __ldg(ROW4(min(y + 1, H - 1)));
+            const float4 P = __ldg(reinterpret_cast<const float4 *>(pw + ((size_t)y - sb) * (size_t)W + cxl));
+            float Wv = __shfl_up_sync(0xffffffffu, T.w, 1);
+            float Ev = __shfl_down_sync(0xffffffffu, T.x, 1);
+            const float *trow = tin + ((size_t)y - sb) * (size_t)W;
+            if (lane == 0) Wv = (base == 0) ? T.x : __ldg(trow + base - 1);
+            if (lane == 31) Ev = (base + 128 >= W) ? T.w : __ldg(trow + base + 128);
+            if (cx + 4 >= W) Ev = T.w;                          // clamp at the east edge
+            if (cx == 0) Wv = T.x;                              // clamp at the west edge
+            float4 o;
+            o.x = hs_cell(T.x, N.x, S.x, T.y, Wv, P.x, c);
+            o.y = hs_cell(T.y, N.y, S.y, T.z, T.x, P.y, c);
+            o.z = hs_cell(T.z, N.z, S.z, T.w, T.y, P.z, c);
+            o.w = hs_cell(T.w, N.w, S.w, Ev, T.z, P.w, c);
+            if (cx < W) *reinterpret_cast<float4 *>(tout + ((size_t)y - db) * (size_t)W + cx) = o;
+            N = T;
+            T = S;
+        }
+#undef ROW4
+    } else {
+        // ---- scalar path (rows not 16-byte aligned): lane owns 4 strided columns ---------
+#pragma unroll 1
+        for (int k = 0; k < 4; ++k) {
+            const int xr = blockIdx.x * 128 + k * 32 + lane;
+            const int x = min(xr, W - 1);
+            const float *col = tin + x;
+            float N = __ldg(col + ((size_t)max(ys - 1, 0) - sb) * (size_t)W);
+            float T = __ldg(col + ((size_t)ys - sb) * (size_t)W);
+#pragma unroll 1
+            for (int y = ys; y < ye; ++y) {
+                const float *trow = tin + ((size_t)y - sb) * (size_t)W;
+                const float S = __ldg(col + ((size_t)min(y + 1, H - 1) - sb) * (size_t)W);
+                const float P = __ldg(pw + ((size_t)y - sb) * (size_t)W + x);
+                const float Wv = __ldg(trow + max(x - 1, 0));
+                const float Ev = __ldg(trow + min(x + 1, W - 1));
+                const float o = hs_cell(T, N, S, Ev, Wv, P, c);
+                if (xr < W) tout[((size_t)y - db) * (size_t)W + xr] = o;
+                N = T;
+                T = S;
+            }
+        }
     }
-#undef ROWP
 }
 
-// T = 256 threads (32 x 8 warps), 16-row strips per warp.
+// T = 256 threads (32 x 8 warps): 128 columns x 8 strips of 16 rows per CTA.
 extern "C" __global__ void __launch_bounds__(256) orion_hotspot_f32_256(orion_kargs a) { hotspot_body<8, 16>(a); }
-// T = 128 threads (32 x 4 warps), 16-row strips per warp.
+// T = 128 threads (32 x 4 warps): 128 columns x 4 strips of 16 rows per CTA.
 extern "C" __global__ void __launch_bounds__(128) orion_hotspot_f32_128(orion_kargs a) { hotspot_body<4, 16>(a); }

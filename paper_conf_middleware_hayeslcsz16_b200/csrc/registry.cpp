@@ -51,8 +51,8 @@ static const KernelDef kKernels[] = {
     {"nlm_f4_direct", 128, "orion_nlm_direct_f4_128", "nlm_direct", 32, 4, 32, 4, 6, K_NLM, 1, 0},
     {"nlm_f4_regheavy", 128, "orion_nlm_regheavy_f4_128", "nlm_regheavy", 32, 4, 32, 4, 6, K_NLM, 1, 0},
     {"nlm_f4_regheavy", 64, "orion_nlm_regheavy_f4_64", "nlm_regheavy", 8, 8, 8, 8, 6, K_NLM, 1, 0},
-    {"hotspot_f32", 256, "orion_hotspot_f32_256", "hotspot", 32, 8, 32, 128, 1, K_STENCIL, 0, 0},
-    {"hotspot_f32", 128, "orion_hotspot_f32_128", "hotspot", 32, 4, 32, 64, 1, K_STENCIL, 0, 0},
+    {"hotspot_f32", 256, "orion_hotspot_f32_256", "hotspot", 32, 8, 128, 128, 1, K_STENCIL, 0, 0},
+    {"hotspot_f32", 128, "orion_hotspot_f32_128", "hotspot", 32, 4, 128, 64, 1, K_STENCIL, 0, 0},
 };
 
 const KernelDef *find_kernel(const char *id, int threads)
