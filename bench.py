@@ -34,12 +34,17 @@ METRIC = "tuned Mpix/s vs max-occupancy build; tuner regret vs exhaustive level 
 # Workloads (BASELINE.json configs).  algorithmic FP32-pipe instructions per output unit
 # of the formulation each kernel implements, and HBM bytes per unit.
 WORKLOADS = {
+    # KNN: 49 taps x (3 FSUB + FMUL + 2 FFMA distance, 1 FFMA exponent, 3 FFMA + 1 FADD
+    # accumulate, 1 compare) + ~10 for the blend
     "c1": dict(kernel="knn_f4", W=64, H=64, sigma=0.2, unit="Mpix/s", name="imageDenoising KNN 64x64 RGBA r=3",
-               insts=49 * 15 + 10, bytes=32),
+               insts=49 * 12 + 10, bytes=32),
+    # NLM box-sum + symmetric pairs, per pixel and offset pair: 1 difference (6), 1 horizontal
+    # and 2 vertical blocked 7-sums (4 each), 2 x (1 FFMA exponent + 3 FFMA + 1 FADD + 1 compare)
     "c2": dict(kernel="nlm_f4", W=2048, H=2048, sigma=0.13, unit="Mpix/s", name="imageDenoising NLM 2048x2048 RGBA",
-               insts=49 * 24 + 10, bytes=32),
+               insts=24 * 30 + 10, bytes=32),
+    # register-heavy direct NLM: 2401 patch terms x 6 + 49 x 6 per-offset terms + blend
     "c4": dict(kernel="nlm_f4_regheavy", W=4096, H=4096, sigma=0.13, unit="Mpix/s",
-               name="register-heavy NLM 4096x4096 RGBA, maxrregcount caps", insts=49 * (49 * 6 + 9) + 10, bytes=32),
+               name="register-heavy NLM 4096x4096 RGBA, maxrregcount caps", insts=2401 * 6 + 49 * 6 + 10, bytes=32),
     "c3": dict(kernel="hotspot_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
                insts=12, bytes=12),
 }
