@@ -1,0 +1,57 @@
+"""Row-sharded multi-GPU composition of the hot path (config C5).
+
+Each rank owns an equal band of output rows, generates its input slab plus the
+R_eff-row halo in place (the generator's hash and the clamping use GLOBAL
+coordinates, so a slab is bit-identical to the same rows of the full image), runs
+its own Orion tuner on that slab (per-GPU tuning), and one NCCL
+``all_gather_into_tensor`` over NVLink collects the output bands -- the only
+inter-GPU exchange of the configuration.
+
+Host-side logic only (partitioning, halo arithmetic, the gather glue); all pixel
+work happens in liborion's kernels.  The gather glue takes any process group, so
+it is exercised with ``gloo`` on CPU tensors in tests/test_shard.py.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+
+@dataclass(frozen=True)
+class Band:
+    rank: int
+    world: int
+    height: int
+    rows_per_rank: int   # equal band height (the last band may be partly past the image)
+    row_begin: int       # first output row owned (global)
+    row_end: int         # one past the last output row owned (global, clipped to height)
+    src_begin: int       # first input row the kernel reads (global, halo included, clamped)
+    src_end: int         # one past the last input row read
+
+    @property
+    def rows(self) -> int:
+        return self.row_end - self.row_begin
+
+    @property
+    def src_rows(self) -> int:
+        return self.src_end - self.src_begin
+
+
+def band(rank: int, world: int, height: int, halo: int) -> Band:
+    """Rank `rank`'s output band and the input rows (with `halo` rows each side) it needs."""
+    if world < 1 or not 0 <= rank < world or height < 1 or halo < 0:
+        raise ValueError("bad band request")
+    per = -(-height // world)
+    r0 = min(height, rank * per)
+    r1 = min(height, r0 + per)
+    return Band(rank, world, height, per, r0, r1, max(0, r0 - halo), min(height, r1 + halo))
+
+
+def gather_bands(out_band, full_out, group=None):
+    """all_gather the equal-height output bands into `full_out` (world * rows_per_rank rows).
+
+    `out_band`: (rows_per_rank, ...) tensor of this rank (rows past the image are padding);
+    `full_out`: (world * rows_per_rank, ...) tensor; rows [0, height) hold the image after.
+    """
+    import torch.distributed as dist
+    dist.all_gather_into_tensor(full_out, out_band.contiguous(), group=group)
+    return full_out
