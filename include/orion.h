@@ -213,6 +213,24 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
                                   void *dev_aux, void *stream, orion_step_report *out,
                                   long long *h2d_bytes, long long *d2h_bytes);
 
+/* Pipelined end-to-end iterations from HOST buffers.  The pipe owns `depth` slots of device
+ * staging buffers (width x max_rows elements each for src, dst and -- stencil -- aux;
+ * allocated here, never in submit) and three non-blocking streams: the H2D copy of frame n,
+ * the kernel of frame n-1 (orion_tune_step on the pipe's compute stream) and the D2H copy of
+ * frame n-2 run concurrently (PCIe is full duplex).  Host buffers must be pinned and must
+ * stay untouched until orion_host_pipe_drain returns.  Errors: ORION_E_INVALID when a frame
+ * does not fit the pipe's width / max_rows; driver errors as ORION_E_CUDA. */
+typedef struct orion_host_pipe orion_host_pipe;   /* opaque, library-owned */
+orion_status orion_host_pipe_create(orion_tuner *t, int width, int max_rows, int depth, orion_host_pipe **out);
+/* Enqueue one iteration: a->src / a->aux / a->dst are HOST pointers laid out as for
+ * orion_launch (src rows [src_row_begin, src_row_end), dst rows from dst_row_begin).
+ * Returns without waiting; bytes copied are reported in *h2d_bytes / *d2h_bytes. */
+orion_status orion_host_pipe_submit(orion_host_pipe *p, const orion_args *a, orion_step_report *out,
+                                    long long *h2d_bytes, long long *d2h_bytes);
+/* Wait until every submitted iteration's output is in host memory. */
+orion_status orion_host_pipe_drain(orion_host_pipe *p);
+void orion_host_pipe_destroy(orion_host_pipe *p);
+
 /* Current ladder: *direction, ladder level indices (ladder[0] = original) -> out[]. */
 orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, int capacity, int *n_out);
 orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final);

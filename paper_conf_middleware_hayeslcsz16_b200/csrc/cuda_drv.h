@@ -20,7 +20,8 @@ namespace orion {
     X(cuModuleGetFunction) X(cuFuncGetAttribute) X(cuFuncSetAttribute) X(cuLaunchKernel)          \
     X(cuOccupancyMaxActiveBlocksPerMultiprocessor) X(cuEventCreate) X(cuEventDestroy)             \
     X(cuEventRecord) X(cuEventSynchronize) X(cuEventElapsedTime) X(cuMemcpyHtoDAsync)             \
-    X(cuMemcpyDtoHAsync) X(cuStreamSynchronize) X(cuGetErrorString) X(cuGetErrorName)
+    X(cuMemcpyDtoHAsync) X(cuStreamSynchronize) X(cuGetErrorString) X(cuGetErrorName)            \
+    X(cuMemAlloc) X(cuMemFree) X(cuStreamCreate) X(cuStreamDestroy) X(cuStreamWaitEvent)
 
 struct Driver {
 #define ORION_DECL(f) decltype(&::f) f = nullptr;

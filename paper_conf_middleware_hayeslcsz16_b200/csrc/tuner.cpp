@@ -307,6 +307,128 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
     return ORION_OK;
 }
 
+}  // extern "C"
+
+// ---- pipelined host-buffer iterations --------------------------------------------------------
+// depth slots of library-owned device staging buffers and three library-owned streams:
+// H2D of frame n+1 and D2H of frame n-1 overlap the kernel of frame n (PCIe is full duplex).
+struct orion_host_pipe {
+    orion_tuner *t = nullptr;
+    int width = 0, max_rows = 0;
+    size_t elem = 16;
+    CUstream s_in = nullptr, s_comp = nullptr, s_out = nullptr;
+    struct Slot {
+        CUdeviceptr src = 0, dst = 0, aux = 0;
+        CUevent ev_in = nullptr, ev_done = nullptr, ev_out = nullptr;
+        bool used = false;
+    };
+    std::vector<Slot> slots;
+    int next = 0;
+};
+
+extern "C" {
+
+void orion_host_pipe_destroy(orion_host_pipe *p)
+{
+    if (!p) return;
+    if (drv().ok) {
+        const Driver &D = drv();
+        for (CUstream s : {p->s_in, p->s_comp, p->s_out})
+            if (s) D.cuStreamSynchronize(s);
+        for (auto &s : p->slots) {
+            for (CUdeviceptr m : {s.src, s.dst, s.aux})
+                if (m) D.cuMemFree(m);
+            for (CUevent e : {s.ev_in, s.ev_done, s.ev_out})
+                if (e) D.cuEventDestroy(e);
+        }
+        for (CUstream s : {p->s_in, p->s_comp, p->s_out})
+            if (s) D.cuStreamDestroy(s);
+    }
+    delete p;
+}
+
+orion_status orion_host_pipe_create(orion_tuner *t, int width, int max_rows, int depth, orion_host_pipe **out)
+{
+    if (!t || !out || width <= 0 || max_rows <= 0 || depth < 1 || depth > 8)
+        return fail(ORION_E_INVALID, "orion_host_pipe_create: bad argument");
+    ORION_TRY(ensure_context(t->v->device));
+    const Driver &D = drv();
+    auto p = new orion_host_pipe();
+    std::unique_ptr<orion_host_pipe, void (*)(orion_host_pipe *)> guard(p, orion_host_pipe_destroy);
+    p->t = t;
+    p->width = width;
+    p->max_rows = max_rows;
+    const bool stencil = t->v->def->kind == K_STENCIL;
+    p->elem = stencil ? 4 : 16;
+    const size_t bytes = (size_t)width * (size_t)max_rows * p->elem;
+    ORION_CU(D.cuStreamCreate(&p->s_in, CU_STREAM_NON_BLOCKING));
+    ORION_CU(D.cuStreamCreate(&p->s_comp, CU_STREAM_NON_BLOCKING));
+    ORION_CU(D.cuStreamCreate(&p->s_out, CU_STREAM_NON_BLOCKING));
+    p->slots.resize(depth);
+    for (auto &s : p->slots) {
+        ORION_CU(D.cuMemAlloc(&s.src, bytes));
+        ORION_CU(D.cuMemAlloc(&s.dst, bytes));
+        if (stencil) ORION_CU(D.cuMemAlloc(&s.aux, bytes));
+        ORION_CU(D.cuEventCreate(&s.ev_in, CU_EVENT_DISABLE_TIMING));
+        ORION_CU(D.cuEventCreate(&s.ev_done, CU_EVENT_DISABLE_TIMING));
+        ORION_CU(D.cuEventCreate(&s.ev_out, CU_EVENT_DISABLE_TIMING));
+    }
+    *out = guard.release();
+    return ORION_OK;
+}
+
+orion_status orion_host_pipe_submit(orion_host_pipe *p, const orion_args *a, orion_step_report *out,
+                                    long long *h2d, long long *d2h)
+{
+    if (!p || !a || !a->src || !a->dst) return fail(ORION_E_INVALID, "orion_host_pipe_submit: NULL");
+    const int in_rows = a->src_row_end - a->src_row_begin;
+    const int out_rows = a->row_end - a->row_begin;
+    if (a->width != p->width || in_rows < 0 || in_rows > p->max_rows || out_rows < 0 || out_rows > p->max_rows ||
+        a->dst_row_begin > a->row_begin || (p->t->v->def->kind == K_STENCIL && !a->aux))
+        return fail(ORION_E_INVALID, "orion_host_pipe_submit: frame does not fit the pipe");
+    const Driver &D = drv();
+    ORION_TRY(ensure_context(p->t->v->device));
+    auto &s = p->slots[p->next];
+    p->next = (p->next + 1) % (int)p->slots.size();
+    const size_t row = (size_t)a->width * p->elem;
+    const size_t in_bytes = (size_t)in_rows * row, out_bytes = (size_t)out_rows * row;
+    if (s.used) ORION_CU(D.cuStreamWaitEvent(p->s_in, s.ev_out, 0));   // slot free again
+    ORION_CU(D.cuMemcpyHtoDAsync(s.src, a->src, in_bytes, p->s_in));
+    size_t aux_bytes = 0;
+    if (s.aux) {
+        aux_bytes = in_bytes;
+        ORION_CU(D.cuMemcpyHtoDAsync(s.aux, a->aux, aux_bytes, p->s_in));
+    }
+    ORION_CU(D.cuEventRecord(s.ev_in, p->s_in));
+    ORION_CU(D.cuStreamWaitEvent(p->s_comp, s.ev_in, 0));
+    orion_args da = *a;
+    da.src = (const void *)s.src;
+    da.dst = (void *)s.dst;
+    da.aux = (const void *)s.aux;
+    da.dst_row_begin = a->row_begin;
+    ORION_TRY(orion_tune_step(p->t, &da, p->s_comp, out));
+    ORION_CU(D.cuEventRecord(s.ev_done, p->s_comp));
+    ORION_CU(D.cuStreamWaitEvent(p->s_out, s.ev_done, 0));
+    ORION_CU(D.cuMemcpyDtoHAsync((char *)a->dst + (size_t)(a->row_begin - a->dst_row_begin) * row, s.dst, out_bytes,
+                                 p->s_out));
+    ORION_CU(D.cuEventRecord(s.ev_out, p->s_out));
+    s.used = true;
+    if (h2d) *h2d = (long long)(in_bytes + aux_bytes);
+    if (d2h) *d2h = (long long)out_bytes;
+    return ORION_OK;
+}
+
+orion_status orion_host_pipe_drain(orion_host_pipe *p)
+{
+    if (!p) return fail(ORION_E_INVALID, "orion_host_pipe_drain: NULL");
+    ORION_TRY(ensure_context(p->t->v->device));
+    const Driver &D = drv();
+    ORION_CU(D.cuStreamSynchronize(p->s_in));
+    ORION_CU(D.cuStreamSynchronize(p->s_comp));
+    ORION_CU(D.cuStreamSynchronize(p->s_out));
+    return ORION_OK;
+}
+
 orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, int capacity, int *n_out)
 {
     if (!t || !n_out || capacity < 0 || (capacity > 0 && !out)) return fail(ORION_E_INVALID, "orion_tuner_ladder");

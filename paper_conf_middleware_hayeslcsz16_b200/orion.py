@@ -120,6 +120,9 @@ def lib() -> ctypes.CDLL:
                 "orion_tune_step": [V, P(Args), V, P(StepReport)],
                 "orion_tune_step_host": [V, P(Args), V, V, V, V, P(StepReport), P(ctypes.c_longlong),
                                          P(ctypes.c_longlong)],
+                "orion_host_pipe_create": [V, I, I, I, P(V)],
+                "orion_host_pipe_submit": [V, P(Args), P(StepReport), P(ctypes.c_longlong), P(ctypes.c_longlong)],
+                "orion_host_pipe_drain": [V],
                 "orion_tuner_ladder": [V, P(I), P(I), I, P(I)],
                 "orion_tuner_final": [V, P(I), P(I)],
                 "orion_tuner_replay": [P(TunerCfg), P(Level), I, I, P(ctypes.c_float), I, P(I), P(I), P(I)],
@@ -131,7 +134,7 @@ def lib() -> ctypes.CDLL:
                 f = getattr(L, name)
                 f.argtypes = args
                 f.restype = ctypes.c_int
-            for name in ("orion_variants_destroy", "orion_tuner_destroy"):
+            for name in ("orion_variants_destroy", "orion_tuner_destroy", "orion_host_pipe_destroy"):
                 getattr(L, name).argtypes = [V]
                 getattr(L, name).restype = None
             L.orion_status_str.restype = ctypes.c_char_p
@@ -354,6 +357,38 @@ class Tuner:
     def close(self):
         if getattr(self, "h", None):
             lib().orion_tuner_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class HostPipe:
+    """orion_host_pipe handle: pipelined iterations from pinned host buffers."""
+
+    def __init__(self, tuner: Tuner, width: int, max_rows: int, depth: int = 2):
+        self.tuner = tuner
+        h = ctypes.c_void_p()
+        _check(lib().orion_host_pipe_create(tuner.h, width, max_rows, depth, ctypes.byref(h)),
+               "orion_host_pipe_create")
+        self.h = h
+
+    def submit(self, args: Args):
+        r = StepReport()
+        hi, ho = ctypes.c_longlong(), ctypes.c_longlong()
+        _check(lib().orion_host_pipe_submit(self.h, ctypes.byref(args), ctypes.byref(r), ctypes.byref(hi),
+                                            ctypes.byref(ho)), "orion_host_pipe_submit")
+        return r, hi.value, ho.value
+
+    def drain(self):
+        _check(lib().orion_host_pipe_drain(self.h), "orion_host_pipe_drain")
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().orion_host_pipe_destroy(self.h)
             self.h = None
 
     def __del__(self):
