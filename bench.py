@@ -209,7 +209,7 @@ def run_ours(args):
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream
     wl = WORKLOADS[args.workload]
-    kernel, W, H = wl["kernel"], wl["W"], wl["H"]
+    kernel, W, H = args.kernel or wl["kernel"], wl["W"], wl["H"]
     is_stencil = kernel == "hotspot_f32"
 
     # ---- multi-version binary: probe -> levels -> build (offline, untimed) ----------------
@@ -518,6 +518,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
+    ap.add_argument("--kernel", default="", help="override the workload's kernel id (same family)")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")

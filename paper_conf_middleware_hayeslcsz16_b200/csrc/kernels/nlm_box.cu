@@ -10,24 +10,28 @@
 // (2) d_{-o}(u,v) = d_o(u-j, v-i), hence D_{-o}(x,y) = D_o(x-j, y-i): one box sum serves
 //     the offset pair (o, -o).  The 48 non-centre offsets form 24 pairs; the centre
 //     offset has D = 0, w = 1 exactly.
-// Both are exact identities; only the order of the fp32 additions differs from the
+// (3) Pairs sharing the row offset i and consecutive column offsets j = j1 .. j1+G-1
+//     are processed in one pass: along a phase-A row the shifted pixels p(u+j, v+i) of
+//     the G offsets form a sliding window, so each new column costs one shifted load for
+//     all G differences (and one centre load), instead of G of each.
+// All three are exact identities; only the order of the fp32 additions differs from the
 // definition (every partial sum is a sum of non-negative terms, at most 4 roundings
-// deep: see DESIGN.md §nlm_f4 for the error budget against the 1e-5 tolerance).
+// deep: DESIGN.md §7 gives the error budget against the 1e-5 tolerance).
 //
 // CTA = 128 threads (4 warps); output tile TW = 122 columns x TH = 23 rows.
 // Shared memory: the input tile (TW+18) x (TH+12) with a 9-column / 6-row
-// clamp-to-edge halo as three planar fp32 arrays (odd pitch), and one H_o buffer of
-// 32 rows x 128 columns (odd pitch).  Per offset pair:
-//   phase A: warp w computes H_o for columns [32w, 32w+32) of the H buffer; lane = row
-//            (32 rows = TH + 9), sliding along the row over 38 difference values.
-//            Lanes touch 32 different rows of an odd-pitch array: conflict-free.
+// clamp-to-edge halo as three planar fp32 arrays (odd pitch), and GMAX buffers of
+// H_o, 32 rows x 128 columns each (odd pitch).  Per pass:
+//   phase A: warp w computes H_o for columns [32w, 32w+32) of each buffer; lane = row
+//            (32 rows = TH + 9), sliding along the row over 38 difference values per
+//            offset.  Lanes touch 32 different rows of odd-pitch arrays: conflict-free.
 //   phase B: thread t owns output column x0+t and all TH rows: vertical 7-sums of
 //            H_o down column t+3 give D_o(x, .), and down column t+3-j, shifted by -i
 //            rows, give D_{-o}(x, .); weights w = 2^(D * (-Noise log2 e) + geo) and
 //            the accumulation of w*p, w and [w > wthr] for both offsets.  Lanes touch
 //            consecutive columns: conflict-free.
-// Two __syncthreads per pair.  ~4 LDS per pixel-offset in phase B, ~0.9 difference
-// evaluations per pixel-offset in phase A (vs 49 patch terms in the direct form).
+// Two __syncthreads per pass.  GMAX = 1: 24 passes, 75.7 KB smem (3 CTAs/SM);
+// GMAX = 3: 10 passes, 108.8 KB smem (2 CTAs/SM), ~2.4x fewer phase-A loads.
 #include "common.cuh"
 
 #define PB_R 3   // window radius
@@ -42,6 +46,7 @@ constexpr int HP = HC + 1;                  // odd H pitch
 constexpr int PC = TW + 18;                 // image tile columns: x0-9 .. x0+TW+9
 constexpr int PR = TH + 12;                 // image tile rows:    y0-6 .. y0+TH+6
 constexpr int PW = PC + 1;                  // odd plane pitch
+constexpr int HBUF = AR * HP;               // floats per H buffer
 static_assert(AR == 32 && HC == 4 * 32 && NT == 128, "phase A: one lane per row, one warp per 32 H columns");
 static_assert(TW <= NT, "phase B: one thread per output column");
 
@@ -59,15 +64,112 @@ ORION_DEVICE void window7(const float (&a)[N + 6], float (&out)[N])
         out[k] = __fadd_rn(__fadd_rn(p[k], p[k + 2]), __fadd_rn(p[k + 4], a[k + 6]));
 }
 
-}  // namespace
+ORION_DEVICE float diff2(float ar, float ag, float ab, float br, float bg, float bb)
+{
+    const float dx = __fsub_rn(ar, br), dy = __fsub_rn(ag, bg), dz = __fsub_rn(ab, bb);
+    return __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));
+}
 
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kargs a)
+// Phase A for G offsets (i, j1 .. j1+G-1): lane = row r, warp's 32 H columns.
+template <int G>
+ORION_DEVICE void phase_a(const float *pr, const float *pg, const float *pb, float *hs, int lane, int warp, int i,
+                          int j1)
+{
+    const int cb = 3 + 32 * warp;               // tile column of u for the first difference
+    const int rowc = lane * PW + cb;            // centre p(u, v)
+    const int rows = rowc + i * PW + j1;        // shifted p(u+j1, v+i)
+    // the shifted window holds columns q + j1 .. q + j1 + G - 1 at step q
+    float wr[G], wg[G], wb[G];
+#pragma unroll
+    for (int g = 0; g < G - 1; ++g) {
+        wr[g + 1] = pr[rows + g];
+        wg[g + 1] = pg[rows + g];
+        wb[g + 1] = pb[rows + g];
+    }
+    float d[G][38];
+#pragma unroll
+    for (int q = 0; q < 38; ++q) {
+#pragma unroll
+        for (int g = 0; g < G - 1; ++g) {
+            wr[g] = wr[g + 1];
+            wg[g] = wg[g + 1];
+            wb[g] = wb[g + 1];
+        }
+        wr[G - 1] = pr[rows + q + G - 1];
+        wg[G - 1] = pg[rows + q + G - 1];
+        wb[G - 1] = pb[rows + q + G - 1];
+        const float cr = pr[rowc + q], cg = pg[rowc + q], cbv = pb[rowc + q];
+#pragma unroll
+        for (int g = 0; g < G; ++g) d[g][q] = diff2(wr[g], wg[g], wb[g], cr, cg, cbv);
+    }
+#pragma unroll
+    for (int g = 0; g < G; ++g) {
+        float h[32];
+        window7<32>(d[g], h);
+        float *hrow = hs + g * HBUF + lane * HP + 32 * warp;
+#pragma unroll
+        for (int q = 0; q < 32; ++q) hrow[q] = h[q];
+    }
+}
+
+struct Acc {
+    float ax[TH], ay[TH], az[TH], sw[TH];
+    unsigned cnt[(TH + 3) / 4];   // 4 x 8-bit counts per word (<= 49)
+};
+
+// Phase B for one pair (i, j) whose H_o lives in hb: thread t = output column x0+t.
+ORION_DEVICE void phase_b(const float *pr, const float *pg, const float *pb, const float *hb, int t, int i, int j,
+                          float nl2, float wthr, Acc &A)
+{
+    const float geo = geo_l2_rt(i, j);
+    float hv[TH + 6], D[TH];
+    // +o: D_o(x, y) = sum_n H_o(x, y+n): H column t+3, rows 3 .. TH+8
+#pragma unroll
+    for (int q = 0; q < TH + 6; ++q) hv[q] = hb[(q + 3) * HP + t + 3];
+    window7<TH>(hv, D);
+#pragma unroll
+    for (int r = 0; r < TH; ++r) {
+        const float w = exp2f(__fmaf_rn(D[r], nl2, geo));
+        const int pc = (r + 6 + i) * PW + t + 9 + j;
+        A.ax[r] = __fmaf_rn(w, pr[pc], A.ax[r]);
+        A.ay[r] = __fmaf_rn(w, pg[pc], A.ay[r]);
+        A.az[r] = __fmaf_rn(w, pb[pc], A.az[r]);
+        A.sw[r] = __fadd_rn(A.sw[r], w);
+        A.cnt[r >> 2] += (w > wthr) ? (1u << (8 * (r & 3))) : 0u;
+    }
+    // -o: D_{-o}(x, y) = D_o(x-j, y-i): H column t+3-j, rows 3-i .. TH+8-i
+#pragma unroll
+    for (int q = 0; q < TH + 6; ++q) hv[q] = hb[(q + 3 - i) * HP + t + 3 - j];
+    window7<TH>(hv, D);
+#pragma unroll
+    for (int r = 0; r < TH; ++r) {
+        const float w = exp2f(__fmaf_rn(D[r], nl2, geo));
+        const int pc = (r + 6 - i) * PW + t + 9 - j;
+        A.ax[r] = __fmaf_rn(w, pr[pc], A.ax[r]);
+        A.ay[r] = __fmaf_rn(w, pg[pc], A.ay[r]);
+        A.az[r] = __fmaf_rn(w, pb[pc], A.az[r]);
+        A.sw[r] = __fadd_rn(A.sw[r], w);
+        A.cnt[r >> 2] += (w > wthr) ? (1u << (8 * (r & 3))) : 0u;
+    }
+}
+
+// Pass tables: (i, j1, G).  Together they cover the 24 half-plane pairs exactly once.
+__constant__ int kPass1[24][3] = {
+    {0, 1, 1}, {0, 2, 1}, {0, 3, 1},
+    {1, -3, 1}, {1, -2, 1}, {1, -1, 1}, {1, 0, 1}, {1, 1, 1}, {1, 2, 1}, {1, 3, 1},
+    {2, -3, 1}, {2, -2, 1}, {2, -1, 1}, {2, 0, 1}, {2, 1, 1}, {2, 2, 1}, {2, 3, 1},
+    {3, -3, 1}, {3, -2, 1}, {3, -1, 1}, {3, 0, 1}, {3, 1, 1}, {3, 2, 1}, {3, 3, 1}};
+__constant__ int kPass3[10][3] = {
+    {0, 1, 3}, {1, -3, 3}, {1, 0, 2}, {1, 2, 2}, {2, -3, 3}, {2, 0, 2}, {2, 2, 2}, {3, -3, 3}, {3, 0, 2}, {3, 2, 2}};
+
+template <int GMAX>
+__device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 {
     extern __shared__ float4 smem4[];
     float *pr = reinterpret_cast<float *>(smem4);
     float *pg = pr + PR * PW;
     float *pb = pg + PR * PW;
-    float *hs = pb + PR * PW;               // H_o: AR rows x HP
+    float *hs = pb + PR * PW;               // GMAX buffers of H_o: AR rows x HP
 
     const int tid = threadIdx.x;
     const int lane = tid & 31, warp = tid >> 5;
@@ -89,82 +191,38 @@ extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kar
 
     const float nl2 = a.fparam[0];
     const float wthr = a.fparam[2];
-    // phase-B state: column t, rows 0..TH-1.  Counts are packed 4 x 8 bits per word (<= 49).
     const int t = tid;
-    float ax[TH], ay[TH], az[TH], sw[TH];
-    unsigned cnt[(TH + 3) / 4];
+    Acc A;
     {
         const unsigned c1 = (1.0f > wthr) ? 1u : 0u;   // centre offset: D = 0, w = 1 exactly
 #pragma unroll
         for (int r = 0; r < TH; ++r) {
             const int pc = (r + 6) * PW + t + 9;
-            ax[r] = pr[pc];
-            ay[r] = pg[pc];
-            az[r] = pb[pc];
-            sw[r] = 1.0f;
+            A.ax[r] = pr[pc];
+            A.ay[r] = pg[pc];
+            A.az[r] = pb[pc];
+            A.sw[r] = 1.0f;
         }
 #pragma unroll
-        for (int q = 0; q < (TH + 3) / 4; ++q) cnt[q] = c1 * 0x01010101u;
+        for (int q = 0; q < (TH + 3) / 4; ++q) A.cnt[q] = c1 * 0x01010101u;
     }
 
+    constexpr int NPASS = GMAX == 1 ? 24 : 10;
 #pragma unroll 1
-    for (int pi = 0; pi < 24; ++pi) {
-        // half-plane pair representative o = (i, j): (0,1..3) then (1..3, -3..3)
-        const int i = pi < 3 ? 0 : (pi - 3) / 7 + 1;
-        const int j = pi < 3 ? pi + 1 : (pi - 3) % 7 - 3;
-        // ---- phase A: H_o(u, v) for this warp's 32 columns, lane = row -------------------
-        {
-            const int r = lane;                           // tile row of v (y0-6+r)
-            const int cb = 3 + 32 * warp;                 // tile column of u for the first d
-            const float *cr = pr + r * PW + cb, *cg = pg + r * PW + cb, *cbp = pb + r * PW + cb;
-            const int so = i * PW + j;                    // shift to p(u+j, v+i)
-            float d[38];
-#pragma unroll
-            for (int q = 0; q < 38; ++q) {
-                const float dx = __fsub_rn(cr[q + so], cr[q]);
-                const float dy = __fsub_rn(cg[q + so], cg[q]);
-                const float dz = __fsub_rn(cbp[q + so], cbp[q]);
-                d[q] = __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));
-            }
-            float h[32];
-            window7<32>(d, h);
-            float *hrow = hs + r * HP + 32 * warp;
-#pragma unroll
-            for (int q = 0; q < 32; ++q) hrow[q] = h[q];
-        }
+    for (int ps = 0; ps < NPASS; ++ps) {
+        const int i = GMAX == 1 ? kPass1[ps][0] : kPass3[ps][0];
+        const int j1 = GMAX == 1 ? kPass1[ps][1] : kPass3[ps][1];
+        const int G = GMAX == 1 ? 1 : kPass3[ps][2];
+        if (GMAX == 1 || G == 1)
+            phase_a<1>(pr, pg, pb, hs, lane, warp, i, j1);
+        else if (G == 2)
+            phase_a<2>(pr, pg, pb, hs, lane, warp, i, j1);
+        else
+            phase_a<(GMAX >= 3 ? 3 : 1)>(pr, pg, pb, hs, lane, warp, i, j1);
         __syncthreads();
-        // ---- phase B: vertical sums for +o and -o, weights, accumulation -----------------
         if (t < TW) {
-            const float geo = geo_l2_rt(i, j);
-            float hv[TH + 6], D[TH];
-            // +o: D_o(x, y) = sum_n H_o(x, y+n): H column t+3, rows 3 .. TH+8
-#pragma unroll
-            for (int q = 0; q < TH + 6; ++q) hv[q] = hs[(q + 3) * HP + t + 3];
-            window7<TH>(hv, D);
-#pragma unroll
-            for (int r = 0; r < TH; ++r) {
-                const float w = exp2f(__fmaf_rn(D[r], nl2, geo));
-                const int pc = (r + 6 + i) * PW + t + 9 + j;
-                ax[r] = __fmaf_rn(w, pr[pc], ax[r]);
-                ay[r] = __fmaf_rn(w, pg[pc], ay[r]);
-                az[r] = __fmaf_rn(w, pb[pc], az[r]);
-                sw[r] = __fadd_rn(sw[r], w);
-                cnt[r >> 2] += (w > wthr) ? (1u << (8 * (r & 3))) : 0u;
-            }
-            // -o: D_{-o}(x, y) = D_o(x-j, y-i): H column t+3-j, rows 3-i .. TH+8-i
-#pragma unroll
-            for (int q = 0; q < TH + 6; ++q) hv[q] = hs[(q + 3 - i) * HP + t + 3 - j];
-            window7<TH>(hv, D);
-#pragma unroll
-            for (int r = 0; r < TH; ++r) {
-                const float w = exp2f(__fmaf_rn(D[r], nl2, geo));
-                const int pc = (r + 6 - i) * PW + t + 9 - j;
-                ax[r] = __fmaf_rn(w, pr[pc], ax[r]);
-                ay[r] = __fmaf_rn(w, pg[pc], ay[r]);
-                az[r] = __fmaf_rn(w, pb[pc], az[r]);
-                sw[r] = __fadd_rn(sw[r], w);
-                cnt[r >> 2] += (w > wthr) ? (1u << (8 * (r & 3))) : 0u;
-            }
+#pragma unroll 1
+            for (int g = 0; g < G; ++g) phase_b(pr, pg, pb, hs + g * HBUF, t, i, j1 + g, nl2, wthr, A);
         }
         __syncthreads();
     }
@@ -177,7 +235,14 @@ extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kar
         if (y >= a.row_end) break;
         const int pc = (r + 6) * PW + t + 9;
         const float4 c00 = make_float4(pr[pc], pg[pc], pb[pc], 0.0f);
-        const int c = (int)((cnt[r >> 2] >> (8 * (r & 3))) & 0xffu);
-        dst[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = lerp_out(c00, ax[r], ay[r], az[r], sw[r], c, a);
+        const int c = (int)((A.cnt[r >> 2] >> (8 * (r & 3))) & 0xffu);
+        dst[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = lerp_out(c00, A.ax[r], A.ay[r], A.az[r], A.sw[r], c, a);
     }
 }
+
+}  // namespace
+
+// One pair per pass: 3 planar planes + 1 H buffer = 75 732 B of shared memory.
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kargs a) { nlm_box_body<1>(a); }
+// Up to three pairs per pass: 3 planar planes + 3 H buffers = 108 756 B of shared memory.
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_box3_f4_128(orion_kargs a) { nlm_box_body<3>(a); }
