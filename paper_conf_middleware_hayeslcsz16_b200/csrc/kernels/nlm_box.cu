@@ -50,18 +50,26 @@ constexpr int HBUF = AR * HP;               // floats per H buffer
 static_assert(AR == 32 && HC == 4 * 32 && NT == 128, "phase A: one lane per row, one warp per 32 H columns");
 static_assert(TW <= NT, "phase B: one thread per output column");
 
+// Packed fp32x2 arithmetic (sm_100 FADD2 / FMUL2 / FFMA2): two independent IEEE
+// round-to-nearest operations per instruction, bit-identical to the scalar .rn forms.
+ORION_DEVICE float2 sub2(float2 a, float2 b) { return __fadd2_rn(a, make_float2(-b.x, -b.y)); }
+ORION_DEVICE float2 mul2(float2 a, float2 b) { return __fmul2_rn(a, b); }
+ORION_DEVICE float2 fma2(float2 a, float2 b, float2 c) { return __ffma2_rn(a, b, c); }
+ORION_DEVICE float add1(float a, float b) { return __fadd_rn(a, b); }
+ORION_DEVICE float2 add1(float2 a, float2 b) { return __fadd2_rn(a, b); }
+
 // Blocked 7-term window sums of a[0 .. N+5]: out[k] = a[k] + ... + a[k+6] evaluated as
 // ((a[k]+a[k+1]) + (a[k+2]+a[k+3])) + ((a[k+4]+a[k+5]) + a[k+6]) -- 4 additions per
 // output with the pair sums shared; every partial sum is a sum of non-negatives.
-template <int N>
-ORION_DEVICE void window7(const float (&a)[N + 6], float (&out)[N])
+// T = float, or float2 for two independent windows in lock step.
+template <int N, typename T>
+ORION_DEVICE void window7(const T (&a)[N + 6], T (&out)[N])
 {
-    float p[N + 5];
+    T p[N + 5];
 #pragma unroll
-    for (int k = 0; k < N + 5; ++k) p[k] = __fadd_rn(a[k], a[k + 1]);
+    for (int k = 0; k < N + 5; ++k) p[k] = add1(a[k], a[k + 1]);
 #pragma unroll
-    for (int k = 0; k < N; ++k)
-        out[k] = __fadd_rn(__fadd_rn(p[k], p[k + 2]), __fadd_rn(p[k + 4], a[k + 6]));
+    for (int k = 0; k < N; ++k) out[k] = add1(add1(p[k], p[k + 2]), add1(p[k + 4], a[k + 6]));
 }
 
 ORION_DEVICE float diff2(float ar, float ag, float ab, float br, float bg, float bb)
@@ -70,7 +78,15 @@ ORION_DEVICE float diff2(float ar, float ag, float ab, float br, float bg, float
     return __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));
 }
 
-// Phase A for G offsets (i, j1 .. j1+G-1): lane = row r, warp's 32 H columns.
+ORION_DEVICE float2 diff2x2(float2 ar, float2 ag, float2 ab, float br, float bg, float bb)
+{
+    const float2 dx = sub2(ar, make_float2(br, br)), dy = sub2(ag, make_float2(bg, bg)),
+                 dz = sub2(ab, make_float2(bb, bb));
+    return fma2(dz, dz, fma2(dy, dy, mul2(dx, dx)));
+}
+
+// Phase A for G offsets (i, j1 .. j1+G-1): lane = row r, warp's 32 H columns.  Offsets
+// g = 0, 1 run packed (fp32x2), offset g = 2 scalar.
 template <int G>
 ORION_DEVICE void phase_a(const float *pr, const float *pg, const float *pb, float *hs, int lane, int warp, int i,
                           int j1)
@@ -86,7 +102,10 @@ ORION_DEVICE void phase_a(const float *pr, const float *pg, const float *pb, flo
         wg[g + 1] = pg[rows + g];
         wb[g + 1] = pb[rows + g];
     }
-    float d[G][38];
+    constexpr int GP = G / 2;                   // packed offset pairs (0 or 1)
+    constexpr int GS = G - 2 * GP;              // scalar offsets left (0 or 1)
+    float2 dp[GP > 0 ? 38 : 1];
+    float ds[GS > 0 ? 38 : 1];
 #pragma unroll
     for (int q = 0; q < 38; ++q) {
 #pragma unroll
@@ -99,57 +118,62 @@ ORION_DEVICE void phase_a(const float *pr, const float *pg, const float *pb, flo
         wg[G - 1] = pg[rows + q + G - 1];
         wb[G - 1] = pb[rows + q + G - 1];
         const float cr = pr[rowc + q], cg = pg[rowc + q], cbv = pb[rowc + q];
-#pragma unroll
-        for (int g = 0; g < G; ++g) d[g][q] = diff2(wr[g], wg[g], wb[g], cr, cg, cbv);
+        if (GP > 0)
+            dp[GP > 0 ? q : 0] = diff2x2(make_float2(wr[0], wr[GP > 0 ? 1 : 0]), make_float2(wg[0], wg[GP > 0 ? 1 : 0]),
+                                         make_float2(wb[0], wb[GP > 0 ? 1 : 0]), cr, cg, cbv);
+        if (GS > 0) ds[GS > 0 ? q : 0] = diff2(wr[G - 1], wg[G - 1], wb[G - 1], cr, cg, cbv);
     }
+    if (GP > 0) {
+        float2 h[32];
+        window7<32>(*reinterpret_cast<float2(*)[38]>(&dp), h);
+        float *h0 = hs + lane * HP + 32 * warp;
+        float *h1 = h0 + HBUF;
 #pragma unroll
-    for (int g = 0; g < G; ++g) {
+        for (int q = 0; q < 32; ++q) {
+            h0[q] = h[q].x;
+            h1[q] = h[q].y;
+        }
+    }
+    if (GS > 0) {
         float h[32];
-        window7<32>(d[g], h);
-        float *hrow = hs + g * HBUF + lane * HP + 32 * warp;
+        window7<32>(*reinterpret_cast<float(*)[38]>(&ds), h);
+        float *h2 = hs + (G - 1) * HBUF + lane * HP + 32 * warp;
 #pragma unroll
-        for (int q = 0; q < 32; ++q) hrow[q] = h[q];
+        for (int q = 0; q < 32; ++q) h2[q] = h[q];
     }
 }
 
 struct Acc {
-    float ax[TH], ay[TH], az[TH], sw[TH];
+    float2 axy[TH];               // (sum w*r, sum w*g)
+    float2 azs[TH];               // (sum w*b, sum w)
     unsigned cnt[(TH + 3) / 4];   // 4 x 8-bit counts per word (<= 49)
 };
 
-// Phase B for one pair (i, j) whose H_o lives in hb: thread t = output column x0+t.
+// Phase B for one pair (i, j) whose H_o lives in hb: thread t = output column x0+t.  The
+// +o and -o vertical windows run packed (fp32x2), as do their exponent arguments and the
+// (r, g) / (b, weight) accumulations.
 ORION_DEVICE void phase_b(const float *pr, const float *pg, const float *pb, const float *hb, int t, int i, int j,
                           float nl2, float wthr, Acc &A)
 {
     const float geo = geo_l2_rt(i, j);
-    float hv[TH + 6], D[TH];
-    // +o: D_o(x, y) = sum_n H_o(x, y+n): H column t+3, rows 3 .. TH+8
+    // x: D_o(x, y) = sum_n H_o(x, y+n) -- H column t+3, rows 3 .. TH+8
+    // y: D_{-o}(x, y) = D_o(x-j, y-i)  -- H column t+3-j, rows 3-i .. TH+8-i
+    float2 hv[TH + 6], D[TH];
 #pragma unroll
-    for (int q = 0; q < TH + 6; ++q) hv[q] = hb[(q + 3) * HP + t + 3];
+    for (int q = 0; q < TH + 6; ++q) hv[q] = make_float2(hb[(q + 3) * HP + t + 3], hb[(q + 3 - i) * HP + t + 3 - j]);
     window7<TH>(hv, D);
+    const float2 n2 = make_float2(nl2, nl2), g2 = make_float2(geo, geo);
 #pragma unroll
     for (int r = 0; r < TH; ++r) {
-        const float w = exp2f(__fmaf_rn(D[r], nl2, geo));
-        const int pc = (r + 6 + i) * PW + t + 9 + j;
-        A.ax[r] = __fmaf_rn(w, pr[pc], A.ax[r]);
-        A.ay[r] = __fmaf_rn(w, pg[pc], A.ay[r]);
-        A.az[r] = __fmaf_rn(w, pb[pc], A.az[r]);
-        A.sw[r] = __fadd_rn(A.sw[r], w);
-        A.cnt[r >> 2] += (w > wthr) ? (1u << (8 * (r & 3))) : 0u;
-    }
-    // -o: D_{-o}(x, y) = D_o(x-j, y-i): H column t+3-j, rows 3-i .. TH+8-i
-#pragma unroll
-    for (int q = 0; q < TH + 6; ++q) hv[q] = hb[(q + 3 - i) * HP + t + 3 - j];
-    window7<TH>(hv, D);
-#pragma unroll
-    for (int r = 0; r < TH; ++r) {
-        const float w = exp2f(__fmaf_rn(D[r], nl2, geo));
-        const int pc = (r + 6 - i) * PW + t + 9 - j;
-        A.ax[r] = __fmaf_rn(w, pr[pc], A.ax[r]);
-        A.ay[r] = __fmaf_rn(w, pg[pc], A.ay[r]);
-        A.az[r] = __fmaf_rn(w, pb[pc], A.az[r]);
-        A.sw[r] = __fadd_rn(A.sw[r], w);
-        A.cnt[r >> 2] += (w > wthr) ? (1u << (8 * (r & 3))) : 0u;
+        const float2 e = fma2(D[r], n2, g2);
+        const float wp = exp2f(e.x), wm = exp2f(e.y);
+        const int pp = (r + 6 + i) * PW + t + 9 + j;      // p(x+j, y+i)
+        const int pm = (r + 6 - i) * PW + t + 9 - j;      // p(x-j, y-i)
+        A.axy[r] = fma2(make_float2(wp, wp), make_float2(pr[pp], pg[pp]), A.axy[r]);
+        A.azs[r] = fma2(make_float2(wp, wp), make_float2(pb[pp], 1.0f), A.azs[r]);
+        A.axy[r] = fma2(make_float2(wm, wm), make_float2(pr[pm], pg[pm]), A.axy[r]);
+        A.azs[r] = fma2(make_float2(wm, wm), make_float2(pb[pm], 1.0f), A.azs[r]);
+        A.cnt[r >> 2] += (((wp > wthr) ? 1u : 0u) + ((wm > wthr) ? 1u : 0u)) << (8 * (r & 3));
     }
 }
 
@@ -198,10 +222,8 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 #pragma unroll
         for (int r = 0; r < TH; ++r) {
             const int pc = (r + 6) * PW + t + 9;
-            A.ax[r] = pr[pc];
-            A.ay[r] = pg[pc];
-            A.az[r] = pb[pc];
-            A.sw[r] = 1.0f;
+            A.axy[r] = make_float2(pr[pc], pg[pc]);
+            A.azs[r] = make_float2(pb[pc], 1.0f);
         }
 #pragma unroll
         for (int q = 0; q < (TH + 3) / 4; ++q) A.cnt[q] = c1 * 0x01010101u;
@@ -236,7 +258,7 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
         const int pc = (r + 6) * PW + t + 9;
         const float4 c00 = make_float4(pr[pc], pg[pc], pb[pc], 0.0f);
         const int c = (int)((A.cnt[r >> 2] >> (8 * (r & 3))) & 0xffu);
-        dst[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = lerp_out(c00, A.ax[r], A.ay[r], A.az[r], A.sw[r], c, a);
+        dst[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = lerp_out(c00, A.axy[r].x, A.axy[r].y, A.azs[r].x, A.azs[r].y, c, a);
     }
 }
 
