@@ -54,6 +54,16 @@ ORION_DEVICE float4 lerp_out(float4 c00, float ax, float ay, float az, float sw,
 }
 
 
+// 2^x on the SFU (MUFU.EX2, ~2 ulp), flushing sub-normal results to zero: the weights
+// that small (< 2^-126) are below every threshold and vanish in the weight sums, which
+// always hold the centre weight 1.  Saves exp2f's sub-normal rescaling (FSETP + 2 FMUL).
+ORION_DEVICE float ex2(float x)
+{
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+
 // Same term evaluated at run time: (i*i + j*j) * (-log2(e)/49) with one rounding.
 ORION_DEVICE float geo_l2_rt(int i, int j)
 {

@@ -51,7 +51,7 @@ __device__ __forceinline__ void knn_body(const orion_kargs &a)
                 if (i < -KNN_R || i > KNN_R) continue; // resolved at compile time
                 const int j = jj - KNN_R;
                 const float d = dist2(c, c00[p]);
-                const float w = exp2f(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
+                const float w = ex2(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
                 ax[p] = __fmaf_rn(w, c.x, ax[p]);
                 ay[p] = __fmaf_rn(w, c.y, ay[p]);
                 az[p] = __fmaf_rn(w, c.z, az[p]);

@@ -166,7 +166,7 @@ ORION_DEVICE void phase_b(const float *pr, const float *pg, const float *pb, con
 #pragma unroll
     for (int r = 0; r < TH; ++r) {
         const float2 e = fma2(D[r], n2, g2);
-        const float wp = exp2f(e.x), wm = exp2f(e.y);
+        const float wp = ex2(e.x), wm = ex2(e.y);
         const int pp = (r + 6 + i) * PW + t + 9 + j;      // p(x+j, y+i)
         const int pm = (r + 6 - i) * PW + t + 9 - j;      // p(x-j, y-i)
         A.axy[r] = fma2(make_float2(wp, wp), make_float2(pr[pp], pg[pp]), A.axy[r]);

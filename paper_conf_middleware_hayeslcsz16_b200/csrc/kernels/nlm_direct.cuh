@@ -49,7 +49,7 @@ __device__ __forceinline__ void nlm_direct_body(const orion_kargs &a)
                     d = __fadd_rn(d, dist2(s, c));
                 }
             }
-            const float w = exp2f(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
+            const float w = ex2(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
             const float4 cij = tile[(ty + i) * TW + tx + j];
             ax = __fmaf_rn(w, cij.x, ax);
             ay = __fmaf_rn(w, cij.y, ay);
