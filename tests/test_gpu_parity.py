@@ -80,7 +80,7 @@ def test_query_limits_match_b200(dev):
 
 
 @pytest.mark.parametrize("kernel,threads", [("knn_f4", 128), ("knn_f4", 64), ("knn_f4", 256), ("nlm_f4", 128),
-                                            ("nlm_f4_g3", 128), ("nlm_f4_direct", 128), ("nlm_f4_regheavy", 128),
+                                            ("nlm_f4_g1", 128), ("nlm_f4_direct", 128), ("nlm_f4_regheavy", 128),
                                             ("hotspot_f32", 256),
                                             ("hotspot_f32", 128)])
 def test_every_level_realised_and_verified(dev, kernel, threads):
@@ -136,7 +136,7 @@ def test_knn_ragged_and_degenerate(dev, shape):
     check_vs_oracle(outs[0], out, alt, amb)
 
 
-@pytest.mark.parametrize("kernel", ["nlm_f4", "nlm_f4_g3"])
+@pytest.mark.parametrize("kernel", ["nlm_f4", "nlm_f4_g1"])
 @pytest.mark.parametrize("sigma", [0.05, 0.13, 0.2])
 def test_nlm_box_all_levels(dev, sigma, kernel):
     img = synth.noisy_rgba(250, 131, seed=2, sigma=sigma)
