@@ -214,7 +214,8 @@ def run_ours(args):
 
     # ---- multi-version binary: probe -> levels -> build (offline, untimed) ----------------
     t_build = time.perf_counter()
-    variants, res = O.build_all_levels(local, kernel)
+    realise = O.REALISE_MIN_CARVEOUT if args.realise == "min" else O.REALISE_MAX_SMEM
+    variants, res = O.build_all_levels(local, kernel, mode=realise)
     t_build = time.perf_counter() - t_build
     nlev = len(variants)
     lv = [variants.level(i) for i in range(nlev)]
@@ -255,6 +256,17 @@ def run_ours(args):
         sweep_args = O.hotspot_args(t_a.data_ptr(), t_b.data_ptr(), pw.data_ptr(), W, H)
     ms = variants.sweep(sweep_args, sp, rounds=args.rounds)
     best = min(range(nlev), key=lambda i: ms[i])
+    # the carveout axis (Table 3 analogue): the same levels realised the other way
+    carveout_axis = None
+    if not args.no_carveout_axis:
+        other = O.REALISE_MAX_SMEM if realise == O.REALISE_MIN_CARVEOUT else O.REALISE_MIN_CARVEOUT
+        v2, _ = O.build_all_levels(local, kernel, mode=other)
+        ms2 = v2.sweep(sweep_args, sp, rounds=args.rounds)
+        carveout_axis = {"realise": "min_carveout" if other == O.REALISE_MIN_CARVEOUT else "max_smem",
+                         "levels": [{"k": v2.level(i).ctas_per_sm, "carveout_kb": v2.level(i).carveout_kb,
+                                     "pad": v2.level(i).smem_pad_bytes, "ms": round(ms2[i], 5)} for i in range(len(v2))],
+                         "ms_best": min(ms2)}
+        v2.close()
     worst = max(range(nlev), key=lambda i: ms[i])
 
     # ---- the tuned loop: warmup (includes Fig. 9 exploration) then K timed steps ----------
@@ -381,8 +393,8 @@ def run_ours(args):
         cpu = {"value": u / dt / 1e6, "unit": wl["unit"], "cores": 1, "kind": "oracle", "sample": sample}
 
     lvl_rows = [{"k": lv[i].ctas_per_sm, "occ": lv[i].occupancy_permille / 1000, "reg_cap": lv[i].reg_cap,
-                 "regs": infos[i].regs, "pad": lv[i].smem_pad_bytes, "spill_st": infos[i].spill_store,
-                 "ms": round(ms[i], 5)} for i in range(nlev)]
+                 "regs": infos[i].regs, "pad": lv[i].smem_pad_bytes, "carveout_kb": lv[i].carveout_kb,
+                 "spill_st": infos[i].spill_store, "ms": round(ms[i], 5)} for i in range(nlev)]
     line = {
         "metric": METRIC, "value": value, "unit": wl["unit"], "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
@@ -404,6 +416,8 @@ def run_ours(args):
         "vs_maxocc": ms[kmax] / t_final,
         "vs_nvcc_default": ms[orig] / t_final,
         "build_seconds": round(t_build, 2),
+        "realise": "min_carveout" if realise == O.REALISE_MIN_CARVEOUT else "max_smem",
+        "carveout_axis": carveout_axis,
     }
     print(json.dumps(line), flush=True)
     if world > 1:
@@ -519,6 +533,9 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
     ap.add_argument("--kernel", default="", help="override the workload's kernel id (same family)")
+    ap.add_argument("--realise", choices=["max", "min"], default="max",
+                    help="level realisation: max = pad against 228 KB smem; min = smallest carveout (more L1)")
+    ap.add_argument("--no-carveout-axis", action="store_true", help="skip the sweep of the other realisation")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")

@@ -71,7 +71,16 @@ typedef struct {
     int reg_cap;             /* ptxas --maxrregcount for this level; 0 = uncapped (natural) */
     int smem_pad_bytes;      /* extra dynamic shared memory that caps residency at k */
     int limiter;             /* ORION_LIM_* bits                                            */
+    int carveout_kb;         /* per-SM shared-memory configuration the level is realised with
+                                (8 .. 228 KB; the rest of the 256 KB array is L1); 0 = left to
+                                the driver (no padding needed)                               */
 } orion_level;
+
+/* How a level's CTA count is realised (the paper's small- vs large-cache axis, P:L757-P:L761,
+ * Table 3): MAX_SMEM pins the carveout at 228 KB whenever padding is needed (smallest L1);
+ * MIN_CARVEOUT picks the smallest shared-memory configuration that still holds k CTAs and
+ * pads within it (largest L1 for spills and cached loads). */
+enum { ORION_REALISE_MAX_SMEM = 0, ORION_REALISE_MIN_CARVEOUT = 1 };
 
 /* ---- occupancy levels (question 1; host-only, pure) -------------------------------------- */
 
@@ -96,6 +105,16 @@ orion_status orion_ctas_per_sm(const orion_device_limits *dev, int block_threads
  * -> ORION_E_CAPACITY with *n_out = the number needed.  `out` may be NULL if capacity = 0. */
 orion_status orion_levels(const orion_device_limits *dev, const orion_kernel_resources *res,
                           orion_level *out, int capacity, int *n_out);
+/* orion_levels with an explicit realisation mode (ORION_REALISE_*); orion_levels = MAX_SMEM.
+ * Same k_max and register caps in both modes; padding and carveout differ. */
+orion_status orion_levels_ex(const orion_device_limits *dev, const orion_kernel_resources *res, int mode,
+                             orion_level *out, int capacity, int *n_out);
+/* orion_ctas_per_sm under a carveout preference of `carveout_pct` percent of the maximum
+ * shared memory (< 0: the default, treated as the maximum), rounded up to a configuration
+ * and raised to fit one CTA, as the driver does. */
+orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int block_threads, int regs,
+                                        int smem_static, int smem_dyn, int carveout_pct, int *ctas,
+                                        int *limiter);
 
 /* ---- code generation (question 1; host-only, no GPU needed) ------------------------------ */
 
@@ -203,6 +222,17 @@ typedef struct {
  * decreasing); then the final kernel every iteration.  Exploration iterations record a
  * CUDA event pair and synchronise on it; final iterations only enqueue the launch. */
 orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, orion_step_report *out);
+/* The measured time of an exploring iteration is work-normalised (ns per output element,
+ * P:L975) before Fig. 9 compares it, so iterations of different sizes compare fairly. */
+
+/* Kernel splitting ("we split one kernel invocation into multiple invocations, such
+ * that every invocation of the split kernel launches a subset of the threads", [30]): the
+ * output rows [row_begin, row_end) of ONE frame are processed as `bands` consecutive row
+ * bands, each one orion_tune_step iteration, so a one-shot frame still gets tuned.  The
+ * union of the bands equals one unsplit launch bit for bit.  reports[bands] may be NULL;
+ * a band left empty by the rounding reports iteration = -1. */
+orion_status orion_tune_split(orion_tuner *t, const orion_args *a, int bands, void *stream,
+                              orion_step_report *reports);
 
 /* Same iteration end to end from HOST buffers: copies a->src (host, pinned for async)
  * into dev_src, runs orion_tune_step with device pointers, copies dev_dst back into

@@ -107,27 +107,60 @@ def smem_alloc_per_cta(dev: Device, smem_static: int, smem_dyn: int) -> int:
     return _round_up(smem_static + dev.smem_reserved_per_block + smem_dyn, dev.smem_alloc_unit)
 
 
-def limit_smem(dev: Device, smem_static: int, smem_dyn: int) -> int:
+# Shared-memory / L1 carveout configurations of cc 10.0 in KB (the unified 256 KB array:
+# what is not shared memory is L1).  The paper's small- vs large-cache configurations
+# (P:L757-P:L761, Table 3) are two points of this axis on Fermi/Kepler.
+CARVEOUT_KB = (0, 8, 16, 32, 64, 100, 132, 164, 196, 228)
+
+
+def smem_config(dev: Device, nbytes: int) -> int | None:
+    """Smallest carveout configuration (bytes) holding `nbytes`."""
+    for kb in CARVEOUT_KB:
+        c = min(kb * 1024, dev.smem_per_sm)
+        if nbytes <= c:
+            return c
+    return None
+
+
+def carveout_budget(dev: Device, carveout_pct: int | None) -> int:
+    """Shared memory per SM a carveout preference asks for: pct of the maximum, rounded up
+    to a configuration; None (the default) counts as the maximum."""
+    if carveout_pct is None:
+        return dev.smem_per_sm
+    return smem_config(dev, carveout_pct * dev.smem_per_sm // 100)
+
+
+def carveout_pct_for(dev: Device, kb: int) -> int:
+    """Largest percentage that still rounds up to exactly `kb` KB."""
+    return (kb * 1024 * 100) // dev.smem_per_sm
+
+
+def limit_smem(dev: Device, smem_static: int, smem_dyn: int, carveout_pct: int | None = None) -> int:
     a = smem_alloc_per_cta(dev, smem_static, smem_dyn)
     if a > dev.smem_per_block_optin + dev.smem_reserved_per_block:
         return 0
     if a == 0:
         return 1 << 30
-    return dev.smem_per_sm // a
+    budget = carveout_budget(dev, carveout_pct)
+    if budget < a:                       # the driver raises the configuration to fit one CTA
+        budget = smem_config(dev, a)
+    return budget // a
 
 
-def ctas_per_sm(dev: Device, T: int, regs: int, smem_static: int = 0, smem_dyn: int = 0) -> int:
+def ctas_per_sm(dev: Device, T: int, regs: int, smem_static: int = 0, smem_dyn: int = 0,
+                carveout_pct: int | None = None) -> int:
     """k = min(L_reg, L_warp, L_blk, L_smem) -- the calculator's answer."""
     return min(limit_regs(dev, T, regs), limit_warps(dev, T), limit_blocks(dev),
-               limit_smem(dev, smem_static, smem_dyn))
+               limit_smem(dev, smem_static, smem_dyn, carveout_pct))
 
 
-def limiter_mask(dev: Device, T: int, regs: int, smem_static: int, smem_dyn: int) -> int:
-    k = ctas_per_sm(dev, T, regs, smem_static, smem_dyn)
+def limiter_mask(dev: Device, T: int, regs: int, smem_static: int, smem_dyn: int,
+                 carveout_pct: int | None = None) -> int:
+    k = ctas_per_sm(dev, T, regs, smem_static, smem_dyn, carveout_pct)
     m = 0
     if limit_regs(dev, T, regs) == k:
         m |= LIM_REGS
-    if limit_smem(dev, smem_static, smem_dyn) == k:
+    if limit_smem(dev, smem_static, smem_dyn, carveout_pct) == k:
         m |= LIM_SMEM
     if limit_warps(dev, T) == k:
         m |= LIM_WARPS
@@ -148,6 +181,10 @@ class Level:
     reg_cap: int            # 0 = uncapped (the kernel's natural register count)
     smem_pad_bytes: int
     limiter: int
+    carveout_kb: int = 0    # shared-memory configuration realising the level; 0 = driver's choice
+
+
+REALISE_MAX_SMEM, REALISE_MIN_CARVEOUT = 0, 1
 
 
 def reg_cap_for(dev: Device, T: int, natural: int, k: int, min_reg_cap: int = 16) -> int | None:
@@ -163,23 +200,50 @@ def reg_cap_for(dev: Device, T: int, natural: int, k: int, min_reg_cap: int = 16
     return None
 
 
-def pad_for(dev: Device, T: int, regs: int, smem_static: int, smem_need: int, k: int) -> int | None:
-    """Smallest extra dynamic shared memory making the CTA count exactly k (0 if already k)."""
-    base = min(limit_regs(dev, T, regs), limit_warps(dev, T), limit_blocks(dev),
-               limit_smem(dev, smem_static, smem_need))
+def pad_for(dev: Device, T: int, regs: int, smem_static: int, smem_need: int, k: int,
+            carveout_pct: int | None = None) -> int | None:
+    """Smallest extra dynamic shared memory making the CTA count exactly k (0 if already k)
+    under the given carveout preference."""
+    base = ctas_per_sm(dev, T, regs, smem_static, smem_need, carveout_pct)
     if base == k:
         return 0
     if base < k:
         return None
-    a_k = _round_up(dev.smem_per_sm // (k + 1) + 1, dev.smem_alloc_unit)
+    budget = carveout_budget(dev, carveout_pct)
+    a_k = _round_up(budget // (k + 1) + 1, dev.smem_alloc_unit)
     pad = a_k - dev.smem_reserved_per_block - smem_static - smem_need
-    if pad < 0 or limit_smem(dev, smem_static, smem_need + pad) != k:
+    if pad < 0 or limit_smem(dev, smem_static, smem_need + pad, carveout_pct) != k:
         return None
     return pad
 
 
+def realise(dev: Device, T: int, regs: int, smem_static: int, smem_need: int, k: int, mode: int):
+    """(pad, carveout_kb) realising k CTAs/SM, or None.  MAX_SMEM: pad against the full
+    228 KB (pinned only when a pad is needed).  MIN_CARVEOUT: the smallest configuration
+    that still admits k CTAs, padded inside it -- the rest of the array stays L1."""
+    if mode == REALISE_MAX_SMEM:
+        pad = pad_for(dev, T, regs, smem_static, smem_need, k)
+        if pad is None:
+            return None
+        return pad, (dev.smem_per_sm // 1024 if pad > 0 else 0)
+    for kb in CARVEOUT_KB:
+        if kb == 0 or kb * 1024 > dev.smem_per_sm:
+            continue
+        pct = carveout_pct_for(dev, kb)
+        if carveout_budget(dev, pct) != kb * 1024:
+            continue
+        pad = pad_for(dev, T, regs, smem_static, smem_need, k, pct)
+        if pad is not None:
+            return pad, kb
+    return None
+
+
+def level_carveout_pct(dev: Device, lv: Level) -> int | None:
+    return carveout_pct_for(dev, lv.carveout_kb) if lv.carveout_kb > 0 else None
+
+
 def levels(dev: Device, T: int, natural_regs: int, smem_static: int = 0, smem_need: int = 0,
-           min_reg_cap: int = 16) -> list[Level]:
+           min_reg_cap: int = 16, mode: int = REALISE_MAX_SMEM) -> list[Level]:
     """All feasible levels k = 1..k_max, ascending k."""
     out = []
     kmax_bound = min(limit_warps(dev, T), limit_blocks(dev), limit_smem(dev, smem_static, smem_need))
@@ -188,15 +252,18 @@ def levels(dev: Device, T: int, natural_regs: int, smem_static: int = 0, smem_ne
         if cap is None:
             continue
         regs = natural_regs if cap == 0 else cap
-        pad = pad_for(dev, T, regs, smem_static, smem_need, k)
-        if pad is None:
+        r = realise(dev, T, regs, smem_static, smem_need, k, mode)
+        if r is None:
             continue
+        pad, kb = r
         w = warps_per_cta(dev, T)
         maxw = dev.max_threads_per_sm // dev.warp_size
+        pct = carveout_pct_for(dev, kb) if kb > 0 else None
         out.append(Level(ctas_per_sm=k, warps_per_sm=k * w,
                          occupancy_permille=(k * w * 1000) // maxw,
                          reg_cap=cap, smem_pad_bytes=pad,
-                         limiter=limiter_mask(dev, T, regs, smem_static, smem_need + pad)))
+                         limiter=limiter_mask(dev, T, regs, smem_static, smem_need + pad, pct),
+                         carveout_kb=kb))
     return out
 
 

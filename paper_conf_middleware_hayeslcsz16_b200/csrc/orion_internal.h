@@ -33,10 +33,15 @@ orion_status ensure_context(int device);
 // ---- occupancy arithmetic (levels.cpp) ----------------------------------------------------
 int limit_regs(const orion_device_limits &d, int T, int regs);
 int limit_warps(const orion_device_limits &d, int T);
-int limit_smem(const orion_device_limits &d, int smem_static, int smem_dyn);
-int ctas_per_sm(const orion_device_limits &d, int T, int regs, int smem_static, int smem_dyn, int *limiter);
+// carveout_pct < 0: the driver default (the calculator treats it as the maximum).
+int limit_smem(const orion_device_limits &d, int smem_static, int smem_dyn, int carveout_pct);
+int ctas_per_sm(const orion_device_limits &d, int T, int regs, int smem_static, int smem_dyn, int carveout_pct,
+                int *limiter);
 // Smallest padding realising exactly k CTAs/SM at `regs` registers (0 if already k); -1 if impossible.
-int pad_for_level(const orion_device_limits &d, int T, int regs, int smem_static, int smem_need, int k);
+int pad_for_level(const orion_device_limits &d, int T, int regs, int smem_static, int smem_need, int k,
+                  int carveout_pct);
+int carveout_pct_for_kb(const orion_device_limits &d, int kb);
+int level_carveout_pct(const orion_device_limits &d, const orion_level &L);
 
 // ---- kernel registry + code generation (registry.cpp) -------------------------------------
 enum KernelKind { K_KNN = 0, K_NLM = 1, K_STENCIL = 2 };
@@ -88,7 +93,7 @@ struct orion_variants {
         std::shared_ptr<const orion::CompiledVariant> cv;
         CUmodule mod = nullptr;
         CUfunction fn = nullptr;
-        int regs = 0, local_bytes = 0, verified = 0, dyn_bytes = 0;
+        int regs = 0, local_bytes = 0, verified = 0, dyn_bytes = 0, carveout_pct = -1;
         bool warmed = false;
     };
     std::vector<Var> vars;

@@ -249,7 +249,11 @@ orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, 
         ORION_CU(D.cuEventRecord(t->e1, s));
         ORION_CU(D.cuEventSynchronize(t->e1));
         ORION_CU(D.cuEventElapsedTime(&ms, t->e0, t->e1));
-        const float m = (t->samples == 0) ? ms : std::min(t->sample_best, ms);
+        // work-normalised runtime: ns per output element, so iterations of
+        // different sizes -- the bands of a split frame -- compare fairly
+        const double work = (double)(a->row_end - a->row_begin) * (double)a->width;
+        const float per = work > 0 ? (float)(ms * 1e6 / work) : ms;
+        const float m = (t->samples == 0) ? per : std::min(t->sample_best, per);
         t->samples += 1;
         t->sample_best = m;
         if (t->samples >= f.cfg.samples_per_level) {
@@ -270,6 +274,31 @@ orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, 
         out->ms = ms;
     }
     f.iter += 1;
+    return ORION_OK;
+}
+
+orion_status orion_tune_split(orion_tuner *t, const orion_args *a, int bands, void *stream, orion_step_report *reports)
+{
+    if (!t || !a || bands < 1) return fail(ORION_E_INVALID, "orion_tune_split: bad argument");
+    const int rows = a->row_end - a->row_begin;
+    if (rows < 0) return fail(ORION_E_INVALID, "orion_tune_split: row_end < row_begin");
+    const int per = rows > 0 ? (rows + bands - 1) / bands : 0;
+    for (int b = 0; b < bands; ++b) {
+        orion_args ba = *a;
+        ba.row_begin = std::min(a->row_end, a->row_begin + b * per);
+        ba.row_end = std::min(a->row_end, ba.row_begin + per);
+        orion_step_report r{};
+        if (ba.row_begin < ba.row_end) {
+            ORION_TRY(orion_tune_step(t, &ba, stream, &r));
+        } else {
+            r.iteration = -1;
+            r.level_idx = -1;
+            r.phase = -1;
+            r.final_level_idx = t->f.final_idx;
+            r.ms = -1.0f;
+        }
+        if (reports) reports[b] = r;
+    }
     return ORION_OK;
 }
 

@@ -112,16 +112,22 @@ orion_status orion_build_variants(int device, const char *kernel_id, int block_t
         ORION_CU(D.cuFuncGetAttribute(&w.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, w.fn));
         ORION_CU(D.cuFuncGetAttribute(&w.local_bytes, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, w.fn));
         ORION_CU(D.cuFuncGetAttribute(&static_smem, CU_FUNC_ATTRIBUTE_SHARED_SIZE_BYTES, w.fn));
-        const int pad = pad_for_level(v->dev, T, w.regs, static_smem, need, L.ctas_per_sm);
+        // the level's carveout: its configuration when it names one, else the maximum
+        // whenever padding turns out to be needed at the actual register count
+        int pct = level_carveout_pct(v->dev, L);
+        int pad = pad_for_level(v->dev, T, w.regs, static_smem, need, L.ctas_per_sm, pct);
+        if (pad > 0 && pct < 0) pct = 100;
         if (pad < 0)
             return fail(ORION_E_INFEASIBLE, "level " + std::to_string(L.ctas_per_sm) + " CTAs/SM not realisable at " +
                                                 std::to_string(w.regs) + " registers");
         w.dyn_bytes = need + pad;
+        w.carveout_pct = pct;
         ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, w.dyn_bytes));
-        if (pad > 0) ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100));
+        if (pct >= 0) ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, pct));
         ORION_CU(D.cuOccupancyMaxActiveBlocksPerMultiprocessor(&w.verified, w.fn, T, (size_t)w.dyn_bytes));
-        if (w.verified != L.ctas_per_sm && pad == 0) {
+        if (w.verified != L.ctas_per_sm && pct < 0) {
             // the driver picked a smaller carveout than the calculator assumes: pin it
+            w.carveout_pct = pct = 100;
             ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100));
             ORION_CU(D.cuOccupancyMaxActiveBlocksPerMultiprocessor(&w.verified, w.fn, T, (size_t)w.dyn_bytes));
         }
@@ -132,8 +138,9 @@ orion_status orion_build_variants(int device, const char *kernel_id, int block_t
         w.realised = L;
         w.realised.smem_pad_bytes = pad;
         int limiter = 0;
-        ctas_per_sm(v->dev, T, w.regs, static_smem, w.dyn_bytes, &limiter);
+        ctas_per_sm(v->dev, T, w.regs, static_smem, w.dyn_bytes, pct, &limiter);
         w.realised.limiter = limiter;
+        w.realised.carveout_kb = pct < 0 ? 0 : (pct >= 100 ? v->dev.smem_per_sm / 1024 : L.carveout_kb);
         w.realised.warps_per_sm = L.ctas_per_sm * warps_of(v->dev, T);
         w.realised.occupancy_permille = w.realised.warps_per_sm * 1000 / (v->dev.max_threads_per_sm / v->dev.warp_size);
     }

@@ -56,15 +56,19 @@ class KernelResources(ctypes.Structure):
 
 class Level(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int) for n in (
-        "ctas_per_sm", "warps_per_sm", "occupancy_permille", "reg_cap", "smem_pad_bytes", "limiter")]
+        "ctas_per_sm", "warps_per_sm", "occupancy_permille", "reg_cap", "smem_pad_bytes", "limiter",
+        "carveout_kb")]
 
     def as_tuple(self):
         return tuple(getattr(self, n) for n, _ in self._fields_)
 
     def __repr__(self):
-        return ("Level(k=%d, warps=%d, occ=%.3f, cap=%d, pad=%d, lim=%d)"
+        return ("Level(k=%d, warps=%d, occ=%.3f, cap=%d, pad=%d, lim=%d, carveout=%dKB)"
                 % (self.ctas_per_sm, self.warps_per_sm, self.occupancy_permille / 1000.0,
-                   self.reg_cap, self.smem_pad_bytes, self.limiter))
+                   self.reg_cap, self.smem_pad_bytes, self.limiter, self.carveout_kb))
+
+
+REALISE_MAX_SMEM, REALISE_MIN_CARVEOUT = 0, 1
 
 
 class Args(ctypes.Structure):
@@ -106,6 +110,8 @@ def lib() -> ctypes.CDLL:
                 "orion_query_limits": [I, P(DeviceLimits)],
                 "orion_ctas_per_sm": [P(DeviceLimits), I, I, I, I, P(I), P(I)],
                 "orion_levels": [P(DeviceLimits), P(KernelResources), P(Level), I, P(I)],
+                "orion_levels_ex": [P(DeviceLimits), P(KernelResources), I, P(Level), I, P(I)],
+                "orion_ctas_per_sm_carveout": [P(DeviceLimits), I, I, I, I, I, P(I), P(I)],
                 "orion_kernel_probe": [ctypes.c_char_p, I, P(KernelResources)],
                 "orion_compile_info": [ctypes.c_char_p, I, I, P(I), P(I), P(I), P(I)],
                 "orion_build_variants": [I, ctypes.c_char_p, I, P(Level), I, P(V)],
@@ -120,6 +126,7 @@ def lib() -> ctypes.CDLL:
                 "orion_tune_step": [V, P(Args), V, P(StepReport)],
                 "orion_tune_step_host": [V, P(Args), V, V, V, V, P(StepReport), P(ctypes.c_longlong),
                                          P(ctypes.c_longlong)],
+                "orion_tune_split": [V, P(Args), I, V, P(StepReport)],
                 "orion_host_pipe_create": [V, I, I, I, P(V)],
                 "orion_host_pipe_submit": [V, P(Args), P(StepReport), P(ctypes.c_longlong), P(ctypes.c_longlong)],
                 "orion_host_pipe_drain": [V],
@@ -169,10 +176,11 @@ def query_limits(device: int = 0) -> DeviceLimits:
     return d
 
 
-def ctas_per_sm(dev: DeviceLimits, T: int, regs: int, smem_static: int = 0, smem_dyn: int = 0):
+def ctas_per_sm(dev: DeviceLimits, T: int, regs: int, smem_static: int = 0, smem_dyn: int = 0,
+                carveout_pct: int = -1):
     c, lim = ctypes.c_int(), ctypes.c_int()
-    _check(lib().orion_ctas_per_sm(ctypes.byref(dev), T, regs, smem_static, smem_dyn, ctypes.byref(c),
-                                   ctypes.byref(lim)), "orion_ctas_per_sm")
+    _check(lib().orion_ctas_per_sm_carveout(ctypes.byref(dev), T, regs, smem_static, smem_dyn, carveout_pct,
+                                            ctypes.byref(c), ctypes.byref(lim)), "orion_ctas_per_sm_carveout")
     return c.value, lim.value
 
 
@@ -181,13 +189,14 @@ def resources(block_threads: int, regs: int, static_smem: int = 0, dyn_smem: int
     return KernelResources(block_threads, regs, static_smem, dyn_smem, min_reg_cap)
 
 
-def levels(dev: DeviceLimits, res: KernelResources) -> list[Level]:
+def levels(dev: DeviceLimits, res: KernelResources, mode: int = REALISE_MAX_SMEM) -> list[Level]:
     n = ctypes.c_int()
-    st = lib().orion_levels(ctypes.byref(dev), ctypes.byref(res), None, 0, ctypes.byref(n))
+    st = lib().orion_levels_ex(ctypes.byref(dev), ctypes.byref(res), mode, None, 0, ctypes.byref(n))
     if st not in (ORION_OK, -2):
-        _check(st, "orion_levels")
+        _check(st, "orion_levels_ex")
     arr = (Level * max(1, n.value))()
-    _check(lib().orion_levels(ctypes.byref(dev), ctypes.byref(res), arr, n.value, ctypes.byref(n)), "orion_levels")
+    _check(lib().orion_levels_ex(ctypes.byref(dev), ctypes.byref(res), mode, arr, n.value, ctypes.byref(n)),
+           "orion_levels_ex")
     return [arr[i] for i in range(n.value)]
 
 
@@ -303,11 +312,12 @@ class Variants:
             pass
 
 
-def build_all_levels(device: int, kernel_id: str, block_threads: int = 0, dev: DeviceLimits | None = None):
-    """Convenience: probe -> orion_levels -> orion_build_variants (every feasible level)."""
+def build_all_levels(device: int, kernel_id: str, block_threads: int = 0, dev: DeviceLimits | None = None,
+                     mode: int = REALISE_MAX_SMEM):
+    """Convenience: probe -> orion_levels_ex -> orion_build_variants (every feasible level)."""
     res = kernel_probe(kernel_id, block_threads)
     dev = dev or query_limits(device)
-    lv = levels(dev, res)
+    lv = levels(dev, res, mode)
     return Variants(device, kernel_id, lv, block_threads), res
 
 
@@ -333,6 +343,11 @@ class Tuner:
         r = StepReport()
         _check(lib().orion_tune_step(self.h, ctypes.byref(args), _s(stream), ctypes.byref(r)), "orion_tune_step")
         return r
+
+    def split(self, args: Args, bands: int, stream=None) -> list[StepReport]:
+        reps = (StepReport * bands)()
+        _check(lib().orion_tune_split(self.h, ctypes.byref(args), bands, _s(stream), reps), "orion_tune_split")
+        return [reps[i] for i in range(bands)]
 
     def step_host(self, args: Args, dev_src: int, dev_dst: int, dev_aux: int | None = None, stream=None):
         r = StepReport()

@@ -22,7 +22,7 @@ def occ_ref(tmp_path_factory):
                            os.path.join(ROOT, "tests", "helpers", "occ_ref.cpp"), "-o", exe])
 
     def run(cases):
-        inp = "".join(f"{T} {r} {s} {d}\n" for (T, r, s, d) in cases)
+        inp = "".join(" ".join(str(x) for x in (tuple(c) + (100,))[:5]) + "\n" for c in cases)
         out = subprocess.run([exe], input=inp, capture_output=True, text=True, check=True).stdout
         return [int(x) for x in out.split()]
     return run

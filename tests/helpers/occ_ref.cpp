@@ -2,7 +2,8 @@
 // (/usr/local/cuda/include/cuda_occupancy.h), used as an independent pin for the
 // oracle's O1 calculator.  Reads lines "T regs smem_static smem_dyn" on stdin and
 // prints the CTAs/SM that cudaOccMaxActiveBlocksPerMultiprocessor reports for a
-// B200 (cc 10.0) with the MAX_SHARED carveout and the dynamic-smem opt-in set.
+// B200 (cc 10.0) with the given carveout preference (percent; -1 = default) and the
+// dynamic-smem opt-in set.  Input lines: "T regs smem_static smem_dyn carveout_pct".
 #include <cuda_occupancy.h>
 #include <cstdio>
 
@@ -20,8 +21,8 @@ int main() {
     prop.numSms = 148;
     prop.sharedMemPerBlockOptin = 232448;
     prop.reservedSharedMemPerBlock = 1024;
-    int T, regs, sst, sdyn;
-    while (std::scanf("%d %d %d %d", &T, &regs, &sst, &sdyn) == 4) {
+    int T, regs, sst, sdyn, pct;
+    while (std::scanf("%d %d %d %d %d", &T, &regs, &sst, &sdyn, &pct) == 5) {
         cudaOccFuncAttributes attr;
         attr.maxThreadsPerBlock = 1024;
         attr.numRegs = regs;
@@ -30,7 +31,8 @@ int main() {
         attr.shmemLimitConfig = FUNC_SHMEM_LIMIT_OPTIN;
         attr.maxDynamicSharedSizeBytes = 232448 - sst;
         cudaOccDeviceState state;
-        state.carveoutConfig = SHAREDMEM_CARVEOUT_MAX_SHARED;
+        state.carveoutConfig = pct;
+        state.cacheConfig = CACHE_PREFER_NONE;
         cudaOccResult res;
         cudaOccError e = cudaOccMaxActiveBlocksPerMultiprocessor(&res, &prop, &attr, &state, T, (size_t)sdyn);
         std::printf("%d\n", e == CUDA_OCC_SUCCESS ? res.activeBlocksPerMultiprocessor : -1);

@@ -54,15 +54,26 @@ def test_ctas_per_sm_matches_oracle_grid():
         assert lim == OC.limiter_mask(OC.B200, T, r, s, dyn), (T, r, s, dyn)
 
 
+@pytest.mark.parametrize("mode", [0, 1])
 @pytest.mark.parametrize("T", [64, 128, 256, 512])
 @pytest.mark.parametrize("natural", [16, 24, 32, 37, 39, 46, 56, 63, 64, 72, 96, 128, 168, 200, 241, 255])
 @pytest.mark.parametrize("smem", [(0, 0), (0, 13376), (1024, 8192), (0, 52544), (0, 100000)])
-def test_levels_bit_exact_vs_oracle(T, natural, smem):
+def test_levels_bit_exact_vs_oracle(T, natural, smem, mode):
     d = O.b200_limits()
-    got = [l.as_tuple() for l in O.levels(d, O.resources(T, natural, smem[0], smem[1]))]
-    want = [(l.ctas_per_sm, l.warps_per_sm, l.occupancy_permille, l.reg_cap, l.smem_pad_bytes, l.limiter)
-            for l in OC.levels(OC.B200, T, natural, smem[0], smem[1])]
+    got = [l.as_tuple() for l in O.levels(d, O.resources(T, natural, smem[0], smem[1]), mode)]
+    want = [(l.ctas_per_sm, l.warps_per_sm, l.occupancy_permille, l.reg_cap, l.smem_pad_bytes, l.limiter,
+             l.carveout_kb) for l in OC.levels(OC.B200, T, natural, smem[0], smem[1], mode=mode)]
     assert got == want
+
+
+def test_ctas_per_sm_carveout_matches_oracle():
+    d = O.b200_limits()
+    for T, r, dyn, pct in itertools.product((64, 128, 256), (24, 64, 128), (0, 3000, 30000, 120000),
+                                            (-1, 0, 3, 14, 28, 43, 71, 100)):
+        k, lim = O.ctas_per_sm(d, T, r, 0, dyn, pct)
+        p = None if pct < 0 else pct
+        assert k == OC.ctas_per_sm(OC.B200, T, r, 0, dyn, p), (T, r, dyn, pct)
+        assert lim == OC.limiter_mask(OC.B200, T, r, 0, dyn, p)
 
 
 def test_levels_capacity_protocol():
@@ -81,6 +92,7 @@ def test_levels_capacity_protocol():
 def _o_levels(T, natural, need=0):
     ol = OC.levels(OC.B200, T, natural, 0, need)
     return ol, [O.Level(*[getattr(l, f) for f, _ in O.Level._fields_]) for l in ol]
+
 
 
 def _replay_both(T, natural, need, ms, iters, **cfgkw):

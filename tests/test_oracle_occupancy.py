@@ -93,3 +93,45 @@ def test_limiter_mask_and_eq1_upper_bound():
         assert k * T <= eq1_threads + 1e-9
         m = O.limiter_mask(O.B200, T, regs, 0, smem)
         assert m != 0
+
+
+CARVEOUT_PCTS = (-1, 0, 3, 7, 14, 28, 43, 50, 57, 71, 85, 99, 100)
+
+
+def test_carveout_preferences_against_nvidia_header(occ_ref):
+    # the unified L1 / shared-memory carveout (small vs large cache, Table 3)
+    cases = []
+    for T in (64, 128, 256):
+        for regs in (24, 40, 64, 128):
+            for sdyn in (0, 3000, 9000, 30000, 60000, 120000):
+                for pct in CARVEOUT_PCTS:
+                    cases.append((T, regs, 0, sdyn, pct))
+    want = occ_ref(cases)
+    got = [O.ctas_per_sm(O.B200, T, r, s, d, None if p < 0 else p) for (T, r, s, d, p) in cases]
+    bad = [(c, g, w) for c, g, w in zip(cases, got, want) if g != w]
+    assert not bad, bad[:10]
+
+
+def test_carveout_percent_maps_to_each_configuration():
+    for kb in O.CARVEOUT_KB[1:]:
+        pct = O.carveout_pct_for(O.B200, kb)
+        assert O.carveout_budget(O.B200, pct) == kb * 1024
+        if pct < 100:
+            assert O.carveout_budget(O.B200, pct + 1) > kb * 1024
+
+
+@pytest.mark.parametrize("T,natural,need", [(256, 46, 0), (128, 255, 11264), (128, 56, 13376), (128, 255, 108756)])
+def test_min_carveout_levels_realise_k_per_nvidia_header(occ_ref, T, natural, need):
+    lmax = O.levels(O.B200, T, natural, 0, need)
+    lmin = O.levels(O.B200, T, natural, 0, need, mode=O.REALISE_MIN_CARVEOUT)
+    assert [l.ctas_per_sm for l in lmin] == [l.ctas_per_sm for l in lmax]
+    assert [l.reg_cap for l in lmin] == [l.reg_cap for l in lmax]
+    cases = [(T, natural if l.reg_cap == 0 else l.reg_cap, 0, need + l.smem_pad_bytes,
+              O.carveout_pct_for(O.B200, l.carveout_kb)) for l in lmin]
+    assert occ_ref(cases) == [l.ctas_per_sm for l in lmin]
+    for a, b in zip(lmin, lmax):        # never a larger shared-memory carve-out than MAX_SMEM
+        assert 0 < a.carveout_kb <= 228
+        assert a.carveout_kb * 1024 <= max(b.carveout_kb * 1024, O.B200.smem_per_sm)
+    # a kernel without shared memory keeps almost all of the array as L1 at every level
+    if need == 0:
+        assert max(l.carveout_kb for l in lmin) <= 100

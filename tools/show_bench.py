@@ -18,7 +18,11 @@ for fn in sys.argv[1:]:
         if "tuner" in d:
             print("  tuner", d["tuner"], "regret=%.4f vs_maxocc=%.4f vs_nvcc=%.4f" % (
                 d["regret"], d["vs_maxocc"], d["vs_nvcc_default"]))
-            print("  sweep", [(l["k"], l["reg_cap"], l["regs"], l["pad"], l["spill_st"], l["ms"]) for l in sw["levels"]])
+            print("  sweep", [(l["k"], l["reg_cap"], l["regs"], l["pad"], l.get("carveout_kb"), l["spill_st"], l["ms"])
+                              for l in sw["levels"]])
+        if d.get("carveout_axis"):
+            ca = d["carveout_axis"]
+            print("  carveout axis", ca["realise"], [(l["k"], l["carveout_kb"], l["pad"], l["ms"]) for l in ca["levels"]])
         for k in ("cpu_baseline", "e2e", "clocks", "gpu_launches"):
             if k in d:
                 print("  ", k, d[k])
