@@ -96,8 +96,15 @@ class ClockSampler:
                 pass
             time.sleep(self.period)
 
+    def _energy_mj(self):
+        try:
+            return self.nv.nvmlDeviceGetTotalEnergyConsumption(self.h)
+        except Exception:
+            return None
+
     def __enter__(self):
         if self.ok:
+            self.e0, self.t0 = self._energy_mj(), time.perf_counter()
             self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
         return self
@@ -106,6 +113,14 @@ class ClockSampler:
         if self.ok:
             self.stop.set()
             self.t.join()
+            self.e1, self.t1 = self._energy_mj(), time.perf_counter()
+
+    def energy(self, steps: int):
+        """Board energy over the timed region (NVML counter, mJ): J per step and mean W."""
+        if not self.ok or self.e0 is None or self.e1 is None:
+            return None
+        j = (self.e1 - self.e0) / 1e3
+        return {"joules_per_step": j / steps, "mean_watts": j / (self.t1 - self.t0), "source": "nvml total energy"}
 
     def summary(self):
         if not self.ok:
@@ -270,7 +285,7 @@ def run_ours(args):
     worst = max(range(nlev), key=lambda i: ms[i])
 
     # ---- the tuned loop: warmup (includes Fig. 9 exploration) then K timed steps ----------
-    cfg = O.default_cfg()
+    cfg = O.default_cfg(select_mode=O.SELECT_LOWEST_WITHIN_TOL if args.select == "lowest" else O.SELECT_FASTEST)
     tuner = O.Tuner(variants, cfg)
     direction, ladder = tuner.ladder()
     if is_stencil:
@@ -405,6 +420,14 @@ def run_ours(args):
                          "grid 768 MiB > L2 (126 MB)",
                    "parallelism": f"dp{world} (independent frames per GPU)"},
         "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
+        "energy": clk.energy(args.steps),
+        "select_mode": args.select,
+        "resources": {"final_regs": infos[final].regs if final >= 0 else None,
+                      "natural_regs": res.regs_per_thread,
+                      "final_warps_per_sm": lv[final].warps_per_sm if final >= 0 else None,
+                      "best_warps_per_sm": lv[best].warps_per_sm,
+                      "register_file_used_frac": (infos[final].regs * lv[final].warps_per_sm * 32 / 65536)
+                      if final >= 0 else None},
         "tuner": {"direction": "increasing" if direction == 1 else "decreasing", "ladder_k": [lv[i].ctas_per_sm
                   for i in ladder], "final_k": lv[final].ctas_per_sm if final >= 0 else None,
                   "final_occupancy": lv[final].occupancy_permille / 1000 if final >= 0 else None,
@@ -507,7 +530,7 @@ def run_c5(args):
             "per_rank": [{"rank": r, "final_k": c[0], "iterations_to_final": c[1], "sweep_best_k": c[2]}
                          for r, c in enumerate(allc)],
             "sweep_rank0": [{"k": variants.level(i).ctas_per_sm, "ms": round(ms[i], 4)} for i in range(nlev)],
-            "gpu_launches": launches, "clocks": clk.summary(),
+            "gpu_launches": launches, "clocks": clk.summary(), "energy": clk.energy(args.steps),
             "e2e": {"value": None, "unit": "Mpix/s", "note": "C5 inputs are generated in place per rank"},
             "cpu_baseline": None,
         }
@@ -533,7 +556,9 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
     ap.add_argument("--kernel", default="", help="override the workload's kernel id (same family)")
-    ap.add_argument("--realise", choices=["max", "min"], default="max",
+    ap.add_argument("--select", choices=["fastest", "lowest"], default="fastest",
+                    help="final-kernel rule: fastest measured, or lowest occupancy within 2%% (resource saving)")
+    ap.add_argument("--realise", choices=["max", "min"], default="min",
                     help="level realisation: max = pad against 228 KB smem; min = smallest carveout (more L1)")
     ap.add_argument("--no-carveout-axis", action="store_true", help="skip the sweep of the other realisation")
     args = ap.parse_args()

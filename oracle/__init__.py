@@ -29,7 +29,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "liboracle.so")
-_SOURCES = [os.path.join(_HERE, "denoise.c"), os.path.join(_HERE, "stencil.c")]
+_SOURCES = [os.path.join(_HERE, "denoise.c"), os.path.join(_HERE, "stencil.c"), os.path.join(_HERE, "srad.c")]
 _lock = threading.Lock()
 _lib = None
 
@@ -77,6 +77,9 @@ def _load():
         lib.oracle_denoise_points.argtypes = [P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                               P, P, ctypes.c_int, ctypes.POINTER(_DnParams),
                                               ctypes.c_int, P, P, P]
+        lib.oracle_srad_f64.restype = ctypes.c_int
+        lib.oracle_srad_f64.argtypes = [P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_double, ctypes.c_int,
+                                        ctypes.c_int, ctypes.c_int, ctypes.c_int, P, P]
         for name in ("oracle_hotspot_f64", "oracle_hotspot_f32"):
             f = getattr(lib, name)
             f.restype = ctypes.c_int
@@ -171,3 +174,16 @@ def hotspot(t0: np.ndarray, power: np.ndarray, steps: int, consts: dict | None =
     if rc != 0:
         raise MemoryError("oracle hotspot allocation failed")
     return out
+
+
+def srad(j0: np.ndarray, iters: int, lam: float = 0.5, roi=(0, 127, 0, 127)):
+    """`iters` SRAD iterations (O5, reading R-SRAD) in double.  roi = (r1, r2, c1, c2)
+    inclusive.  Returns (J float64 (H, W), q0sqr per iteration)."""
+    j0 = np.ascontiguousarray(j0, dtype=np.float64)
+    H, W = j0.shape
+    r1, r2, c1, c2 = roi
+    out = np.zeros((H, W), np.float64)
+    q0 = np.zeros(max(1, iters), np.float64)
+    if _load().oracle_srad_f64(_ptr(j0), W, H, iters, lam, r1, r2, c1, c2, _ptr(out), _ptr(q0)) != 0:
+        raise MemoryError("oracle srad allocation failed")
+    return out, q0[:iters]
