@@ -47,6 +47,9 @@ WORKLOADS = {
                name="register-heavy NLM 4096x4096 RGBA, maxrregcount caps", insts=2401 * 6 + 49 * 6 + 10, bytes=32),
     "c3": dict(kernel="hotspot_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
                insts=12, bytes=12),
+    # NEXT-4: a second Rodinia stencil (srad), 8 B/cell-iteration (read J, write J')
+    "srad": dict(kernel="srad_f32", W=8192, H=8192, unit="Mcell-steps/s", name="SRAD 8192x8192 fp32 (NEXT-4)",
+                 insts=60, bytes=8),
     "c5": dict(kernel="nlm_f4", W=16384, H=16384, sigma=0.13, unit="Mpix/s",
                name="imageDenoising NLM 16384x16384 RGBA row-sharded with halos + NCCL all-gather",
                insts=24 * 30 + 10, bytes=32),
@@ -164,6 +167,22 @@ def cpu_baseline_nlm(kind: str, W: int, H: int, sigma: float, budget_s: float):
     return n * W, dt, f"{n} rows x {W} px of the C2 frame (rows {y0}..{y0 + n}), oracle/denoise.c, double"
 
 
+def cpu_baseline_srad(W: int, steps: int, budget_s: float):
+    import oracle
+    import synth
+    rows = 128
+    t0a, _ = synth.thermal_inputs(W, rows, seed=1)
+    t0 = time.perf_counter()
+    n = 0
+    while True:
+        oracle.srad(t0a.astype("float64"), steps, 0.5, (0, 127, 0, 127))
+        n += 1
+        dt = time.perf_counter() - t0
+        if dt >= budget_s:
+            break
+    return n * rows * W * steps, dt, f"{n} x ({rows} x {W} cells x {steps} iterations), oracle/srad.c f64"
+
+
 def cpu_baseline_hotspot(W: int, steps: int, budget_s: float):
     import oracle
     import synth
@@ -225,7 +244,8 @@ def run_ours(args):
     sp = stream.cuda_stream
     wl = WORKLOADS[args.workload]
     kernel, W, H = args.kernel or wl["kernel"], wl["W"], wl["H"]
-    is_stencil = kernel == "hotspot_f32"
+    is_srad = kernel == "srad_f32"
+    is_stencil = kernel == "hotspot_f32" or is_srad
 
     # ---- multi-version binary: probe -> levels -> build (offline, untimed) ----------------
     t_build = time.perf_counter()
@@ -248,9 +268,17 @@ def run_ours(args):
         pw = torch.empty((H, W), device=dev)
         O.generate_thermal(local, t_a.data_ptr(), pw.data_ptr(), W, H, seed=1 + rank, stream=sp)
         state = {"a": t_a, "b": t_b}
+        q0 = torch.empty(1, device=dev)   # srad: the ROI statistic of the current iteration
+
+        def grid_args(src, dst):
+            if is_srad:
+                return O.srad_args(src.data_ptr(), dst.data_ptr(), q0.data_ptr(), W, H)
+            return O.hotspot_args(src.data_ptr(), dst.data_ptr(), pw.data_ptr(), W, H)
 
         def step_args(s):
-            a = O.hotspot_args(state["a"].data_ptr(), state["b"].data_ptr(), pw.data_ptr(), W, H)
+            if is_srad:   # the iteration's ROI statistics precede the tuned update kernel
+                O.srad_roi_stats(local, state["a"].data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
+            a = grid_args(state["a"], state["b"])
             state["a"], state["b"] = state["b"], state["a"]
             return a
     else:
@@ -268,7 +296,9 @@ def run_ours(args):
     sweep_args = step_args(0)
     if is_stencil:
         state["a"], state["b"] = t_a, t_b
-        sweep_args = O.hotspot_args(t_a.data_ptr(), t_b.data_ptr(), pw.data_ptr(), W, H)
+        if is_srad:
+            O.srad_roi_stats(local, t_a.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
+        sweep_args = grid_args(t_a, t_b)
     ms = variants.sweep(sweep_args, sp, rounds=args.rounds)
     best = min(range(nlev), key=lambda i: ms[i])
     # the carveout axis (Table 3 analogue): the same levels realised the other way
@@ -401,7 +431,7 @@ def run_ours(args):
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         if is_stencil:
-            u, dt, sample = cpu_baseline_hotspot(W, 1, args.cpu_seconds)
+            u, dt, sample = (cpu_baseline_srad if is_srad else cpu_baseline_hotspot)(W, 1, args.cpu_seconds)
         else:
             u, dt, sample = cpu_baseline_nlm("knn" if kernel.startswith("knn") else "nlm", W, H, wl["sigma"],
                                              args.cpu_seconds)

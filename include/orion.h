@@ -118,7 +118,8 @@ orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int bloc
 
 /* ---- code generation (question 1; host-only, no GPU needed) ------------------------------ */
 
-/* Kernel ids: "knn_f4", "nlm_f4", "nlm_f4_g1", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32".
+/* Kernel ids: "knn_f4", "nlm_f4", "nlm_f4_g1", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32",
+ * "srad_f32".
  * block_threads = 0 selects the kernel's default CTA size.  Fills the natural resources
  * (compiles the kernel's PTX once, uncapped, with the embedded ptxas). */
 orion_status orion_kernel_probe(const char *kernel_id, int block_threads, orion_kernel_resources *out);
@@ -282,6 +283,13 @@ orion_status orion_generate_rgba(int device, void *dst, int width, int height, i
 /* Thermal T0 and power map (W x H) into t0 / power. */
 orion_status orion_generate_thermal(int device, void *t0, void *power, int width, int height, unsigned seed,
                                     void *stream);
+/* SRAD's per-iteration ROI statistics (Rodinia srad_v2, reading R-SRAD; Table 2
+ * P:L739): q0sqr = var / mean^2 of J over rows [r1, r2] x cols [c1, c2] (inclusive) of the
+ * width-pitched device image J, reduced in double in a fixed order by one CTA and stored as
+ * one float at device address q0 -- the `aux` of the "srad_f32" kernel's orion_args
+ * (whose fparam[0] = lambda).  Asynchronous on `stream`. */
+orion_status orion_srad_roi_stats(int device, const void *J, int width, int height, int r1, int r2, int c1, int c2,
+                                  void *q0, void *stream);
 /* Write `bytes` of `buf` (a device scratch buffer larger than L2) to evict the L2. */
 orion_status orion_flush_l2(int device, void *buf, long long bytes, void *stream);
 

@@ -44,7 +44,7 @@ int carveout_pct_for_kb(const orion_device_limits &d, int kb);
 int level_carveout_pct(const orion_device_limits &d, const orion_level &L);
 
 // ---- kernel registry + code generation (registry.cpp) -------------------------------------
-enum KernelKind { K_KNN = 0, K_NLM = 1, K_STENCIL = 2 };
+enum KernelKind { K_KNN = 0, K_NLM = 1, K_STENCIL = 2, K_SRAD = 3 };
 
 struct KernelDef {
     const char *id;

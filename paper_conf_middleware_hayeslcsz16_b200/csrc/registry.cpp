@@ -25,6 +25,7 @@ extern "C" const char liborion_ptx_nlm_direct[];
 extern "C" const char liborion_ptx_nlm_regheavy[];
 extern "C" const char liborion_ptx_hotspot[];
 extern "C" const char liborion_ptx_gen[];
+extern "C" const char liborion_ptx_srad[];
 
 namespace orion {
 
@@ -36,6 +37,7 @@ static const char *module_ptx(const char *module)
     if (!std::strcmp(module, "nlm_regheavy")) return liborion_ptx_nlm_regheavy;
     if (!std::strcmp(module, "hotspot")) return liborion_ptx_hotspot;
     if (!std::strcmp(module, "gen")) return liborion_ptx_gen;
+    if (!std::strcmp(module, "srad")) return liborion_ptx_srad;
     return nullptr;
 }
 
@@ -57,6 +59,8 @@ static const KernelDef kKernels[] = {
     {"nlm_f4_regheavy", 64, "orion_nlm_regheavy_f4_64", "nlm_regheavy", 8, 8, 8, 8, 6, K_NLM, 1, 0},
     {"hotspot_f32", 256, "orion_hotspot_f32_256", "hotspot", 32, 8, 128, 128, 1, K_STENCIL, 0, 0},
     {"hotspot_f32", 128, "orion_hotspot_f32_128", "hotspot", 32, 4, 128, 64, 1, K_STENCIL, 0, 0},
+    // srad: J tile (32+3)^2 + coefficient tile (32+1)^2 floats; reads 2 rows below the tile
+    {"srad_f32", 256, "orion_srad_f32_256", "srad", 32, 8, 32, 32, 2, K_SRAD, 0, (35 * 35 + 33 * 33) * 4},
 };
 
 const KernelDef *find_kernel(const char *id, int threads)

@@ -307,6 +307,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
 {
     if (!t || !a || !dev_src || !dev_dst) return fail(ORION_E_INVALID, "orion_tune_step_host: NULL");
     const KernelDef &def = *t->v->def;
+    if (def.kind == K_SRAD) return fail(ORION_E_INVALID, "orion_tune_step_host: not available for srad");
     const size_t elem = def.kind == K_STENCIL ? 4 : 16;
     const size_t row = (size_t)a->width * elem;
     const size_t in_bytes = (size_t)(a->src_row_end - a->src_row_begin) * row;
@@ -387,6 +388,7 @@ orion_status orion_host_pipe_create(orion_tuner *t, int width, int max_rows, int
     p->t = t;
     p->width = width;
     p->max_rows = max_rows;
+    if (t->v->def->kind == K_SRAD) return fail(ORION_E_INVALID, "orion_host_pipe_create: not available for srad");
     const bool stencil = t->v->def->kind == K_STENCIL;
     p->elem = stencil ? 4 : 16;
     const size_t bytes = (size_t)width * (size_t)max_rows * p->elem;

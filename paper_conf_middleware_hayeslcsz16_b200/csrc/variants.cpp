@@ -30,7 +30,7 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
     if (a->width <= 0 || a->height <= 0 || a->row_begin < 0 || a->row_end > a->height || a->row_begin > a->row_end)
         return fail(ORION_E_INVALID, "orion_launch: bad image geometry");
     if (a->row_begin == a->row_end) return ORION_OK;
-    if (!a->src || !a->dst || (def.kind == K_STENCIL && !a->aux))
+    if (!a->src || !a->dst || ((def.kind == K_STENCIL || def.kind == K_SRAD) && !a->aux))
         return fail(ORION_E_INVALID, "orion_launch: NULL buffer");
     const int need_lo = std::max(0, a->row_begin - def.halo);
     const int need_hi = std::min(a->height, a->row_end + def.halo);
@@ -48,8 +48,8 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
     k->src_row_begin = a->src_row_begin;
     k->src_row_end = a->src_row_end;
     k->dst_row_begin = a->dst_row_begin;
-    if (def.kind == K_STENCIL) {
-        for (int i = 0; i < 5; ++i) k->fparam[i] = a->fparam[i];
+    if (def.kind == K_STENCIL || def.kind == K_SRAD) {
+        for (int i = 0; i < 8; ++i) k->fparam[i] = a->fparam[i];
     } else {
         // SDK parameters -> kernel form: w = 2^(d * (-Noise log2 e) + geo); count threshold
         // "cnt/A > lthr" on an integer count == cnt >= floor(lthr*A) + 1.
@@ -328,3 +328,19 @@ orion_status orion_flush_l2(int device, void *buf, long long bytes, void *stream
 }
 
 }  // extern "C"
+
+extern "C" orion_status orion_srad_roi_stats(int device, const void *J, int width, int height, int r1, int r2, int c1,
+                                             int c2, void *q0, void *stream)
+{
+    if (!J || !q0 || width <= 0 || height <= 0 || r1 < 0 || c1 < 0 || r2 < r1 || c2 < c1 || r2 >= height ||
+        c2 >= width)
+        return fail(ORION_E_INVALID, "orion_srad_roi_stats: bad argument");
+    CUmodule m;
+    ORION_TRY(load_aux_module(device, "srad", &m));
+    CUfunction f;
+    ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_srad_stats"));
+    void *params[] = {&J, &width, &r1, &r2, &c1, &c2, &q0};
+    ORION_CU(drv().cuLaunchKernel(f, 1, 1, 1, 1024, 1, 1, 0, (CUstream)stream, params, nullptr));
+    g_launches.fetch_add(1);
+    return ORION_OK;
+}

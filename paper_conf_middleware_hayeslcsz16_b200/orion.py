@@ -31,8 +31,9 @@ SELECT_FASTEST, SELECT_LOWEST_WITHIN_TOL = 0, 1
 # threshold, lerp threshold (fraction of the 49 window taps).
 KNN_PARAMS = (1.0 / (0.32 * 0.32), 0.2, 0.02, 0.79)
 NLM_PARAMS = (1.0 / (1.45 * 1.45), 0.2, 0.10, 0.10)
-HALO = {"knn_f4": 3, "nlm_f4": 6, "nlm_f4_g1": 6, "nlm_f4_direct": 6, "nlm_f4_regheavy": 6, "hotspot_f32": 1}
-KERNELS = ("knn_f4", "nlm_f4", "nlm_f4_g1", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32")
+HALO = {"knn_f4": 3, "nlm_f4": 6, "nlm_f4_g1": 6, "nlm_f4_direct": 6, "nlm_f4_regheavy": 6, "hotspot_f32": 1,
+        "srad_f32": 2}
+KERNELS = ("knn_f4", "nlm_f4", "nlm_f4_g1", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32", "srad_f32")
 
 
 class OrionError(RuntimeError):
@@ -136,6 +137,7 @@ def lib() -> ctypes.CDLL:
                 "orion_generate_rgba": [I, V, I, I, I, I, ctypes.c_uint, ctypes.c_float, V],
                 "orion_generate_thermal": [I, V, V, I, I, ctypes.c_uint, V],
                 "orion_flush_l2": [I, V, ctypes.c_longlong, V],
+                "orion_srad_roi_stats": [I, V, I, I, I, I, I, I, V, V],
             }
             for name, args in sig.items():
                 f = getattr(L, name)
@@ -435,6 +437,19 @@ def generate_rgba(device: int, dst: int, width: int, height: int, row_begin: int
 def generate_thermal(device: int, t0: int, power: int, width: int, height: int, seed: int = 1, stream=None):
     _check(lib().orion_generate_thermal(device, ctypes.c_void_p(t0), ctypes.c_void_p(power), width, height, seed,
                                         _s(stream)), "orion_generate_thermal")
+
+
+def srad_args(j_in: int, j_out: int, q0: int, width: int, height: int, lam: float = 0.5) -> Args:
+    """Arguments of one "srad_f32" iteration; q0 = device address of the float q0sqr."""
+    a = Args(j_in, j_out, q0, width, height, 0, height, 0, height, 0)
+    a.fparam[0] = lam
+    return a
+
+
+def srad_roi_stats(device: int, j: int, width: int, height: int, roi, q0: int, stream=None):
+    r1, r2, c1, c2 = roi
+    _check(lib().orion_srad_roi_stats(device, ctypes.c_void_p(j), width, height, r1, r2, c1, c2, ctypes.c_void_p(q0),
+                                      _s(stream)), "orion_srad_roi_stats")
 
 
 def flush_l2(device: int, buf: int, nbytes: int, stream=None):
