@@ -255,7 +255,8 @@ def run_ours(args):
     nlev = len(variants)
     lv = [variants.level(i) for i in range(nlev)]
     infos = [variants.info(i) for i in range(nlev)]
-    orig = next(i for i, l in enumerate(variants.planned) if l.reg_cap == 0 and l.smem_pad_bytes == 0)
+    orig = max((i for i, l in enumerate(variants.planned) if l.reg_cap == 0),
+               key=lambda i: variants.planned[i].ctas_per_sm)   # the original / nvcc-default build
     kmax = nlev - 1
 
     # ---- inputs resident in HBM: a pool of frames larger than L2 -------------------------

@@ -268,8 +268,9 @@ def levels(dev: Device, T: int, natural_regs: int, smem_static: int = 0, smem_ne
 
 
 def original_level_index(lv: list[Level]) -> int:
-    """The 'original' version: uncapped registers, no padding."""
-    for i, l in enumerate(lv):
-        if l.reg_cap == 0 and l.smem_pad_bytes == 0:
-            return i
-    raise ValueError("no uncapped, unpadded level")
+    """The 'original' version: natural (uncapped) registers at the most CTAs
+    they admit -- the unpadded level when padding is the only other limiter."""
+    cands = [i for i, l in enumerate(lv) if l.reg_cap == 0]
+    if not cands:
+        raise ValueError("no uncapped level")
+    return max(cands, key=lambda i: lv[i].ctas_per_sm)

@@ -35,17 +35,21 @@ struct Fig9 {
     void prune(const orion_level *lv, int n, int natural_regs)
     {
         ks.resize(n);
-        int orig = -1;
+        // the original: the most CTAs the natural register count admits; a rung
+        // of the register ladder: the most CTAs a given register cap admits
+        std::map<int, int> top_of_cap;   // reg_cap -> level index with the largest k
         for (int i = 0; i < n; ++i) {
             ks[i] = lv[i].ctas_per_sm;
-            if (lv[i].reg_cap == 0 && lv[i].smem_pad_bytes == 0) orig = i;
+            auto it = top_of_cap.find(lv[i].reg_cap);
+            if (it == top_of_cap.end() || ks[i] > ks[it->second]) top_of_cap[lv[i].reg_cap] = i;
         }
+        const int orig = top_of_cap.at(0);
         const int k0 = ks[orig];
         std::vector<int> up, down;
-        for (int i = 0; i < n; ++i) {
-            if (lv[i].smem_pad_bytes == 0 && ks[i] > k0) up.push_back(i);   // register-cap rungs
+        for (auto &kv : top_of_cap)
+            if (ks[kv.second] > k0) up.push_back(kv.second);                // register-cap rungs
+        for (int i = 0; i < n; ++i)
             if (ks[i] < k0) down.push_back(i);                              // padding levels
-        }
         std::sort(up.begin(), up.end(), [&](int a, int b) { return ks[a] < ks[b]; });
         std::sort(down.begin(), down.end(), [&](int a, int b) { return ks[a] > ks[b]; });
         up.insert(up.begin(), orig);
@@ -144,8 +148,8 @@ orion_status check_levels(const orion_level *lv, int n)
 {
     if (!lv || n <= 0) return fail(ORION_E_INVALID, "no levels");
     for (int i = 0; i < n; ++i)
-        if (lv[i].reg_cap == 0 && lv[i].smem_pad_bytes == 0) return ORION_OK;
-    return fail(ORION_E_INVALID, "levels lack the original (uncapped, unpadded) version");
+        if (lv[i].reg_cap == 0) return ORION_OK;
+    return fail(ORION_E_INVALID, "levels lack the original (uncapped) version");
 }
 
 }  // namespace

@@ -89,14 +89,14 @@ def test_levels_capacity_protocol():
     assert "bad kernel resources" in O.lib().orion_last_error().decode()
 
 
-def _o_levels(T, natural, need=0):
-    ol = OC.levels(OC.B200, T, natural, 0, need)
+def _o_levels(T, natural, need=0, mode=0):
+    ol = OC.levels(OC.B200, T, natural, 0, need, mode=mode)
     return ol, [O.Level(*[getattr(l, f) for f, _ in O.Level._fields_]) for l in ol]
 
 
 
-def _replay_both(T, natural, need, ms, iters, **cfgkw):
-    ol, pl = _o_levels(T, natural, need)
+def _replay_both(T, natural, need, ms, iters, mode=0, **cfgkw):
+    ol, pl = _o_levels(T, natural, need, mode)
     ocfg = OT.TunerCfg(**{k: v for k, v in cfgkw.items()})
     pcfg = O.default_cfg(**{k: (int(v) if isinstance(v, bool) else v) for k, v in cfgkw.items()})
     tr = OT.replay(ol, natural, ocfg, ms, iters)
@@ -124,14 +124,14 @@ def test_replay_vectors_match_oracle(T, natural, need, ladder_ms, mode):
 
 @settings(max_examples=200, deadline=None)
 @given(st.sampled_from([(128, 255, 0), (128, 56, 0), (256, 20, 0), (256, 46, 0), (128, 128, 52544), (64, 39, 13376)]),
-       st.integers(0, 2**31 - 1), st.sampled_from([0, 1]), st.booleans(), st.integers(0, 20))
-def test_replay_random_tables_match_oracle(shape, seed, mode, switch, expected):
+       st.integers(0, 2**31 - 1), st.sampled_from([0, 1]), st.booleans(), st.integers(0, 20), st.sampled_from([0, 1]))
+def test_replay_random_tables_match_oracle(shape, seed, mode, switch, expected, realise):
     T, natural, need = shape
-    ol, _ = _o_levels(T, natural, need)
+    ol, _ = _o_levels(T, natural, need, realise)
     rng = random.Random(seed)
     ms = [round(rng.uniform(0.5, 2.0), 3) for _ in ol]
-    tr, ran, fin, fit = _replay_both(T, natural, need, ms, 25, select_mode=mode, allow_direction_switch=switch,
-                                     expected_iterations=expected)
+    tr, ran, fin, fit = _replay_both(T, natural, need, ms, 25, realise, select_mode=mode,
+                                     allow_direction_switch=switch, expected_iterations=expected)
     assert ran == tr.ran
     assert fin == (tr.final if tr.final is not None else -1)
     assert fit == (tr.final_iteration if tr.final_iteration is not None else -1)

@@ -125,3 +125,15 @@ def test_principle1_unimodal_walk_finds_global_argmin(argmin_pos, seed):
     assert TU.regret(ms[tr.final], ms[brute]) == 0.0
     # iterations spent exploring: up to the first worse level (or the whole ladder)
     assert tr.final_iteration == min(argmin_pos + 1, n - 1) + (1 if argmin_pos == n - 1 else 0)
+
+
+def test_fig8_ladders_under_min_carveout_realisation():
+    # the smallest-carveout realisation leaves some capped levels unpadded; the ladders are
+    # defined by register caps, so they do not change with the realisation
+    for T, natural, need in ((256, 30, 9256), (128, 255, 11264), (256, 46, 0)):
+        a = O.levels(O.B200, T, natural, 0, need)
+        b = O.levels(O.B200, T, natural, 0, need, mode=O.REALISE_MIN_CARVEOUT)
+        ca, cb = TU.candidates(a, natural, TU.TunerCfg()), TU.candidates(b, natural, TU.TunerCfg())
+        assert ca[0] == cb[0]
+        assert ladder_ks(a, ca[1]) == ladder_ks(b, cb[1]) and ladder_ks(a, ca[2]) == ladder_ks(b, cb[2])
+        assert O.original_level_index(a) == O.original_level_index(b)

@@ -18,7 +18,7 @@ torch.cuda.set_device(0)
 sp = torch.cuda.current_stream().cuda_stream
 v, res = O.build_all_levels(0, kernel, threads)
 if lev == "orig":
-    li = next(i for i, l in enumerate(v.planned) if l.reg_cap == 0 and l.smem_pad_bytes == 0)
+    li = max((i for i, l in enumerate(v.planned) if l.reg_cap == 0), key=lambda i: v.planned[i].ctas_per_sm)
 else:
     li = int(lev) % len(v)
 if kernel == "hotspot_f32":
