@@ -41,7 +41,7 @@ extern "C" __global__ void __launch_bounds__(256) orion_srad_f32_256(orion_kargs
     }
     const float q0 = *(const float *)a.aux;
     const float lam4 = __fmul_rn(0.25f, a.fparam[0]);
-    const float qden = __fmul_rn(q0, __fadd_rn(1.0f, q0));
+    const float iqden = __frcp_rn(__fmul_rn(q0, __fadd_rn(1.0f, q0)));
     __syncthreads();
     // coefficient tile: cell (y0+cy, x0+cx), cy in [0, CH), cx in [0, CW).  The cell at
     // global (gy, gx) with gy >= H or gx >= W is a clamped copy: its coefficient is the
@@ -58,13 +58,16 @@ extern "C" __global__ void __launch_bounds__(256) orion_srad_f32_256(orion_kargs
         const float dW = __fsub_rn(js[ty * JW + tw], Jc), dE = __fsub_rn(js[ty * JW + te], Jc);
         const float g2n = __fadd_rn(__fadd_rn(__fadd_rn(__fmul_rn(dN, dN), __fmul_rn(dS, dS)), __fmul_rn(dW, dW)),
                                     __fmul_rn(dE, dE));
-        const float G2 = __fdiv_rn(g2n, __fmul_rn(Jc, Jc));
-        const float L = __fdiv_rn(__fadd_rn(__fadd_rn(__fadd_rn(dN, dS), dW), dE), Jc);
+        // one IEEE reciprocal of J serves G2 = sum d^2 / J^2 and L = sum d / J; the
+        // (qsqr - q0sqr) / (q0sqr (1 + q0sqr)) division uses the launch-uniform reciprocal
+        const float ij = __frcp_rn(Jc);
+        const float G2 = __fmul_rn(__fmul_rn(g2n, ij), ij);
+        const float L = __fmul_rn(__fadd_rn(__fadd_rn(__fadd_rn(dN, dS), dW), dE), ij);
         const float num = __fsub_rn(__fmul_rn(0.5f, G2), __fmul_rn(0.0625f, __fmul_rn(L, L)));
         const float den = __fadd_rn(1.0f, __fmul_rn(0.25f, L));
         const float qsqr = __fdiv_rn(num, __fmul_rn(den, den));
-        const float dd = __fdiv_rn(__fsub_rn(qsqr, q0), qden);
-        const float c = __fdiv_rn(1.0f, __fadd_rn(1.0f, dd));
+        const float dd = __fmul_rn(__fsub_rn(qsqr, q0), iqden);
+        const float c = __frcp_rn(__fadd_rn(1.0f, dd));
         cs[idx] = fminf(fmaxf(c, 0.0f), 1.0f);
     }
     __syncthreads();
