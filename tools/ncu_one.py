@@ -21,7 +21,15 @@ if lev == "orig":
     li = max((i for i, l in enumerate(v.planned) if l.reg_cap == 0), key=lambda i: v.planned[i].ctas_per_sm)
 else:
     li = int(lev) % len(v)
-if kernel == "hotspot_f32":
+if kernel == "srad_f32":
+    a = torch.empty((H, W), device="cuda")
+    b = torch.empty((H, W), device="cuda")
+    p = torch.empty((H, W), device="cuda")
+    q0 = torch.empty(1, device="cuda")
+    O.generate_thermal(0, a.data_ptr(), p.data_ptr(), W, H, stream=sp)
+    O.srad_roi_stats(0, a.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
+    args = O.srad_args(a.data_ptr(), b.data_ptr(), q0.data_ptr(), W, H)
+elif kernel == "hotspot_f32":
     a = torch.empty((H, W), device="cuda")
     b = torch.empty((H, W), device="cuda")
     p = torch.empty((H, W), device="cuda")
