@@ -177,6 +177,111 @@ ORION_DEVICE void phase_b(const float *pr, const float *pg, const float *pb, con
     }
 }
 
+// ---- integer box sums ------------------------------------------------------------------
+// d in [0, 3] (pixels in [0, 1]) is quantised once to a fixed-point integer with 21 fraction
+// bits by a single rounding: bits(fma(d, 2^21, 2^23)) = bits(2^23) + round(d 2^21).  Box sums of
+// those integers are exact, so the 7-term windows slide with one IADD3 per output (the 2^23
+// offsets cancel in the slides; the first window subtracts 7 of them, in wrapping uint32
+// arithmetic).  |error| per difference <= 2^-22, per patch sum <= 49 * 2^-22 = 1.2e-5: a weight
+// error <= 5.7e-6 relative, inside the R-AMB band and the 1e-5 output tolerance.
+constexpr float kQScale = 2097152.0f;            // 2^21
+constexpr float kQMagic = 8388608.0f;            // 2^23
+constexpr unsigned kQMagicBits = 0x4B000000u;    // bits of 2^23
+
+ORION_DEVICE unsigned quant(float d) { return __float_as_uint(__fmaf_rn(d, kQScale, kQMagic)); }
+
+// Sliding 7-term sums of the raw quantised words q[0 .. N+5] (each = magic + value).
+template <int N>
+ORION_DEVICE void window7_q(const unsigned (&q)[N + 6], unsigned (&out)[N])
+{
+    unsigned s = q[0] + q[1] + q[2] + q[3] + q[4] + q[5] + q[6] - 7u * kQMagicBits;
+    out[0] = s;
+#pragma unroll
+    for (int k = 1; k < N; ++k) {
+        s = s + q[k + 6] - q[k - 1];
+        out[k] = s;
+    }
+}
+
+// Sliding 7-term sums of exact integers h[0 .. N+5].
+template <int N>
+ORION_DEVICE void window7_i(const unsigned (&h)[N + 6], unsigned (&out)[N])
+{
+    unsigned s = h[0] + h[1] + h[2] + h[3] + h[4] + h[5] + h[6];
+    out[0] = s;
+#pragma unroll
+    for (int k = 1; k < N; ++k) {
+        s = s + h[k + 6] - h[k - 1];
+        out[k] = s;
+    }
+}
+
+template <int G>
+ORION_DEVICE void phase_a_int(const float *pr, const float *pg, const float *pb, unsigned *hs, int lane, int warp,
+                              int i, int j1)
+{
+    const int cb = 3 + 32 * warp;
+    const int rowc = lane * PW + cb;
+    const int rows = rowc + i * PW + j1;
+    float wr[G], wg[G], wb[G];
+#pragma unroll
+    for (int g = 0; g < G - 1; ++g) {
+        wr[g + 1] = pr[rows + g];
+        wg[g + 1] = pg[rows + g];
+        wb[g + 1] = pb[rows + g];
+    }
+    unsigned q[G][38];
+#pragma unroll
+    for (int c = 0; c < 38; ++c) {
+#pragma unroll
+        for (int g = 0; g < G - 1; ++g) {
+            wr[g] = wr[g + 1];
+            wg[g] = wg[g + 1];
+            wb[g] = wb[g + 1];
+        }
+        wr[G - 1] = pr[rows + c + G - 1];
+        wg[G - 1] = pg[rows + c + G - 1];
+        wb[G - 1] = pb[rows + c + G - 1];
+        const float cr = pr[rowc + c], cg = pg[rowc + c], cbv = pb[rowc + c];
+#pragma unroll
+        for (int g = 0; g < G; ++g) q[g][c] = quant(diff2(wr[g], wg[g], wb[g], cr, cg, cbv));
+    }
+#pragma unroll
+    for (int g = 0; g < G; ++g) {
+        unsigned h[32];
+        window7_q<32>(q[g], h);
+        unsigned *hrow = hs + g * HBUF + lane * HP + 32 * warp;
+#pragma unroll
+        for (int c = 0; c < 32; ++c) hrow[c] = h[c];
+    }
+}
+
+ORION_DEVICE void phase_b_int(const float *pr, const float *pg, const float *pb, const unsigned *hb, int t, int i,
+                              int j, float nl2q, float wthr, Acc &A)
+{
+    const float geo = geo_l2_rt(i, j);
+    unsigned hp[TH + 6], hm[TH + 6], Dp[TH], Dm[TH];
+#pragma unroll
+    for (int c = 0; c < TH + 6; ++c) {
+        hp[c] = hb[(c + 3) * HP + t + 3];           // +o: H column t+3, rows 3 .. TH+8
+        hm[c] = hb[(c + 3 - i) * HP + t + 3 - j];   // -o: H column t+3-j, rows 3-i .. TH+8-i
+    }
+    window7_i<TH>(hp, Dp);
+    window7_i<TH>(hm, Dm);
+#pragma unroll
+    for (int r = 0; r < TH; ++r) {
+        const float wp = ex2(__fmaf_rn(__uint2float_rn(Dp[r]), nl2q, geo));
+        const float wm = ex2(__fmaf_rn(__uint2float_rn(Dm[r]), nl2q, geo));
+        const int pp = (r + 6 + i) * PW + t + 9 + j;      // p(x+j, y+i)
+        const int pm = (r + 6 - i) * PW + t + 9 - j;      // p(x-j, y-i)
+        A.axy[r] = fma2(make_float2(wp, wp), make_float2(pr[pp], pg[pp]), A.axy[r]);
+        A.azs[r] = fma2(make_float2(wp, wp), make_float2(pb[pp], 1.0f), A.azs[r]);
+        A.axy[r] = fma2(make_float2(wm, wm), make_float2(pr[pm], pg[pm]), A.axy[r]);
+        A.azs[r] = fma2(make_float2(wm, wm), make_float2(pb[pm], 1.0f), A.azs[r]);
+        A.cnt[r >> 2] += (((wp > wthr) ? 1u : 0u) + ((wm > wthr) ? 1u : 0u)) << (8 * (r & 3));
+    }
+}
+
 // Pass tables: (i, j1, G).  Together they cover the 24 half-plane pairs exactly once.
 __constant__ int kPass1[24][3] = {
     {0, 1, 1}, {0, 2, 1}, {0, 3, 1},
@@ -186,7 +291,7 @@ __constant__ int kPass1[24][3] = {
 __constant__ int kPass3[10][3] = {
     {0, 1, 3}, {1, -3, 3}, {1, 0, 2}, {1, 2, 2}, {2, -3, 3}, {2, 0, 2}, {2, 2, 2}, {3, -3, 3}, {3, 0, 2}, {3, 2, 2}};
 
-template <int GMAX>
+template <int GMAX, bool INT>
 __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 {
     extern __shared__ float4 smem4[];
@@ -235,16 +340,31 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
         const int i = GMAX == 1 ? kPass1[ps][0] : kPass3[ps][0];
         const int j1 = GMAX == 1 ? kPass1[ps][1] : kPass3[ps][1];
         const int G = GMAX == 1 ? 1 : kPass3[ps][2];
-        if (GMAX == 1 || G == 1)
-            phase_a<1>(pr, pg, pb, hs, lane, warp, i, j1);
-        else if (G == 2)
-            phase_a<2>(pr, pg, pb, hs, lane, warp, i, j1);
-        else
-            phase_a<(GMAX >= 3 ? 3 : 1)>(pr, pg, pb, hs, lane, warp, i, j1);
+        unsigned *hi = reinterpret_cast<unsigned *>(hs);
+        if (INT) {
+            if (GMAX == 1 || G == 1)
+                phase_a_int<1>(pr, pg, pb, hi, lane, warp, i, j1);
+            else if (G == 2)
+                phase_a_int<2>(pr, pg, pb, hi, lane, warp, i, j1);
+            else
+                phase_a_int<(GMAX >= 3 ? 3 : 1)>(pr, pg, pb, hi, lane, warp, i, j1);
+        } else {
+            if (GMAX == 1 || G == 1)
+                phase_a<1>(pr, pg, pb, hs, lane, warp, i, j1);
+            else if (G == 2)
+                phase_a<2>(pr, pg, pb, hs, lane, warp, i, j1);
+            else
+                phase_a<(GMAX >= 3 ? 3 : 1)>(pr, pg, pb, hs, lane, warp, i, j1);
+        }
         __syncthreads();
         if (t < TW) {
 #pragma unroll 1
-            for (int g = 0; g < G; ++g) phase_b(pr, pg, pb, hs + g * HBUF, t, i, j1 + g, nl2, wthr, A);
+            for (int g = 0; g < G; ++g) {
+                if (INT)
+                    phase_b_int(pr, pg, pb, hi + g * HBUF, t, i, j1 + g, nl2 * (1.0f / kQScale), wthr, A);
+                else
+                    phase_b(pr, pg, pb, hs + g * HBUF, t, i, j1 + g, nl2, wthr, A);
+            }
         }
         __syncthreads();
     }
@@ -265,6 +385,8 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 }  // namespace
 
 // One pair per pass: 3 planar planes + 1 H buffer = 75 732 B of shared memory.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kargs a) { nlm_box_body<1>(a); }
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kargs a) { nlm_box_body<1, false>(a); }
 // Up to three pairs per pass: 3 planar planes + 3 H buffers = 108 756 B of shared memory.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_box3_f4_128(orion_kargs a) { nlm_box_body<3>(a); }
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_box3_f4_128(orion_kargs a) { nlm_box_body<3, false>(a); }
+// Integer (fixed-point, exact) box sums, up to three pairs per pass.
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_boxi3_f4_128(orion_kargs a) { nlm_box_body<3, true>(a); }

@@ -51,6 +51,9 @@ static const KernelDef kKernels[] = {
     // up to 3 offset pairs per pass: 3 H_o buffers (2 CTAs/SM) -- the C2 / C5 default
     {"nlm_f4", 128, "orion_nlm_box3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
      3 * 35 * 141 * 4 + 3 * 32 * 129 * 4},
+    // same, integer (fixed-point, exact) box sums
+    {"nlm_f4_i", 128, "orion_nlm_boxi3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
+     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4},
     // one offset pair per pass: 1 H_o buffer (3 CTAs/SM)
     {"nlm_f4_g1", 128, "orion_nlm_box_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
      3 * 35 * 141 * 4 + 32 * 129 * 4},

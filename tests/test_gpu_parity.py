@@ -136,7 +136,7 @@ def test_knn_ragged_and_degenerate(dev, shape):
     check_vs_oracle(outs[0], out, alt, amb)
 
 
-@pytest.mark.parametrize("kernel", ["nlm_f4", "nlm_f4_g1"])
+@pytest.mark.parametrize("kernel", ["nlm_f4", "nlm_f4_g1", "nlm_f4_i"])
 @pytest.mark.parametrize("sigma", [0.05, 0.13, 0.2])
 def test_nlm_box_all_levels(dev, sigma, kernel):
     img = synth.noisy_rgba(250, 131, seed=2, sigma=sigma)
@@ -174,7 +174,8 @@ def _sample_points(W, H, n, seed):
     return np.array(xs), np.array(ys)
 
 
-@pytest.mark.parametrize("kernel,size", [("nlm_f4", 2048), ("knn_f4", 2048), ("nlm_f4_regheavy", 4096)])
+@pytest.mark.parametrize("kernel,size", [("nlm_f4", 2048), ("nlm_f4_i", 2048), ("knn_f4", 2048),
+                                         ("nlm_f4_regheavy", 4096)])
 def test_full_size_sampled(dev, kernel, size):
     # C2 / C4 sizes, launched as bench.py launches them (max-occupancy and original levels)
     W = H = size
