@@ -226,8 +226,11 @@ def realise(dev: Device, T: int, regs: int, smem_static: int, smem_need: int, k:
         if pad is None:
             return None
         return pad, (dev.smem_per_sm // 1024 if pad > 0 else 0)
+    need_alloc = smem_alloc_per_cta(dev, smem_static, smem_need)
     for kb in CARVEOUT_KB:
-        if kb == 0 or kb * 1024 > dev.smem_per_sm:
+        # a configuration smaller than one CTA would be raised by the driver: skip it so
+        # carveout_kb names the configuration actually used
+        if kb == 0 or kb * 1024 > dev.smem_per_sm or kb * 1024 < need_alloc:
             continue
         pct = carveout_pct_for(dev, kb)
         if carveout_budget(dev, pct) != kb * 1024:

@@ -131,8 +131,11 @@ bool realise(const orion_device_limits &d, int T, int regs, int smem_static, int
         *carveout_kb = p > 0 ? d.smem_per_sm / 1024 : 0;
         return true;
     }
+    const int need_alloc = round_up(smem_static + d.smem_reserved_per_block + smem_need, d.smem_alloc_unit);
     for (int kb : kCarveoutKB) {
-        if (kb == 0 || (long long)kb * 1024 > d.smem_per_sm) continue;
+        // configurations too small for one CTA would be raised by the driver: skip them so
+        // carveout_kb names the configuration actually used
+        if (kb == 0 || (long long)kb * 1024 > d.smem_per_sm || kb * 1024 < need_alloc) continue;
         const int pct = carveout_pct_for_kb(d, kb);
         if (carveout_pref_bytes(d, pct) != kb * 1024) continue;
         const int p = pad_for_level(d, T, regs, smem_static, smem_need, k, pct);

@@ -26,6 +26,7 @@ extern "C" const char liborion_ptx_nlm_regheavy[];
 extern "C" const char liborion_ptx_hotspot[];
 extern "C" const char liborion_ptx_gen[];
 extern "C" const char liborion_ptx_srad[];
+extern "C" const char liborion_ptx_nlm_box256[];
 
 namespace orion {
 
@@ -38,6 +39,7 @@ static const char *module_ptx(const char *module)
     if (!std::strcmp(module, "hotspot")) return liborion_ptx_hotspot;
     if (!std::strcmp(module, "gen")) return liborion_ptx_gen;
     if (!std::strcmp(module, "srad")) return liborion_ptx_srad;
+    if (!std::strcmp(module, "nlm_box256")) return liborion_ptx_nlm_box256;
     return nullptr;
 }
 
@@ -53,6 +55,9 @@ static const KernelDef kKernels[] = {
      3 * 35 * 141 * 4 + 3 * 32 * 129 * 4},
     // same, integer (fixed-point, exact) box sums
     {"nlm_f4_i", 128, "orion_nlm_boxi3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
+     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4},
+    // same tile, 256 threads (8 warps per CTA)
+    {"nlm_f4_w8", 256, "orion_nlm_box256_f4_256", "nlm_box256", 256, 1, 122, 23, 6, K_NLM, 0,
      3 * 35 * 141 * 4 + 3 * 32 * 129 * 4},
     // one offset pair per pass: 1 H_o buffer (3 CTAs/SM)
     {"nlm_f4_g1", 128, "orion_nlm_box_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,

@@ -136,7 +136,7 @@ def test_knn_ragged_and_degenerate(dev, shape):
     check_vs_oracle(outs[0], out, alt, amb)
 
 
-@pytest.mark.parametrize("kernel", ["nlm_f4", "nlm_f4_g1", "nlm_f4_i"])
+@pytest.mark.parametrize("kernel", ["nlm_f4", "nlm_f4_g1", "nlm_f4_i", "nlm_f4_w8"])
 @pytest.mark.parametrize("sigma", [0.05, 0.13, 0.2])
 def test_nlm_box_all_levels(dev, sigma, kernel):
     img = synth.noisy_rgba(250, 131, seed=2, sigma=sigma)
