@@ -423,6 +423,20 @@ def run_ours(args):
                 pj = json.load(f)
             ent = pj.get(kernel) or {}
             roof["traffic"] = ent.get("dram_bytes_per_launch")
+            m = ent.get("metrics", {})
+
+            def num(k):
+                return float(m[k].split()[0].replace(",", ""))
+            # the resource that actually binds the denoisers: shared-memory wavefronts per SM
+            # cycle (1 / clk / SM peak) and the issue slots, from the committed ncu capture
+            wf = num("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum")
+            dur = num("gpu__time_duration.sum") * {"ns": 1e-9, "us": 1e-6, "ms": 1e-3}.get(
+                m["gpu__time_duration.sum"].split()[-1][:2], 1e-6)
+            clk = num("sm__cycles_elapsed.avg.per_second") * 1e9
+            roof["ncu"] = {"report": ent.get("report"), "smem_wavefront_frac": wf / (148 * dur * clk),
+                           "issue_active_pct": num("smsp__issue_active.avg.pct_of_peak_sustained_active"),
+                           "lsu_pipe_pct": num("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active"),
+                           "fma_pipe_pct": num("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active")}
         except Exception:
             pass
     roof["kernel"] = kernel
