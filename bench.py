@@ -132,6 +132,23 @@ class ClockSampler:
                 "reasons": sorted(self.reasons - {"gpu_idle"}), "samples": len(self.samples)}
 
 
+def init_dist(world: int, local: int) -> int:
+    """One process per GPU: bind the device and (N > 1) the NCCL process group.  The
+    ORION_BENCH_BACKEND=gloo override exists only to exercise the multi-rank control flow
+    on a single-GPU box (ranks then share device local % device_count)."""
+    import torch
+    import torch.distributed as dist
+    backend = os.environ.get("ORION_BENCH_BACKEND", "nccl")
+    dev = local % max(1, torch.cuda.device_count()) if backend != "nccl" else local
+    torch.cuda.set_device(dev)
+    if world > 1:
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group(backend)
+    return dev
+
+
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -236,9 +253,7 @@ def run_ours(args):
     world, rank, local = dist_env()
     if not torch.cuda.is_available():
         raise SystemExit("bench.py: no CUDA device (the product has no CPU path)")
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    local = init_dist(world, local)
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream
@@ -502,9 +517,7 @@ def run_c5(args):
     from paper_conf_middleware_hayeslcsz16_b200 import shard
 
     world, rank, local = dist_env()
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    local = init_dist(world, local)
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream

@@ -53,5 +53,11 @@ def gather_bands(out_band, full_out, group=None):
     `full_out`: (world * rows_per_rank, ...) tensor; rows [0, height) hold the image after.
     """
     import torch.distributed as dist
+    if full_out.is_cuda and dist.get_backend(group) != "nccl":
+        # control-flow checks on a single-GPU box (gloo): stage through host memory
+        host = full_out.new_empty(full_out.shape, device="cpu")
+        dist.all_gather_into_tensor(host, out_band.contiguous().cpu(), group=group)
+        full_out.copy_(host)
+        return full_out
     dist.all_gather_into_tensor(full_out, out_band.contiguous(), group=group)
     return full_out
