@@ -447,8 +447,8 @@ def run_ours(args):
             wf = num("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum")
             dur = num("gpu__time_duration.sum") * {"ns": 1e-9, "us": 1e-6, "ms": 1e-3}.get(
                 m["gpu__time_duration.sum"].split()[-1][:2], 1e-6)
-            clk = num("sm__cycles_elapsed.avg.per_second") * 1e9
-            roof["ncu"] = {"report": ent.get("report"), "smem_wavefront_frac": wf / (148 * dur * clk),
+            sm_hz = num("sm__cycles_elapsed.avg.per_second") * 1e9
+            roof["ncu"] = {"report": ent.get("report"), "smem_wavefront_frac": wf / (148 * dur * sm_hz),
                            "issue_active_pct": num("smsp__issue_active.avg.pct_of_peak_sustained_active"),
                            "lsu_pipe_pct": num("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active"),
                            "fma_pipe_pct": num("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active")}
