@@ -366,7 +366,8 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     final, iters_to_final = tuner.final()
-    units_per_step = W * H
+    spl = 2 if kernel == "hotspot2_f32" else 1        # stencil steps per launch (temporal blocking)
+    units_per_step = W * H * spl
     value = world * units_per_step * args.steps / (total_ms * 1e-3) / 1e6
     ms_step = total_ms / args.steps
     t_final = ms[final] if final >= 0 else float("nan")
@@ -420,7 +421,7 @@ def run_ours(args):
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     kernel_ms = ms_step  # one launch per steady-state step; the stream holds only our kernel
     if is_stencil:
-        achieved = wl["bytes"] * units_per_step / (kernel_ms * 1e-3) / 1e9
+        achieved = wl["bytes"] * W * H / (kernel_ms * 1e-3) / 1e9   # bytes per launch (T, P in; T' out)
         roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / peaks["hbm_gbs"], "peak_kind": peak_kind + " (copy bandwidth)"}
     else:

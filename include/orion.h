@@ -119,7 +119,7 @@ orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int bloc
 /* ---- code generation (question 1; host-only, no GPU needed) ------------------------------ */
 
 /* Kernel ids: "knn_f4", "nlm_f4", "nlm_f4_g1", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32",
- * "srad_f32".
+ * "hotspot2_f32" (two stencil steps per launch; width % 4 == 0), "srad_f32".
  * block_threads = 0 selects the kernel's default CTA size.  Fills the natural resources
  * (compiles the kernel's PTX once, uncapped, with the embedded ptxas). */
 orion_status orion_kernel_probe(const char *kernel_id, int block_threads, orion_kernel_resources *out);

@@ -57,6 +57,8 @@ struct KernelDef {
     int kind;               // KernelKind
     int smem_tile;          // 1: stages a (tile + halo) float4 tile in dynamic smem; 0: none
     int smem_bytes;         // > 0: explicit dynamic shared-memory need (overrides smem_tile)
+    int width_align;        // > 1: the image width must be a multiple of this
+    int steps_per_launch;   // stencil steps one launch performs (0 / 1 = one)
     int dyn_need() const
     {
         if (smem_bytes > 0) return smem_bytes;

@@ -67,6 +67,8 @@ static const KernelDef kKernels[] = {
     {"nlm_f4_regheavy", 64, "orion_nlm_regheavy_f4_64", "nlm_regheavy", 8, 8, 8, 8, 6, K_NLM, 1, 0},
     {"hotspot_f32", 256, "orion_hotspot_f32_256", "hotspot", 32, 8, 128, 128, 1, K_STENCIL, 0, 0},
     {"hotspot_f32", 128, "orion_hotspot_f32_128", "hotspot", 32, 4, 128, 64, 1, K_STENCIL, 0, 0},
+    // two steps per launch (temporal blocking): reads 2 rows beyond its strip; width % 4 == 0
+    {"hotspot2_f32", 256, "orion_hotspot2_f32_256", "hotspot", 32, 8, 128, 128, 2, K_STENCIL, 0, 0, 4, 2},
     // srad: J tile (32+3)^2 + coefficient tile (32+1)^2 floats; reads 2 rows below the tile
     {"srad_f32", 256, "orion_srad_f32_256", "srad", 32, 8, 32, 32, 2, K_SRAD, 0, (35 * 35 + 33 * 33) * 4},
 };

@@ -37,6 +37,9 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
     if (a->src_row_begin > need_lo || a->src_row_end < need_hi)
         return fail(ORION_E_INVALID, "orion_launch: src rows do not cover the halo of the output rows");
     if (a->dst_row_begin > a->row_begin) return fail(ORION_E_INVALID, "orion_launch: dst_row_begin > row_begin");
+    if (def.width_align > 1 && a->width % def.width_align)
+        return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + " needs width % " +
+                                         std::to_string(def.width_align) + " == 0");
     std::memset(k, 0, sizeof *k);
     k->src = a->src;
     k->dst = a->dst;

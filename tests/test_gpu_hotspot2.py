@@ -1,0 +1,57 @@
+"""hotspot2_f32 (two explicit steps per launch, the intermediate step kept in registers):
+bit-identical to two launches of the one-step kernel and to the oracle's fp32 form, at every
+occupancy level, on ragged heights and at the image borders."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
+
+
+@pytest.fixture(scope="module")
+def v2():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return O.build_all_levels(0, "hotspot2_f32", mode=O.REALISE_MIN_CARVEOUT)[0]
+
+
+def run(v, level, t0, pw, launches):
+    sp = torch.cuda.current_stream().cuda_stream
+    H, W = t0.shape
+    a = torch.from_numpy(t0).cuda()
+    b = torch.empty_like(a)
+    p = torch.from_numpy(pw).cuda()
+    for _ in range(launches):
+        v.launch(level, O.hotspot_args(a.data_ptr(), b.data_ptr(), p.data_ptr(), W, H), sp)
+        a, b = b, a
+    torch.cuda.synchronize()
+    return a.cpu().numpy()
+
+
+@pytest.mark.parametrize("shape", [(300, 203), (128, 1), (132, 2), (260, 3), (512, 129), (4, 37)])
+def test_two_steps_bit_exact_vs_oracle_fp32(v2, shape):
+    W, H = shape
+    t0, pw = synth.thermal_inputs(W, H, seed=5)
+    ref = oracle.hotspot(t0, pw, 10, precision="f32")
+    for lvl in (0, len(v2) - 1):
+        assert np.array_equal(run(v2, lvl, t0, pw, 5), ref), (shape, lvl)
+
+
+def test_all_levels_identical(v2):
+    t0, pw = synth.thermal_inputs(520, 300, seed=1)
+    outs = [run(v2, i, t0, pw, 3) for i in range(len(v2))]
+    for o in outs[1:]:
+        assert np.array_equal(o, outs[0])
+    assert np.array_equal(outs[0], oracle.hotspot(t0, pw, 6, precision="f32"))
+
+
+def test_unaligned_width_rejected(v2):
+    t0, pw = synth.thermal_inputs(130, 20, seed=1)
+    with pytest.raises(O.OrionError) as e:
+        run(v2, 0, np.ascontiguousarray(t0[:, :129]), np.ascontiguousarray(pw[:, :129]), 1)
+    assert e.value.status == -1
