@@ -260,7 +260,7 @@ def run_ours(args):
     wl = WORKLOADS[args.workload]
     kernel, W, H = args.kernel or wl["kernel"], wl["W"], wl["H"]
     is_srad = kernel == "srad_f32"
-    is_stencil = kernel == "hotspot_f32" or is_srad
+    is_stencil = kernel in ("hotspot_f32", "hotspot2_f32") or is_srad
 
     # ---- multi-version binary: probe -> levels -> build (offline, untimed) ----------------
     t_build = time.perf_counter()
