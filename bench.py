@@ -45,7 +45,8 @@ WORKLOADS = {
     # register-heavy direct NLM: 2401 patch terms x 6 + 49 x 6 per-offset terms + blend
     "c4": dict(kernel="nlm_f4_regheavy", W=4096, H=4096, sigma=0.13, unit="Mpix/s",
                name="register-heavy NLM 4096x4096 RGBA, maxrregcount caps", insts=2401 * 6 + 49 * 6 + 10, bytes=32),
-    "c3": dict(kernel="hotspot_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
+    # thermal stencil: two explicit steps per launch (hotspot2_f32), 12 B per cell per launch
+    "c3": dict(kernel="hotspot2_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
                insts=12, bytes=12),
     # NEXT-4: a second Rodinia stencil (srad), 8 B/cell-iteration (read J, write J')
     "srad": dict(kernel="srad_f32", W=8192, H=8192, unit="Mcell-steps/s", name="SRAD 8192x8192 fp32 (NEXT-4)",
@@ -226,8 +227,10 @@ def run_reference(args):
     per_step = max(0.2, min(2.0, 150.0 / max(1, K + Wm)))
     times, units = [], []
     for s in range(Wm + K):
-        if wl["kernel"] == "hotspot_f32":
+        if wl["kernel"].startswith("hotspot"):
             u, dt, sample = cpu_baseline_hotspot(wl["W"], 1, per_step)
+        elif wl["kernel"] == "srad_f32":
+            u, dt, sample = cpu_baseline_srad(wl["W"], 1, per_step)
         else:
             u, dt, sample = cpu_baseline_nlm("knn" if wl["kernel"].startswith("knn") else "nlm", wl["W"], wl["H"],
                                              wl.get("sigma", 0.13), per_step)
@@ -331,7 +334,8 @@ def run_ours(args):
     worst = max(range(nlev), key=lambda i: ms[i])
 
     # ---- the tuned loop: warmup (includes Fig. 9 exploration) then K timed steps ----------
-    cfg = O.default_cfg(select_mode=O.SELECT_LOWEST_WITHIN_TOL if args.select == "lowest" else O.SELECT_FASTEST)
+    cfg = O.default_cfg(select_mode=O.SELECT_LOWEST_WITHIN_TOL if args.select == "lowest" else O.SELECT_FASTEST,
+                        samples_per_level=args.samples)
     tuner = O.Tuner(variants, cfg)
     direction, ladder = tuner.ladder()
     if is_stencil:
@@ -615,6 +619,7 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
     ap.add_argument("--kernel", default="", help="override the workload's kernel id (same family)")
+    ap.add_argument("--samples", type=int, default=1, help="timed launches per explored level (paper: 1)")
     ap.add_argument("--select", choices=["fastest", "lowest"], default="fastest",
                     help="final-kernel rule: fastest measured, or lowest occupancy within 2%% (resource saving)")
     ap.add_argument("--realise", choices=["max", "min"], default="min",

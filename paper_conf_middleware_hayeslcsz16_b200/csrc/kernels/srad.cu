@@ -124,3 +124,86 @@ extern "C" __global__ void __launch_bounds__(1024) orion_srad_stats(const float 
         *q0 = (float)(var / (mean * mean));
     }
 }
+
+// ---- register-sliding variant ------------------------------------------------------------
+// Same arithmetic, no shared memory: lane l of a warp owns column x0 + l (x0 = 31 * block
+// column; lanes 0..30 write, lane 31 only supplies the coefficient its west neighbour needs
+// as c_E) and walks a strip of RY rows keeping J rows y-1 .. y+2 and the coefficients of rows
+// y, y+1 in registers.  E / W neighbours come by shuffle; lanes 0 / 31 load the column just
+// outside the warp.  One coefficient per cell, one coalesced 128-byte row load per step.
+namespace {
+struct JRow {
+    float c, w, e;   // J at the lane's column and at its west / east neighbours
+};
+}  // namespace
+
+template <int BY, int RY>
+__device__ __forceinline__ void srad2_body(const orion_kargs &a)
+{
+    const float *J = (const float *)a.src;
+    float *Jo = (float *)a.dst;
+    const int W = a.width, H = a.height;
+    const int lane = threadIdx.x;
+    const int x0 = blockIdx.x * 31;
+    const int xr = x0 + lane;
+    const int x = min(xr, W - 1);
+    const int ys = a.row_begin + (blockIdx.y * BY + threadIdx.y) * RY;
+    if (ys >= a.row_end) return;
+    const int ye = min(ys + RY, a.row_end);
+    const size_t sb = (size_t)a.src_row_begin;
+    const float q0 = *(const float *)a.aux;
+    const float lam4 = __fmul_rn(0.25f, a.fparam[0]);
+    const float iqden = __frcp_rn(__fmul_rn(q0, __fadd_rn(1.0f, q0)));
+    const int xw = clampi(x0 - 1, 0, W - 1), xe = clampi(x0 + 32, 0, W - 1);
+
+    auto load = [&](int y) {
+        const float *row = J + ((size_t)y - sb) * (size_t)W;
+        JRow r;
+        r.c = __ldg(row + x);
+        r.w = __shfl_up_sync(0xffffffffu, r.c, 1);
+        r.e = __shfl_down_sync(0xffffffffu, r.c, 1);
+        if (lane == 0) r.w = __ldg(row + xw);
+        if (lane == 31) r.e = __ldg(row + xe);
+        if (xr == 0) r.w = r.c;                       // clamp at the west edge
+        if (xr >= W - 1) r.e = r.c;                   // clamp at the east edge
+        return r;
+    };
+    // diffusion coefficient of the cell (row of T, north row N, south row S)
+    auto coeff = [&](const JRow &T, float Nc, float Sc) {
+        const float Jc = T.c;
+        const float dN = __fsub_rn(Nc, Jc), dS = __fsub_rn(Sc, Jc);
+        const float dW = __fsub_rn(T.w, Jc), dE = __fsub_rn(T.e, Jc);
+        const float g2n = __fadd_rn(__fadd_rn(__fadd_rn(__fmul_rn(dN, dN), __fmul_rn(dS, dS)), __fmul_rn(dW, dW)),
+                                    __fmul_rn(dE, dE));
+        const float ij = __frcp_rn(Jc);
+        const float G2 = __fmul_rn(__fmul_rn(g2n, ij), ij);
+        const float L = __fmul_rn(__fadd_rn(__fadd_rn(__fadd_rn(dN, dS), dW), dE), ij);
+        const float num = __fsub_rn(__fmul_rn(0.5f, G2), __fmul_rn(0.0625f, __fmul_rn(L, L)));
+        const float den = __fadd_rn(1.0f, __fmul_rn(0.25f, L));
+        const float qsqr = __fdiv_rn(num, __fmul_rn(den, den));
+        const float dd = __fmul_rn(__fsub_rn(qsqr, q0), iqden);
+        return fminf(fmaxf(__frcp_rn(__fadd_rn(1.0f, dd)), 0.0f), 1.0f);
+    };
+    JRow jm = load(max(ys - 1, 0)), j0 = load(ys), j1 = load(min(ys + 1, H - 1));
+    float c0 = coeff(j0, jm.c, j1.c);
+    for (int y = ys; y < ye; ++y) {
+        const JRow j2 = load(min(y + 2, H - 1));
+        const float c1 = (y + 1 <= H - 1) ? coeff(j1, j0.c, j2.c) : c0;   // c of row clamp(y+1)
+        float cE = __shfl_down_sync(0xffffffffu, c0, 1);
+        if (xr >= W - 1) cE = c0;
+        const float Jc = j0.c;
+        const float dN = __fsub_rn(jm.c, Jc), dS = __fsub_rn(j1.c, Jc);
+        const float dW = __fsub_rn(j0.w, Jc), dE = __fsub_rn(j0.e, Jc);
+        const float D = __fadd_rn(__fadd_rn(__fadd_rn(__fmul_rn(c0, dN), __fmul_rn(c1, dS)), __fmul_rn(c0, dW)),
+                                  __fmul_rn(cE, dE));
+        if (lane < 31 && xr < W)
+            Jo[((size_t)y - (size_t)a.dst_row_begin) * (size_t)W + xr] = __fadd_rn(Jc, __fmul_rn(lam4, D));
+        jm = j0;
+        j0 = j1;
+        j1 = j2;
+        c0 = c1;
+    }
+}
+
+// T = 256 threads (32 x 8 warps): 31 output columns x 8 strips of 16 rows per CTA.
+extern "C" __global__ void __launch_bounds__(256) orion_srad2_f32_256(orion_kargs a) { srad2_body<8, 16>(a); }

@@ -63,6 +63,14 @@ def test_bit_exact_across_levels_and_vs_oracle(srad):
     assert abs(outs[0].astype(np.float64).sum() - t0.astype(np.float64).sum()) < 1e-6 * t0.sum()
 
 
+def test_tile_and_sliding_kernels_identical(srad):
+    vt, _ = O.build_all_levels(0, "srad_f32_tile", mode=O.REALISE_MIN_CARVEOUT)
+    t0, _ = synth.thermal_inputs(257, 190, seed=8)
+    a, _ = run(srad[0], len(srad[0]) - 1, t0, 6)
+    b, _ = run(vt, 0, t0, 6)
+    assert np.array_equal(a, b)
+
+
 def test_roi_statistics(srad):
     t0, _ = synth.thermal_inputs(200, 150, seed=7)
     _, qs = run(srad[0], 0, t0, 1, roi=(3, 120, 10, 170))

@@ -29,7 +29,7 @@ if kernel == "srad_f32":
     O.generate_thermal(0, a.data_ptr(), p.data_ptr(), W, H, stream=sp)
     O.srad_roi_stats(0, a.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
     args = O.srad_args(a.data_ptr(), b.data_ptr(), q0.data_ptr(), W, H)
-elif kernel == "hotspot_f32":
+elif kernel in ("hotspot_f32", "hotspot2_f32"):
     a = torch.empty((H, W), device="cuda")
     b = torch.empty((H, W), device="cuda")
     p = torch.empty((H, W), device="cuda")
