@@ -38,14 +38,16 @@ def run(v, level, j0, iters, lam=0.5, roi=ROI):
     return a.cpu().numpy(), [float(q) for q in qs]
 
 
-def test_levels_verified_downward_direction(srad):
+def test_levels_verified_and_ladder_per_fig8(srad):
+    from oracle import occupancy as OC
+    from oracle import tuner as OT
     v, res = srad
     t = O.Tuner(v)
     d, ladder = t.ladder()
-    if res.regs_per_thread < 32:             # MAXLIVE < 32: Fig. 8 predicts "decreasing"
-        assert d == O.DIR_DECREASING and [v.level(i).ctas_per_sm for i in ladder] == list(range(len(v), 0, -1))
-    else:                                    # at the register maximum already: nothing above
-        assert d == O.DIR_INCREASING and [v.level(i).ctas_per_sm for i in ladder] == [len(v)]
+    ol = OC.levels(OC.B200, res.block_threads, res.regs_per_thread, res.static_smem_bytes, res.dyn_smem_bytes,
+                   mode=OC.REALISE_MIN_CARVEOUT)
+    od, oladder, _ = OT.candidates(ol, res.regs_per_thread, OT.TunerCfg())
+    assert d == od and [v.level(i).ctas_per_sm for i in ladder] == [ol[i].ctas_per_sm for i in oladder]
     for i in range(len(v)):
         assert v.info(i).verified_ctas == v.level(i).ctas_per_sm
 
