@@ -46,6 +46,25 @@ def band(rank: int, world: int, height: int, halo: int) -> Band:
     return Band(rank, world, height, per, r0, r1, max(0, r0 - halo), min(height, r1 + halo))
 
 
+def gather_rows(out_band, full_out, rows_per_rank: int, r0: int, r1: int, group=None):
+    """all_gather rows [r0, r1) of every rank's band straight into their places in
+    `full_out` (rank k's rows land at k * rows_per_rank + [r0, r1)).  Issue it on a side
+    stream right after the kernel that produced those rows, so the collective of one chunk
+    overlaps the compute of the next (kernel splitting, feeding the exchange)."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    views = [full_out[k * rows_per_rank + r0:k * rows_per_rank + r1] for k in range(world)]
+    src = out_band[r0:r1].contiguous()
+    if full_out.is_cuda and dist.get_backend(group) != "nccl":
+        host = [v.new_empty(v.shape, device="cpu") for v in views]
+        dist.all_gather(host, src.cpu(), group=group)
+        for v, h in zip(views, host):
+            v.copy_(h)
+        return full_out
+    dist.all_gather(views, src, group=group)
+    return full_out
+
+
 def gather_bands(out_band, full_out, group=None):
     """all_gather the equal-height output bands into `full_out` (world * rows_per_rank rows).
 

@@ -71,3 +71,36 @@ def test_gloo_sharded_equals_full_image(world, H, kind):
         assert p.exitcode == 0
     full, _, _ = oracle.denoise(kind, synth.noisy_rgba(W, H, seed=5, sigma=0.13))
     assert np.array_equal(got, full)
+
+
+def _chunk_worker(rank, world, port, H, W, chunks, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    b = shard.band(rank, world, H, 6)
+    out = torch.full((b.rows_per_rank, W), -1.0)
+    out[: b.rows] = torch.arange(b.row_begin, b.row_end, dtype=torch.float32)[:, None] + torch.zeros(W)
+    full = torch.zeros((world * b.rows_per_rank, W))
+    per = -(-b.rows_per_rank // chunks)
+    for c in range(chunks):
+        r0, r1 = min(b.rows_per_rank, c * per), min(b.rows_per_rank, (c + 1) * per)
+        if r0 < r1:
+            shard.gather_rows(out, full, b.rows_per_rank, r0, r1)
+    if rank == 0:
+        q.put(full[:H].numpy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,H,chunks", [(2, 37, 3), (3, 20, 4)])
+def test_chunked_gather_places_rows(world, H, chunks):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_chunk_worker, args=(r, world, port, H, 5, chunks, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=300)
+        assert p.exitcode == 0
+    assert np.array_equal(got, np.repeat(np.arange(H, dtype=np.float32)[:, None], 5, axis=1))
