@@ -501,6 +501,15 @@ def run_ours(args):
                   "worst_k": lv[worst].ctas_per_sm, "ms_worst": ms[worst], "maxocc_k": lv[kmax].ctas_per_sm,
                   "ms_maxocc": ms[kmax], "nvcc_default_k": lv[orig].ctas_per_sm, "ms_nvcc_default": ms[orig]},
         "regret": t_final / ms[best] - 1.0,
+        # the paper's Fig. 11 report (P:L747-P:L755): worst level (Orion-Min), best level
+        # (Orion-Max), the nvcc build (the original), and Orion-Select = the tuned run
+        # INCLUDING its exploration iterations, over the warm-up + timed horizon
+        "fig11": {"orion_min_ms": ms[worst], "orion_max_ms": ms[best], "nvcc_ms": ms[orig],
+                  "orion_select_ms": (sum(explore_ms) + (args.warmup + args.steps - len(explore_ms)) * ms_step)
+                  / (args.warmup + args.steps),
+                  "speedup_select_vs_nvcc": ms[orig] / ((sum(explore_ms) + (args.warmup + args.steps
+                                                          - len(explore_ms)) * ms_step) / (args.warmup + args.steps)),
+                  "speedup_max_vs_nvcc": ms[orig] / ms[best], "speedup_min_vs_nvcc": ms[orig] / ms[worst]},
         "vs_maxocc": ms[kmax] / t_final,
         "vs_nvcc_default": ms[orig] / t_final,
         "build_seconds": round(t_build, 2),
