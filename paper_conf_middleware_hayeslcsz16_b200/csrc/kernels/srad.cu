@@ -9,21 +9,85 @@
 // Clamp-to-edge neighbours.  One iteration = the ROI statistics kernel (one CTA, a
 // deterministic fixed-order double reduction) + the tunable update kernel.
 //
-// Update kernel: CTA = 32 x 8 threads, output tile 32 x 32 cells (4 rows per thread).
-// The J tile with a 1-cell halo (+1 extra row / column south / east for the neighbours'
-// coefficients) is staged in shared memory; the coefficients c of the tile plus one row
-// south and one column east are computed once into shared memory (the two-kernel
-// Rodinia form writes c and four derivative arrays to DRAM instead); then J' is formed.
-// HBM: 8 algorithmic bytes per cell-iteration (read J, write J').
+// fp32 evaluation (reading R-SRAD-FP): multiplying numerator and denominator of qsqr by
+// J^2 gives the same quantity with ONE reciprocal,
+//   qsqr = (sum d^2 / 2 - (sum d)^2 / 16) / (J + sum d / 4)^2,
+// and the two reciprocals left are MUFU.RCP (rcp.approx.ftz, <= 1 ulp) instead of IEEE
+// divisions; products feeding sums are FFMA.  The operation sequence is fixed in
+// srad_coeff / srad_update below (explicit .rn intrinsics, PTX built with -fmad=false),
+// so every kernel of this file and every occupancy variant is bit-identical; the oracle
+// (double, Rodinia's order) is matched to the tolerance the tests state.
 #include "common.cuh"
 
 namespace {
+
+ORION_DEVICE float rcp_approx(float x)
+{
+    float y;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+
+// The coefficient of a cell and the differences its own update reuses.
+struct SradCell {
+    float c;     // diffusion coefficient, in [0, 1]
+    float dnw;   // dN + dW
+    float ds, de;
+};
+
+// q0 = q0sqr; nq = -q0sqr * iqden; iqden = 1 / (q0sqr (1 + q0sqr)) (launch-uniform).
+ORION_DEVICE SradCell srad_coeff(float Jc, float N, float S, float Wv, float E, float iqden, float nq)
+{
+    const float dN = __fsub_rn(N, Jc), dS = __fsub_rn(S, Jc);
+    const float dW = __fsub_rn(Wv, Jc), dE = __fsub_rn(E, Jc);
+    const float g2 = __fmaf_rn(dE, dE, __fmaf_rn(dW, dW, __fmaf_rn(dS, dS, __fmul_rn(dN, dN))));
+    const float dnw = __fadd_rn(dN, dW);
+    const float sd = __fadd_rn(__fadd_rn(dnw, dS), dE);
+    const float num = __fmaf_rn(__fmul_rn(-0.0625f, sd), sd, __fmul_rn(0.5f, g2));
+    const float den = __fmaf_rn(0.25f, sd, Jc);
+    const float qsqr = __fmul_rn(num, rcp_approx(__fmul_rn(den, den)));
+    const float c = rcp_approx(__fadd_rn(1.0f, __fmaf_rn(qsqr, iqden, nq)));
+    SradCell r;
+    r.c = __saturatef(c);
+    r.dnw = dnw;
+    r.ds = dS;
+    r.de = dE;
+    return r;
+}
+
+// J' = J + lambda/4 * (c (dN + dW) + c_S dS + c_E dE)
+ORION_DEVICE float srad_update(float Jc, const SradCell &k, float cS, float cE, float lam4)
+{
+    return __fmaf_rn(lam4, __fmaf_rn(k.c, k.dnw, __fmaf_rn(cS, k.ds, __fmul_rn(cE, k.de))), Jc);
+}
+
+struct SradConsts {
+    float lam4, iqden, nq;
+};
+
+ORION_DEVICE SradConsts srad_consts(const orion_kargs &a)
+{
+    const float q0 = *(const float *)a.aux;
+    SradConsts k;
+    k.lam4 = __fmul_rn(0.25f, a.fparam[0]);
+    k.iqden = __frcp_rn(__fmul_rn(q0, __fadd_rn(1.0f, q0)));
+    k.nq = -__fmul_rn(q0, k.iqden);
+    return k;
+}
+
 constexpr int SX = 32, SY = 8, RY = 4;        // threads, rows per thread
 constexpr int TW = SX, TH = SY * RY;          // output tile 32 x 32
 constexpr int JW = TW + 3, JH = TH + 3;       // J tile: x0-1 .. x0+TW+1, y0-1 .. y0+TH+1
 constexpr int CW = TW + 1, CH = TH + 1;       // c tile: x0 .. x0+TW, y0 .. y0+TH
+
 }  // namespace
 
+// ---- shared-memory tile kernel (cross-check form) -----------------------------------------
+// CTA = 32 x 8 threads, output tile 32 x 32 cells (4 rows per thread).  The J tile with a
+// 1-cell halo (+1 extra row / column south / east for the neighbours' coefficients) is
+// staged in shared memory; the coefficients of the tile plus one row south and one column
+// east are computed once into shared memory (the two-kernel Rodinia form writes c and four
+// derivative arrays to DRAM instead); then J' is formed.
 extern "C" __global__ void __launch_bounds__(256) orion_srad_f32_256(orion_kargs a)
 {
     extern __shared__ float4 smem4[];
@@ -39,36 +103,21 @@ extern "C" __global__ void __launch_bounds__(256) orion_srad_f32_256(orion_kargs
         const int gx = clampi(x0 - 1 + tx, 0, W - 1), gy = clampi(y0 - 1 + ty, 0, H - 1);
         js[idx] = __ldg(J + (size_t)(gy - a.src_row_begin) * (size_t)W + gx);
     }
-    const float q0 = *(const float *)a.aux;
-    const float lam4 = __fmul_rn(0.25f, a.fparam[0]);
-    const float iqden = __frcp_rn(__fmul_rn(q0, __fadd_rn(1.0f, q0)));
+    const SradConsts k = srad_consts(a);
     __syncthreads();
     // coefficient tile: cell (y0+cy, x0+cx), cy in [0, CH), cx in [0, CW).  The cell at
     // global (gy, gx) with gy >= H or gx >= W is a clamped copy: its coefficient is the
     // edge cell's, which the clamped J values reproduce (all its neighbours clamp alike).
-    for (int idx = tid; idx < CW * CH; idx += SX * SY) {
-        const int cy = idx / CW, cx = idx - cy * CW;
-        const int gy = y0 + cy, gx = x0 + cx;
-        // tile coordinates of (gy, gx) and its clamped neighbours
+    auto tile_cell = [&](int gy, int gx) {
         const int ty = min(gy, H - 1) - (y0 - 1), tx = min(gx, W - 1) - (x0 - 1);
         const int tn = max(min(gy, H - 1) - 1, 0) - (y0 - 1), ts = min(min(gy, H - 1) + 1, H - 1) - (y0 - 1);
         const int tw = max(min(gx, W - 1) - 1, 0) - (x0 - 1), te = min(min(gx, W - 1) + 1, W - 1) - (x0 - 1);
-        const float Jc = js[ty * JW + tx];
-        const float dN = __fsub_rn(js[tn * JW + tx], Jc), dS = __fsub_rn(js[ts * JW + tx], Jc);
-        const float dW = __fsub_rn(js[ty * JW + tw], Jc), dE = __fsub_rn(js[ty * JW + te], Jc);
-        const float g2n = __fadd_rn(__fadd_rn(__fadd_rn(__fmul_rn(dN, dN), __fmul_rn(dS, dS)), __fmul_rn(dW, dW)),
-                                    __fmul_rn(dE, dE));
-        // one IEEE reciprocal of J serves G2 = sum d^2 / J^2 and L = sum d / J; the
-        // (qsqr - q0sqr) / (q0sqr (1 + q0sqr)) division uses the launch-uniform reciprocal
-        const float ij = __frcp_rn(Jc);
-        const float G2 = __fmul_rn(__fmul_rn(g2n, ij), ij);
-        const float L = __fmul_rn(__fadd_rn(__fadd_rn(__fadd_rn(dN, dS), dW), dE), ij);
-        const float num = __fsub_rn(__fmul_rn(0.5f, G2), __fmul_rn(0.0625f, __fmul_rn(L, L)));
-        const float den = __fadd_rn(1.0f, __fmul_rn(0.25f, L));
-        const float qsqr = __fdiv_rn(num, __fmul_rn(den, den));
-        const float dd = __fmul_rn(__fsub_rn(qsqr, q0), iqden);
-        const float c = __frcp_rn(__fadd_rn(1.0f, dd));
-        cs[idx] = fminf(fmaxf(c, 0.0f), 1.0f);
+        return srad_coeff(js[ty * JW + tx], js[tn * JW + tx], js[ts * JW + tx], js[ty * JW + tw], js[ty * JW + te],
+                          k.iqden, k.nq);
+    };
+    for (int idx = tid; idx < CW * CH; idx += SX * SY) {
+        const int cy = idx / CW, cx = idx - cy * CW;
+        cs[idx] = tile_cell(y0 + cy, x0 + cx).c;
     }
     __syncthreads();
     const int cx = threadIdx.x, gx = x0 + cx;
@@ -77,133 +126,176 @@ extern "C" __global__ void __launch_bounds__(256) orion_srad_f32_256(orion_kargs
     for (int r = 0; r < RY; ++r) {
         const int cy = threadIdx.y * RY + r, gy = y0 + cy;
         if (gy >= a.row_end) return;
-        const int ty = gy - (y0 - 1), tx = gx - (x0 - 1);
-        const int tn = max(gy - 1, 0) - (y0 - 1), ts = min(gy + 1, H - 1) - (y0 - 1);
-        const int tw = max(gx - 1, 0) - (x0 - 1), te = min(gx + 1, W - 1) - (x0 - 1);
-        const float Jc = js[ty * JW + tx];
-        const float dN = __fsub_rn(js[tn * JW + tx], Jc), dS = __fsub_rn(js[ts * JW + tx], Jc);
-        const float dW = __fsub_rn(js[ty * JW + tw], Jc), dE = __fsub_rn(js[ty * JW + te], Jc);
-        const float cC = cs[cy * CW + cx];
+        const SradCell kc = tile_cell(gy, gx);
+        const float Jc = js[(gy - (y0 - 1)) * JW + (gx - (x0 - 1))];
         const float cS = cs[(min(gy + 1, H - 1) - y0) * CW + cx];
         const float cE = cs[cy * CW + (min(gx + 1, W - 1) - x0)];
-        const float D = __fadd_rn(__fadd_rn(__fadd_rn(__fmul_rn(cC, dN), __fmul_rn(cS, dS)), __fmul_rn(cC, dW)),
-                                  __fmul_rn(cE, dE));
-        ((float *)a.dst)[(size_t)(gy - a.dst_row_begin) * (size_t)W + gx] = __fadd_rn(Jc, __fmul_rn(lam4, D));
+        ((float *)a.dst)[(size_t)(gy - a.dst_row_begin) * (size_t)W + gx] = srad_update(Jc, kc, cS, cE, k.lam4);
     }
 }
 
 // ROI statistics: one CTA of 1024 threads; thread t sums elements t, t+1024, ... of the
-// row-major ROI in double, then a fixed-shape tree in shared memory -- deterministic, so
-// every occupancy variant of the update kernel sees the same q0sqr.
+// row-major ROI in double (4 loads in flight), then a fixed-shape shuffle tree per warp and
+// across the 32 warp sums -- deterministic, so every occupancy variant of the update kernel
+// sees the same q0sqr.
 extern "C" __global__ void __launch_bounds__(1024) orion_srad_stats(const float *J, int W, int r1, int r2, int c1,
                                                                      int c2, float *q0)
 {
-    __shared__ double s1[1024], s2[1024];
+    __shared__ double s1[32], s2[32];
     const int t = threadIdx.x;
     const int rw = c2 - c1 + 1, n = (r2 - r1 + 1) * rw;
     double a = 0.0, b = 0.0;
+#pragma unroll 4
     for (int e = t; e < n; e += 1024) {
         const int i = r1 + e / rw, j = c1 + e % rw;
-        const double v = J[(size_t)i * (size_t)W + j];
+        const double v = __ldg(J + (size_t)i * (size_t)W + j);
         a += v;
         b += v * v;
     }
-    s1[t] = a;
-    s2[t] = b;
-    __syncthreads();
-    for (int s = 512; s > 0; s >>= 1) {
-        if (t < s) {
-            s1[t] += s1[t + s];
-            s2[t] += s2[t + s];
-        }
-        __syncthreads();
+#pragma unroll
+    for (int s = 16; s > 0; s >>= 1) {
+        a += __shfl_down_sync(0xffffffffu, a, s);
+        b += __shfl_down_sync(0xffffffffu, b, s);
     }
-    if (t == 0) {
-        const double mean = s1[0] / n;
-        const double var = s2[0] / n - mean * mean;
-        *q0 = (float)(var / (mean * mean));
+    if ((t & 31) == 0) {
+        s1[t >> 5] = a;
+        s2[t >> 5] = b;
+    }
+    __syncthreads();
+    if (t < 32) {
+        a = s1[t];
+        b = s2[t];
+#pragma unroll
+        for (int s = 16; s > 0; s >>= 1) {
+            a += __shfl_down_sync(0xffffffffu, a, s);
+            b += __shfl_down_sync(0xffffffffu, b, s);
+        }
+        if (t == 0) {
+            const double mean = a / n;
+            const double var = b / n - mean * mean;
+            *q0 = (float)(var / (mean * mean));
+        }
     }
 }
 
-// ---- register-sliding variant ------------------------------------------------------------
-// Same arithmetic, no shared memory: lane l of a warp owns column x0 + l (x0 = 31 * block
-// column; lanes 0..30 write, lane 31 only supplies the coefficient its west neighbour needs
-// as c_E) and walks a strip of RY rows keeping J rows y-1 .. y+2 and the coefficients of rows
-// y, y+1 in registers.  E / W neighbours come by shuffle; lanes 0 / 31 load the column just
-// outside the warp.  One coefficient per cell, one coalesced 128-byte row load per step.
+// ---- register-sliding kernel (the default srad_f32) ------------------------------------------
+// A warp owns 32*V consecutive columns from x0 (V = 4: float4 lanes, 16-byte loads / stores,
+// width % 4 == 0; V = 1: scalar lanes for any width), of which lanes 0..30 write their cells
+// and lane 31 only supplies the coefficient lane 30's last cell needs as c_E (31V output
+// columns per warp: 3 % of the arithmetic instead of a divergent extra cell).  It walks a strip
+// of rows top to bottom with J rows y .. y+2 and the coefficient row y in registers, the next
+// two rows in flight: every J row is read once per strip, every coefficient computed once.
+// W / E neighbours come by shuffle; lane 0 fetches column x0-1, lane 31 column x0+32V.
+// CTA = 8 warps over a 124 x 128 tile: V = 4 -> 8 strips of 16 rows; V = 1 -> 4 column
+// groups of 31 x 2 strips of 64 rows.
 namespace {
-struct JRow {
-    float c, w, e;   // J at the lane's column and at its west / east neighbours
+template <int V>
+struct SRow {
+    float v[V];
+    float xa;   // lane 0: J[max(x0-1, 0)]; lane 31: J[min(x0+32V, W-1)]; others: unused
+};
+template <int V>
+struct CRow {
+    SradCell k[V];
 };
 }  // namespace
 
-template <int BY, int RY>
-__device__ __forceinline__ void srad2_body(const orion_kargs &a)
+template <int V>
+__device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys, int ye)
 {
-    const float *J = (const float *)a.src;
-    float *Jo = (float *)a.dst;
     const int W = a.width, H = a.height;
     const int lane = threadIdx.x;
-    const int x0 = blockIdx.x * 31;
-    const int xr = x0 + lane;
-    const int x = min(xr, W - 1);
-    const int ys = a.row_begin + (blockIdx.y * BY + threadIdx.y) * RY;
-    if (ys >= a.row_end) return;
-    const int ye = min(ys + RY, a.row_end);
-    const size_t sb = (size_t)a.src_row_begin;
-    const float q0 = *(const float *)a.aux;
-    const float lam4 = __fmul_rn(0.25f, a.fparam[0]);
-    const float iqden = __frcp_rn(__fmul_rn(q0, __fadd_rn(1.0f, q0)));
-    const int xw = clampi(x0 - 1, 0, W - 1), xe = clampi(x0 + 32, 0, W - 1);
+    const int cx = x0 + V * lane;
+    const int cxl = min(cx, W - V);
+    const bool east_clamp = cx + V >= W;      // the lane's last cell is the image's last column
+    const bool writer = lane < 31 && cx < W;
+    const SradConsts kc = srad_consts(a);
+    const int xa = lane == 0 ? max(x0 - 1, 0) : (lane == 31 ? min(x0 + 32 * V, W - 1) : cxl);
+    const float *J = (const float *)a.src - (size_t)a.src_row_begin * (size_t)W;   // global row 0
+    float *Jo = (float *)a.dst + (size_t)cx - (size_t)a.dst_row_begin * (size_t)W;
 
-    auto load = [&](int y) {
-        const float *row = J + ((size_t)y - sb) * (size_t)W;
-        JRow r;
-        r.c = __ldg(row + x);
-        r.w = __shfl_up_sync(0xffffffffu, r.c, 1);
-        r.e = __shfl_down_sync(0xffffffffu, r.c, 1);
-        if (lane == 0) r.w = __ldg(row + xw);
-        if (lane == 31) r.e = __ldg(row + xe);
-        if (xr == 0) r.w = r.c;                       // clamp at the west edge
-        if (xr >= W - 1) r.e = r.c;                   // clamp at the east edge
+    auto load = [&](const float *row) {
+        SRow<V> r;
+        if constexpr (V == 4) {
+            const float4 q = __ldg(reinterpret_cast<const float4 *>(row + cxl));
+            r.v[0] = q.x;
+            r.v[1] = q.y;
+            r.v[2] = q.z;
+            r.v[3] = q.w;
+        } else {
+            r.v[0] = __ldg(row + cxl);
+        }
+        r.xa = __ldg(row + xa);
         return r;
     };
-    // diffusion coefficient of the cell (row of T, north row N, south row S)
-    auto coeff = [&](const JRow &T, float Nc, float Sc) {
-        const float Jc = T.c;
-        const float dN = __fsub_rn(Nc, Jc), dS = __fsub_rn(Sc, Jc);
-        const float dW = __fsub_rn(T.w, Jc), dE = __fsub_rn(T.e, Jc);
-        const float g2n = __fadd_rn(__fadd_rn(__fadd_rn(__fmul_rn(dN, dN), __fmul_rn(dS, dS)), __fmul_rn(dW, dW)),
-                                    __fmul_rn(dE, dE));
-        const float ij = __frcp_rn(Jc);
-        const float G2 = __fmul_rn(__fmul_rn(g2n, ij), ij);
-        const float L = __fmul_rn(__fadd_rn(__fadd_rn(__fadd_rn(dN, dS), dW), dE), ij);
-        const float num = __fsub_rn(__fmul_rn(0.5f, G2), __fmul_rn(0.0625f, __fmul_rn(L, L)));
-        const float den = __fadd_rn(1.0f, __fmul_rn(0.25f, L));
-        const float qsqr = __fdiv_rn(num, __fmul_rn(den, den));
-        const float dd = __fmul_rn(__fsub_rn(qsqr, q0), iqden);
-        return fminf(fmaxf(__frcp_rn(__fadd_rn(1.0f, dd)), 0.0f), 1.0f);
+    auto coeff_row = [&](const SRow<V> &N, const SRow<V> &T, const SRow<V> &S) {
+        float Wv = __shfl_up_sync(0xffffffffu, T.v[V - 1], 1);
+        float Ev = __shfl_down_sync(0xffffffffu, T.v[0], 1);
+        if (lane == 0) Wv = T.xa;
+        if (lane == 31) Ev = T.xa;
+        if (east_clamp) Ev = T.v[V - 1];
+        CRow<V> c;
+#pragma unroll
+        for (int k = 0; k < V; ++k)
+            c.k[k] = srad_coeff(T.v[k], N.v[k], S.v[k], k == 0 ? Wv : T.v[k - 1], k == V - 1 ? Ev : T.v[k + 1],
+                                kc.iqden, kc.nq);
+        return c;
     };
-    JRow jm = load(max(ys - 1, 0)), j0 = load(ys), j1 = load(min(ys + 1, H - 1));
-    float c0 = coeff(j0, jm.c, j1.c);
-    for (int y = ys; y < ye; ++y) {
-        const JRow j2 = load(min(y + 2, H - 1));
-        const float c1 = (y + 1 <= H - 1) ? coeff(j1, j0.c, j2.c) : c0;   // c of row clamp(y+1)
-        float cE = __shfl_down_sync(0xffffffffu, c0, 1);
-        if (xr >= W - 1) cE = c0;
-        const float Jc = j0.c;
-        const float dN = __fsub_rn(jm.c, Jc), dS = __fsub_rn(j1.c, Jc);
-        const float dW = __fsub_rn(j0.w, Jc), dE = __fsub_rn(j0.e, Jc);
-        const float D = __fadd_rn(__fadd_rn(__fadd_rn(__fmul_rn(c0, dN), __fmul_rn(c1, dS)), __fmul_rn(c0, dW)),
-                                  __fmul_rn(cE, dE));
-        if (lane < 31 && xr < W)
-            Jo[((size_t)y - (size_t)a.dst_row_begin) * (size_t)W + xr] = __fadd_rn(Jc, __fmul_rn(lam4, D));
-        jm = j0;
+    auto update_row = [&](int y, const SRow<V> &T, const CRow<V> &c0, const CRow<V> &c1) {
+        float cE = __shfl_down_sync(0xffffffffu, c0.k[0].c, 1);
+        if (east_clamp) cE = c0.k[V - 1].c;
+        float o[V];
+#pragma unroll
+        for (int k = 0; k < V; ++k)
+            o[k] = srad_update(T.v[k], c0.k[k], c1.k[k].c, k == V - 1 ? cE : c0.k[k + 1].c, kc.lam4);
+        if (writer) {
+            float *orow = Jo + (size_t)y * (size_t)W;
+            if constexpr (V == 4)
+                *reinterpret_cast<float4 *>(orow) = make_float4(o[0], o[1], o[2], o[3]);
+            else
+                *orow = o[0];
+        }
+    };
+
+    // rows are fetched through a pointer that stops at the last image row (clamp to edge)
+    int rn = ys + 3;                                            // next row to fetch
+    const float *pn = J + (size_t)min(rn, H - 1) * (size_t)W;
+    auto fetch = [&]() {
+        const SRow<V> r = load(pn);
+        if (rn < H - 1) pn += W;
+        ++rn;
+        return r;
+    };
+    SRow<V> j0 = load(J + (size_t)ys * (size_t)W);
+    SRow<V> j1 = load(J + (size_t)min(ys + 1, H - 1) * (size_t)W);
+    SRow<V> j2 = load(J + (size_t)min(ys + 2, H - 1) * (size_t)W);
+    SRow<V> j3 = fetch();
+    CRow<V> c0 = coeff_row(load(J + (size_t)max(ys - 1, 0) * (size_t)W), j0, j1);
+    const int yb = min(ye, H - 1);                              // rows with a distinct south row
+#pragma unroll 4
+    for (int y = ys; y < yb; ++y) {
+        const SRow<V> j4 = fetch();                             // two rows in flight
+        const CRow<V> c1 = coeff_row(j0, j1, j2);               // c of row y+1
+        update_row(y, j0, c0, c1);
         j0 = j1;
         j1 = j2;
+        j2 = j3;
+        j3 = j4;
         c0 = c1;
     }
+    if (ye == H) update_row(H - 1, j0, c0, c0);               // last image row: c_S = own c
 }
 
-// T = 256 threads (32 x 8 warps): 31 output columns x 8 strips of 16 rows per CTA.
-extern "C" __global__ void __launch_bounds__(256) orion_srad2_f32_256(orion_kargs a) { srad2_body<8, 16>(a); }
+// T = 256 threads (32 x 8 warps), output tile 124 x 128.
+extern "C" __global__ void __launch_bounds__(256) orion_srad4_f32_256(orion_kargs a)
+{
+    const int w = threadIdx.y;
+    if ((a.width & 3) == 0) {
+        const int ys = a.row_begin + blockIdx.y * 128 + w * 16;
+        if (ys < a.row_end) srad_strip<4>(a, blockIdx.x * 124, ys, min(ys + 16, a.row_end));
+    } else {
+        const int x0 = blockIdx.x * 124 + (w & 3) * 31;
+        const int ys = a.row_begin + blockIdx.y * 128 + (w >> 2) * 64;
+        if (ys < a.row_end && x0 < a.width) srad_strip<1>(a, x0, ys, min(ys + 64, a.row_end));
+    }
+}

@@ -71,8 +71,8 @@ static const KernelDef kKernels[] = {
     {"hotspot2_f32", 256, "orion_hotspot2_f32_256", "hotspot", 32, 8, 128, 128, 2, K_STENCIL, 0, 0, 4, 2},
     // srad: J tile (32+3)^2 + coefficient tile (32+1)^2 floats; reads 2 rows below the tile
     {"srad_f32_tile", 256, "orion_srad_f32_256", "srad", 32, 8, 32, 32, 2, K_SRAD, 0, (35 * 35 + 33 * 33) * 4},
-    // srad, register-sliding: warp = 31 output columns + 1 coefficient-only lane, 16-row strips
-    {"srad_f32", 256, "orion_srad2_f32_256", "srad", 32, 8, 31, 128, 2, K_SRAD, 0, 0},
+    // srad, register-sliding: 124 x 128 tile; float4 lanes (width % 4 == 0) or scalar lanes
+    {"srad_f32", 256, "orion_srad4_f32_256", "srad", 32, 8, 124, 128, 2, K_SRAD, 0, 0},
 };
 
 const KernelDef *find_kernel(const char *id, int threads)
