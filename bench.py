@@ -662,7 +662,8 @@ def main():
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
     ap.add_argument("--kernel", default="", help="override the workload's kernel id (same family)")
     ap.add_argument("--c5-chunks", type=int, default=4, help="C5: row chunks per band whose all-gathers overlap compute")
-    ap.add_argument("--samples", type=int, default=1, help="timed launches per explored level (paper: 1)")
+    ap.add_argument("--samples", type=int, default=2,
+                    help="timed launches per explored level, the fastest kept (paper: 1; reading R-A11)")
     ap.add_argument("--select", choices=["fastest", "lowest"], default="fastest",
                     help="final-kernel rule: fastest measured, or lowest occupancy within 2%% (resource saving)")
     ap.add_argument("--realise", choices=["max", "min"], default="min",

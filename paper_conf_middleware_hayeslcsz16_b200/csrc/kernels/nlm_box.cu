@@ -88,18 +88,18 @@ ORION_DEVICE float2 diff2x2(float2 ar, float2 ag, float2 ab, float br, float bg,
 // Phase A for G offsets (i, j1 .. j1+G-1): lane = row r, warp's 32 H columns.  Offsets
 // g = 0, 1 run packed (fp32x2), offset g = 2 scalar.
 template <int G>
-ORION_DEVICE void phase_a(const float *pr, const float *pg, const float *pb, float *hs, int lane, int warp, int i,
+ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lane, int warp, int i,
                           int j1)
 {
     const int cb = 3 + 32 * warp;               // tile column of u for the first difference
     const int rowc = lane * PW + cb;            // centre p(u, v)
     const int rows = rowc + i * PW + j1;        // shifted p(u+j1, v+i)
     // the shifted window holds columns q + j1 .. q + j1 + G - 1 at step q
-    float wr[G], wg[G], wb[G];
+    float2 wrg[G];
+    float wb[G];
 #pragma unroll
     for (int g = 0; g < G - 1; ++g) {
-        wr[g + 1] = pr[rows + g];
-        wg[g + 1] = pg[rows + g];
+        wrg[g + 1] = prg[rows + g];
         wb[g + 1] = pb[rows + g];
     }
     constexpr int GP = G / 2;                   // packed offset pairs (0 or 1)
@@ -110,18 +110,18 @@ ORION_DEVICE void phase_a(const float *pr, const float *pg, const float *pb, flo
     for (int q = 0; q < 38; ++q) {
 #pragma unroll
         for (int g = 0; g < G - 1; ++g) {
-            wr[g] = wr[g + 1];
-            wg[g] = wg[g + 1];
+            wrg[g] = wrg[g + 1];
             wb[g] = wb[g + 1];
         }
-        wr[G - 1] = pr[rows + q + G - 1];
-        wg[G - 1] = pg[rows + q + G - 1];
+        wrg[G - 1] = prg[rows + q + G - 1];
         wb[G - 1] = pb[rows + q + G - 1];
-        const float cr = pr[rowc + q], cg = pg[rowc + q], cbv = pb[rowc + q];
+        const float2 crg = prg[rowc + q];
+        const float cr = crg.x, cg = crg.y, cbv = pb[rowc + q];
         if (GP > 0)
-            dp[GP > 0 ? q : 0] = diff2x2(make_float2(wr[0], wr[GP > 0 ? 1 : 0]), make_float2(wg[0], wg[GP > 0 ? 1 : 0]),
+            dp[GP > 0 ? q : 0] = diff2x2(make_float2(wrg[0].x, wrg[GP > 0 ? 1 : 0].x),
+                                         make_float2(wrg[0].y, wrg[GP > 0 ? 1 : 0].y),
                                          make_float2(wb[0], wb[GP > 0 ? 1 : 0]), cr, cg, cbv);
-        if (GS > 0) ds[GS > 0 ? q : 0] = diff2(wr[G - 1], wg[G - 1], wb[G - 1], cr, cg, cbv);
+        if (GS > 0) ds[GS > 0 ? q : 0] = diff2(wrg[G - 1].x, wrg[G - 1].y, wb[G - 1], cr, cg, cbv);
     }
     if (GP > 0) {
         float2 h[32];
@@ -152,7 +152,7 @@ struct Acc {
 // Phase B for one pair (i, j) whose H_o lives in hb: thread t = output column x0+t.  The
 // +o and -o vertical windows run packed (fp32x2), as do their exponent arguments and the
 // (r, g) / (b, weight) accumulations.
-ORION_DEVICE void phase_b(const float *pr, const float *pg, const float *pb, const float *hb, int t, int i, int j,
+ORION_DEVICE void phase_b(const float2 *prg, const float *pb, const float *hb, int t, int i, int j,
                           float nl2, float wthr, Acc &A)
 {
     const float geo = geo_l2_rt(i, j);
@@ -169,9 +169,9 @@ ORION_DEVICE void phase_b(const float *pr, const float *pg, const float *pb, con
         const float wp = ex2(e.x), wm = ex2(e.y);
         const int pp = (r + 6 + i) * PW + t + 9 + j;      // p(x+j, y+i)
         const int pm = (r + 6 - i) * PW + t + 9 - j;      // p(x-j, y-i)
-        A.axy[r] = fma2(make_float2(wp, wp), make_float2(pr[pp], pg[pp]), A.axy[r]);
+        A.axy[r] = fma2(make_float2(wp, wp), prg[pp], A.axy[r]);
         A.azs[r] = fma2(make_float2(wp, wp), make_float2(pb[pp], 1.0f), A.azs[r]);
-        A.axy[r] = fma2(make_float2(wm, wm), make_float2(pr[pm], pg[pm]), A.axy[r]);
+        A.axy[r] = fma2(make_float2(wm, wm), prg[pm], A.axy[r]);
         A.azs[r] = fma2(make_float2(wm, wm), make_float2(pb[pm], 1.0f), A.azs[r]);
         A.cnt[r >> 2] += (((wp > wthr) ? 1u : 0u) + ((wm > wthr) ? 1u : 0u)) << (8 * (r & 3));
     }
@@ -217,17 +217,17 @@ ORION_DEVICE void window7_i(const unsigned (&h)[N + 6], unsigned (&out)[N])
 }
 
 template <int G>
-ORION_DEVICE void phase_a_int(const float *pr, const float *pg, const float *pb, unsigned *hs, int lane, int warp,
+ORION_DEVICE void phase_a_int(const float2 *prg, const float *pb, unsigned *hs, int lane, int warp,
                               int i, int j1)
 {
     const int cb = 3 + 32 * warp;
     const int rowc = lane * PW + cb;
     const int rows = rowc + i * PW + j1;
-    float wr[G], wg[G], wb[G];
+    float2 wrg[G];
+    float wb[G];
 #pragma unroll
     for (int g = 0; g < G - 1; ++g) {
-        wr[g + 1] = pr[rows + g];
-        wg[g + 1] = pg[rows + g];
+        wrg[g + 1] = prg[rows + g];
         wb[g + 1] = pb[rows + g];
     }
     unsigned q[G][38];
@@ -235,16 +235,15 @@ ORION_DEVICE void phase_a_int(const float *pr, const float *pg, const float *pb,
     for (int c = 0; c < 38; ++c) {
 #pragma unroll
         for (int g = 0; g < G - 1; ++g) {
-            wr[g] = wr[g + 1];
-            wg[g] = wg[g + 1];
+            wrg[g] = wrg[g + 1];
             wb[g] = wb[g + 1];
         }
-        wr[G - 1] = pr[rows + c + G - 1];
-        wg[G - 1] = pg[rows + c + G - 1];
+        wrg[G - 1] = prg[rows + c + G - 1];
         wb[G - 1] = pb[rows + c + G - 1];
-        const float cr = pr[rowc + c], cg = pg[rowc + c], cbv = pb[rowc + c];
+        const float2 crg = prg[rowc + c];
+        const float cr = crg.x, cg = crg.y, cbv = pb[rowc + c];
 #pragma unroll
-        for (int g = 0; g < G; ++g) q[g][c] = quant(diff2(wr[g], wg[g], wb[g], cr, cg, cbv));
+        for (int g = 0; g < G; ++g) q[g][c] = quant(diff2(wrg[g].x, wrg[g].y, wb[g], cr, cg, cbv));
     }
 #pragma unroll
     for (int g = 0; g < G; ++g) {
@@ -256,7 +255,7 @@ ORION_DEVICE void phase_a_int(const float *pr, const float *pg, const float *pb,
     }
 }
 
-ORION_DEVICE void phase_b_int(const float *pr, const float *pg, const float *pb, const unsigned *hb, int t, int i,
+ORION_DEVICE void phase_b_int(const float2 *prg, const float *pb, const unsigned *hb, int t, int i,
                               int j, float nl2q, float wthr, Acc &A)
 {
     const float geo = geo_l2_rt(i, j);
@@ -274,9 +273,9 @@ ORION_DEVICE void phase_b_int(const float *pr, const float *pg, const float *pb,
         const float wm = ex2(__fmaf_rn(__uint2float_rn(Dm[r]), nl2q, geo));
         const int pp = (r + 6 + i) * PW + t + 9 + j;      // p(x+j, y+i)
         const int pm = (r + 6 - i) * PW + t + 9 - j;      // p(x-j, y-i)
-        A.axy[r] = fma2(make_float2(wp, wp), make_float2(pr[pp], pg[pp]), A.axy[r]);
+        A.axy[r] = fma2(make_float2(wp, wp), prg[pp], A.axy[r]);
         A.azs[r] = fma2(make_float2(wp, wp), make_float2(pb[pp], 1.0f), A.azs[r]);
-        A.axy[r] = fma2(make_float2(wm, wm), make_float2(pr[pm], pg[pm]), A.axy[r]);
+        A.axy[r] = fma2(make_float2(wm, wm), prg[pm], A.axy[r]);
         A.azs[r] = fma2(make_float2(wm, wm), make_float2(pb[pm], 1.0f), A.azs[r]);
         A.cnt[r >> 2] += (((wp > wthr) ? 1u : 0u) + ((wm > wthr) ? 1u : 0u)) << (8 * (r & 3));
     }
@@ -295,9 +294,8 @@ template <int GMAX, bool INT>
 __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 {
     extern __shared__ float4 smem4[];
-    float *pr = reinterpret_cast<float *>(smem4);
-    float *pg = pr + PR * PW;
-    float *pb = pg + PR * PW;
+    float2 *prg = reinterpret_cast<float2 *>(smem4);             // (r, g) plane
+    float *pb = reinterpret_cast<float *>(prg + PR * PW);         // b plane
     float *hs = pb + PR * PW;               // GMAX buffers of H_o: AR rows x HP
 
     const int tid = threadIdx.x;
@@ -311,8 +309,7 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
             const int gx = clampi(x0 - 9 + tx, 0, a.width - 1);
             const int gy = clampi(y0 - 6 + ty, 0, a.height - 1);
             const float4 v = __ldg(src + (size_t)(gy - a.src_row_begin) * (size_t)a.width + gx);
-            pr[ty * PW + tx] = v.x;
-            pg[ty * PW + tx] = v.y;
+            prg[ty * PW + tx] = make_float2(v.x, v.y);
             pb[ty * PW + tx] = v.z;
         }
     }
@@ -327,7 +324,7 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 #pragma unroll
         for (int r = 0; r < TH; ++r) {
             const int pc = (r + 6) * PW + t + 9;
-            A.axy[r] = make_float2(pr[pc], pg[pc]);
+            A.axy[r] = prg[pc];
             A.azs[r] = make_float2(pb[pc], 1.0f);
         }
 #pragma unroll
@@ -343,27 +340,27 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
         unsigned *hi = reinterpret_cast<unsigned *>(hs);
         if (INT) {
             if (GMAX == 1 || G == 1)
-                phase_a_int<1>(pr, pg, pb, hi, lane, warp, i, j1);
+                phase_a_int<1>(prg, pb, hi, lane, warp, i, j1);
             else if (G == 2)
-                phase_a_int<2>(pr, pg, pb, hi, lane, warp, i, j1);
+                phase_a_int<2>(prg, pb, hi, lane, warp, i, j1);
             else
-                phase_a_int<(GMAX >= 3 ? 3 : 1)>(pr, pg, pb, hi, lane, warp, i, j1);
+                phase_a_int<(GMAX >= 3 ? 3 : 1)>(prg, pb, hi, lane, warp, i, j1);
         } else {
             if (GMAX == 1 || G == 1)
-                phase_a<1>(pr, pg, pb, hs, lane, warp, i, j1);
+                phase_a<1>(prg, pb, hs, lane, warp, i, j1);
             else if (G == 2)
-                phase_a<2>(pr, pg, pb, hs, lane, warp, i, j1);
+                phase_a<2>(prg, pb, hs, lane, warp, i, j1);
             else
-                phase_a<(GMAX >= 3 ? 3 : 1)>(pr, pg, pb, hs, lane, warp, i, j1);
+                phase_a<(GMAX >= 3 ? 3 : 1)>(prg, pb, hs, lane, warp, i, j1);
         }
         __syncthreads();
         if (t < TW) {
 #pragma unroll 1
             for (int g = 0; g < G; ++g) {
                 if (INT)
-                    phase_b_int(pr, pg, pb, hi + g * HBUF, t, i, j1 + g, nl2 * (1.0f / kQScale), wthr, A);
+                    phase_b_int(prg, pb, hi + g * HBUF, t, i, j1 + g, nl2 * (1.0f / kQScale), wthr, A);
                 else
-                    phase_b(pr, pg, pb, hs + g * HBUF, t, i, j1 + g, nl2, wthr, A);
+                    phase_b(prg, pb, hs + g * HBUF, t, i, j1 + g, nl2, wthr, A);
             }
         }
         __syncthreads();
@@ -376,7 +373,7 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
         const int y = y0 + r;
         if (y >= a.row_end) break;
         const int pc = (r + 6) * PW + t + 9;
-        const float4 c00 = make_float4(pr[pc], pg[pc], pb[pc], 0.0f);
+        const float4 c00 = make_float4(prg[pc].x, prg[pc].y, pb[pc], 0.0f);
         const int c = (int)((A.cnt[r >> 2] >> (8 * (r & 3))) & 0xffu);
         dst[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = lerp_out(c00, A.axy[r].x, A.axy[r].y, A.azs[r].x, A.azs[r].y, c, a);
     }
