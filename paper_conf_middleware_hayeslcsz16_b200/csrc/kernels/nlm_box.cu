@@ -78,6 +78,17 @@ ORION_DEVICE float diff2(float ar, float ag, float ab, float br, float bg, float
     return __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));
 }
 
+// |a - c|^2 with the (r, g) channels packed: a.rg + (-c.rg) on FADD2, squares on FMUL2, then
+// (dr^2 + dg^2) + db^2.  A sum of non-negative terms, 3 roundings deep.
+ORION_DEVICE float2 neg2(float2 a) { return make_float2(-a.x, -a.y); }
+ORION_DEVICE float diff2rg(float2 arg, float ab, float2 ncrg, float cb)
+{
+    const float2 d = __fadd2_rn(arg, ncrg);
+    const float2 q = __fmul2_rn(d, d);
+    const float db = __fsub_rn(ab, cb);
+    return __fmaf_rn(db, db, __fadd_rn(q.x, q.y));
+}
+
 ORION_DEVICE float2 diff2x2(float2 ar, float2 ag, float2 ab, float br, float bg, float bb)
 {
     const float2 dx = sub2(ar, make_float2(br, br)), dy = sub2(ag, make_float2(bg, bg)),
@@ -115,13 +126,11 @@ ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lan
         }
         wrg[G - 1] = prg[rows + q + G - 1];
         wb[G - 1] = pb[rows + q + G - 1];
-        const float2 crg = prg[rowc + q];
-        const float cr = crg.x, cg = crg.y, cbv = pb[rowc + q];
+        const float2 ncrg = neg2(prg[rowc + q]);
+        const float cbv = pb[rowc + q];
         if (GP > 0)
-            dp[GP > 0 ? q : 0] = diff2x2(make_float2(wrg[0].x, wrg[GP > 0 ? 1 : 0].x),
-                                         make_float2(wrg[0].y, wrg[GP > 0 ? 1 : 0].y),
-                                         make_float2(wb[0], wb[GP > 0 ? 1 : 0]), cr, cg, cbv);
-        if (GS > 0) ds[GS > 0 ? q : 0] = diff2(wrg[G - 1].x, wrg[G - 1].y, wb[G - 1], cr, cg, cbv);
+            dp[GP > 0 ? q : 0] = make_float2(diff2rg(wrg[0], wb[0], ncrg, cbv), diff2rg(wrg[GP > 0 ? 1 : 0], wb[GP > 0 ? 1 : 0], ncrg, cbv));
+        if (GS > 0) ds[GS > 0 ? q : 0] = diff2rg(wrg[G - 1], wb[G - 1], ncrg, cbv);
     }
     if (GP > 0) {
         float2 h[32];
@@ -149,6 +158,12 @@ struct Acc {
     unsigned cnt[(TH + 3) / 4];   // 4 x 8-bit counts per word (<= 49)
 };
 
+// [w > wthr] into row r's 8-bit count: FSETP + one predicated IADD of an immediate.
+ORION_DEVICE void count_above(Acc &A, int r, float w, float wthr)
+{
+    if (w > wthr) A.cnt[r >> 2] += 1u << (8 * (r & 3));
+}
+
 // Phase B for one pair (i, j) whose H_o lives in hb: thread t = output column x0+t.  The
 // +o and -o vertical windows run packed (fp32x2), as do their exponent arguments and the
 // (r, g) / (b, weight) accumulations.
@@ -173,7 +188,8 @@ ORION_DEVICE void phase_b(const float2 *prg, const float *pb, const float *hb, i
         A.azs[r] = fma2(make_float2(wp, wp), make_float2(pb[pp], 1.0f), A.azs[r]);
         A.axy[r] = fma2(make_float2(wm, wm), prg[pm], A.axy[r]);
         A.azs[r] = fma2(make_float2(wm, wm), make_float2(pb[pm], 1.0f), A.azs[r]);
-        A.cnt[r >> 2] += (((wp > wthr) ? 1u : 0u) + ((wm > wthr) ? 1u : 0u)) << (8 * (r & 3));
+        count_above(A, r, wp, wthr);
+        count_above(A, r, wm, wthr);
     }
 }
 
@@ -277,7 +293,8 @@ ORION_DEVICE void phase_b_int(const float2 *prg, const float *pb, const unsigned
         A.azs[r] = fma2(make_float2(wp, wp), make_float2(pb[pp], 1.0f), A.azs[r]);
         A.axy[r] = fma2(make_float2(wm, wm), prg[pm], A.axy[r]);
         A.azs[r] = fma2(make_float2(wm, wm), make_float2(pb[pm], 1.0f), A.azs[r]);
-        A.cnt[r >> 2] += (((wp > wthr) ? 1u : 0u) + ((wm > wthr) ? 1u : 0u)) << (8 * (r & 3));
+        count_above(A, r, wp, wthr);
+        count_above(A, r, wm, wthr);
     }
 }
 
