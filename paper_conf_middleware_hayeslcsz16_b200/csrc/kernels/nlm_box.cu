@@ -20,7 +20,8 @@
 //
 // CTA = 128 threads (4 warps); output tile TW = 122 columns x TH = 23 rows.
 // Shared memory: the input tile (TW+18) x (TH+12) with a 9-column / 6-row
-// clamp-to-edge halo as three planar fp32 arrays (odd pitch), and GMAX buffers of
+// clamp-to-edge halo as an (r, g) float2 plane and a b plane (odd pitch; one LDS.64 + one
+// LDS per pixel, conflict-free for both access patterns below), and GMAX buffers of
 // H_o, 32 rows x 128 columns each (odd pitch).  Per pass:
 //   phase A: warp w computes H_o for columns [32w, 32w+32) of each buffer; lane = row
 //            (32 rows = TH + 9), sliding along the row over 38 difference values per
@@ -72,12 +73,6 @@ ORION_DEVICE void window7(const T (&a)[N + 6], T (&out)[N])
     for (int k = 0; k < N; ++k) out[k] = add1(add1(p[k], p[k + 2]), add1(p[k + 4], a[k + 6]));
 }
 
-ORION_DEVICE float diff2(float ar, float ag, float ab, float br, float bg, float bb)
-{
-    const float dx = __fsub_rn(ar, br), dy = __fsub_rn(ag, bg), dz = __fsub_rn(ab, bb);
-    return __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));
-}
-
 // |a - c|^2 with the (r, g) channels packed: a.rg + (-c.rg) on FADD2, squares on FMUL2, then
 // (dr^2 + dg^2) + db^2.  A sum of non-negative terms, 3 roundings deep.
 ORION_DEVICE float2 neg2(float2 a) { return make_float2(-a.x, -a.y); }
@@ -89,15 +84,9 @@ ORION_DEVICE float diff2rg(float2 arg, float ab, float2 ncrg, float cb)
     return __fmaf_rn(db, db, __fadd_rn(q.x, q.y));
 }
 
-ORION_DEVICE float2 diff2x2(float2 ar, float2 ag, float2 ab, float br, float bg, float bb)
-{
-    const float2 dx = sub2(ar, make_float2(br, br)), dy = sub2(ag, make_float2(bg, bg)),
-                 dz = sub2(ab, make_float2(bb, bb));
-    return fma2(dz, dz, fma2(dy, dy, mul2(dx, dx)));
-}
-
-// Phase A for G offsets (i, j1 .. j1+G-1): lane = row r, warp's 32 H columns.  Offsets
-// g = 0, 1 run packed (fp32x2), offset g = 2 scalar.
+// Phase A for G offsets (i, j1 .. j1+G-1): lane = row r, warp's 32 H columns.  Differences
+// are channel-packed (diff2rg); the window sums of offsets g = 0, 1 run packed (fp32x2),
+// offset g = 2 scalar.
 template <int G>
 ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lane, int warp, int i,
                           int j1)
@@ -129,7 +118,8 @@ ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lan
         const float2 ncrg = neg2(prg[rowc + q]);
         const float cbv = pb[rowc + q];
         if (GP > 0)
-            dp[GP > 0 ? q : 0] = make_float2(diff2rg(wrg[0], wb[0], ncrg, cbv), diff2rg(wrg[GP > 0 ? 1 : 0], wb[GP > 0 ? 1 : 0], ncrg, cbv));
+            dp[GP > 0 ? q : 0] = make_float2(diff2rg(wrg[0], wb[0], ncrg, cbv),
+                                             diff2rg(wrg[GP > 0 ? 1 : 0], wb[GP > 0 ? 1 : 0], ncrg, cbv));
         if (GS > 0) ds[GS > 0 ? q : 0] = diff2rg(wrg[G - 1], wb[G - 1], ncrg, cbv);
     }
     if (GP > 0) {
@@ -256,10 +246,10 @@ ORION_DEVICE void phase_a_int(const float2 *prg, const float *pb, unsigned *hs, 
         }
         wrg[G - 1] = prg[rows + c + G - 1];
         wb[G - 1] = pb[rows + c + G - 1];
-        const float2 crg = prg[rowc + c];
-        const float cr = crg.x, cg = crg.y, cbv = pb[rowc + c];
+        const float2 ncrg = neg2(prg[rowc + c]);
+        const float cbv = pb[rowc + c];
 #pragma unroll
-        for (int g = 0; g < G; ++g) q[g][c] = quant(diff2(wrg[g].x, wrg[g].y, wb[g], cr, cg, cbv));
+        for (int g = 0; g < G; ++g) q[g][c] = quant(diff2rg(wrg[g], wb[g], ncrg, cbv));
     }
 #pragma unroll
     for (int g = 0; g < G; ++g) {
