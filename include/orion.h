@@ -118,8 +118,11 @@ orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int bloc
 
 /* ---- code generation (question 1; host-only, no GPU needed) ------------------------------ */
 
-/* Kernel ids: "knn_f4", "nlm_f4", "nlm_f4_g1", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32",
- * "hotspot2_f32" (two stencil steps per launch; width % 4 == 0), "srad_f32".
+/* Kernel ids: "knn_f4" (T = 128 / 256 / 64), "nlm_f4" (box sums, 3 offset pairs per pass),
+ * "nlm_f4_i" (same, exact fixed-point integer windows), "nlm_f4_w8" (same tile, 256 threads),
+ * "nlm_f4_g1" (1 pair per pass), "nlm_f4_direct", "nlm_f4_regheavy" (T = 128 / 64),
+ * "hotspot_f32" (T = 256 / 128), "hotspot2_f32" (two stencil steps per launch; width % 4 == 0),
+ * "srad_f32" (register-sliding, any width), "srad_f32_tile" (shared-memory form, same bits).
  * block_threads = 0 selects the kernel's default CTA size.  Fills the natural resources
  * (compiles the kernel's PTX once, uncapped, with the embedded ptxas). */
 orion_status orion_kernel_probe(const char *kernel_id, int block_threads, orion_kernel_resources *out);

@@ -3,6 +3,8 @@
 # command, and one ncu --set full capture per hot kernel.  Outputs land in gpurun_out/
 # (scratch); tools/collect_round.sh copies the summaries into profiles/.
 OUT=gpurun_out
+python -m pytest tests -m gpu -q > $OUT/pytest_gpu.log 2>&1
+python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke.log 2>&1; echo "smoke rc=$?" >> $OUT/smoke.log
 python bench.py > $OUT/bench_c2.log 2>&1
 python bench.py --impl reference --steps 5 --warmup 3 > $OUT/bench_reference.log 2>&1
 python bench.py --workload c1 --cpu-seconds 5 > $OUT/bench_c1.log 2>&1
@@ -14,7 +16,7 @@ python bench.py --workload srad --steps 100 --warmup 12 --cpu-seconds 5 > $OUT/b
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
     python bench.py --steps 20 --warmup 5 --rounds 3 --no-cpu-baseline --no-carveout-axis > $OUT/bench_under_ncu.log 2>&1
 for spec in "nlm_f4 -1 2048 2048 nlm_box3" "knn_f4 orig 2048 2048 knn" "nlm_f4_regheavy orig 4096 4096 nlm_regheavy" \
-            "hotspot_f32 3 8192 8192 hotspot_f32" "hotspot2_f32 2 8192 8192 hotspot2" "srad_f32 5 8192 8192 srad2" \
+            "hotspot_f32 3 8192 8192 hotspot_f32" "hotspot2_f32 2 8192 8192 hotspot2" "srad_f32 2 8192 8192 srad4" \
             "nlm_f4_w8 -1 2048 2048 nlm_box256"; do
   set -- $spec
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:orion_$5 -c 1 -f -o $OUT/prof_$1 \
