@@ -1,0 +1,69 @@
+"""Per-level ncu evidence (SURVEY 8(d) "ncu evidence per level"): profile one launch of every
+occupancy level of a kernel with a small metric set and write a table to profiles/.
+
+On the GPU box:   python tools/ncu_levels.py run KERNEL W H [THREADS]   -> gpurun_out/levels_KERNEL.csv
+Here:             python tools/ncu_levels.py summarise KERNEL ROUND     -> profiles/ncu_levels_ROUND_KERNEL.txt
+"""
+import csv
+import os
+import subprocess
+import sys
+
+METRICS = [
+    "gpu__time_duration.sum",
+    "launch__registers_per_thread",
+    "launch__occupancy_limit_registers",
+    "launch__occupancy_limit_shared_mem",
+    "sm__maximum_warps_per_active_cycle_pct",
+    "sm__warps_active.avg.pct_of_peak_sustained_active",
+    "l1tex__t_bytes_pipe_lsu_mem_local_op_ld.sum",
+    "l1tex__t_bytes_pipe_lsu_mem_local_op_st.sum",
+    "dram__bytes_read.sum",
+    "dram__bytes_write.sum",
+    "smsp__issue_active.avg.pct_of_peak_sustained_active",
+    "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
+    "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
+]
+SHORT = ["us", "regs", "lim_reg", "lim_smem", "occ_theo%", "occ_ach%", "local_ld_MB", "local_st_MB", "dram_rd_MB",
+         "dram_wr_MB", "issue%", "fma%", "long_sb"]
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def run(kernel, W, H, threads="0"):
+    out = os.path.join(ROOT, "gpurun_out", f"levels_{kernel}.csv")
+    cmd = ["ncu", "--clock-control", "none", "--csv", "--metrics", ",".join(METRICS), "-k", "regex:orion_",
+           "--log-file", out, sys.executable, os.path.join(ROOT, "tools", "ncu_one.py"), kernel, "all", W, H, threads]
+    subprocess.run(cmd, check=True)
+
+
+def summarise(kernel, rnd):
+    path = os.path.join(ROOT, "gpurun_out", f"levels_{kernel}.csv")
+    rows = [r for r in csv.reader(l for l in open(path) if l.startswith('"'))]
+    hdr, data = rows[0], rows[1:]
+    iid, iname, ival, iunit = hdr.index("ID"), hdr.index("Metric Name"), hdr.index("Metric Value"), hdr.index("Metric Unit")
+    per = {}
+    for r in data:
+        per.setdefault(int(r[iid]), {})[r[iname]] = (r[ival], r[iunit])
+
+    def val(m, name):
+        v, unit = m.get(name, ("nan", ""))
+        x = float(v.replace(",", ""))
+        scale = {"byte": 1e-6, "Kbyte": 1e-3, "Mbyte": 1.0, "Gbyte": 1e3, "nsecond": 1e-3, "usecond": 1.0,
+                 "msecond": 1e3}.get(unit, 1.0)
+        return x * scale
+
+    lines = [f"# ncu per-level evidence: {kernel} (one launch per level, MIN_CARVEOUT realisation, "
+             f"--clock-control none; times are cold, single-launch)",
+             "level " + " ".join(f"{s:>11s}" for s in SHORT)]
+    for k in sorted(per):
+        lines.append(f"{k:5d} " + " ".join(f"{val(per[k], m):11.2f}" for m in METRICS))
+    dst = os.path.join(ROOT, "profiles", f"ncu_levels_{rnd}_{kernel}.txt")
+    open(dst, "w").write("\n".join(lines) + "\n")
+    print("\n".join(lines))
+
+
+if __name__ == "__main__":
+    if sys.argv[1] == "run":
+        run(*sys.argv[2:])
+    else:
+        summarise(sys.argv[2], sys.argv[3])

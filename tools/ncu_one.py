@@ -1,7 +1,8 @@
 """Launch ONE kernel variant once on a synthetic frame (for ncu --set full captures).
 
 usage: python tools/ncu_one.py KERNEL LEVEL W H [THREADS] [REPEAT]
-  LEVEL = index into the level list (-1 = max occupancy, 'orig' = natural build)
+  LEVEL = index into the level list (-1 = max occupancy, 'orig' = natural build, 'all' = every
+  level once, in order).  Levels are realised as bench.py realises them (MIN_CARVEOUT).
 """
 import os
 import sys
@@ -16,8 +17,10 @@ threads = int(sys.argv[5]) if len(sys.argv) > 5 else 0
 repeat = int(sys.argv[6]) if len(sys.argv) > 6 else 1
 torch.cuda.set_device(0)
 sp = torch.cuda.current_stream().cuda_stream
-v, res = O.build_all_levels(0, kernel, threads)
-if lev == "orig":
+v, res = O.build_all_levels(0, kernel, threads, mode=O.REALISE_MIN_CARVEOUT)
+if lev == "all":
+    li = None
+elif lev == "orig":
     li = max((i for i, l in enumerate(v.planned) if l.reg_cap == 0), key=lambda i: v.planned[i].ctas_per_sm)
 else:
     li = int(lev) % len(v)
@@ -40,7 +43,8 @@ else:
     b = torch.empty((H, W, 4), device="cuda")
     O.generate_rgba(0, a.data_ptr(), W, H, sigma=0.13, stream=sp)
     args = O.denoise_args(kernel, a.data_ptr(), b.data_ptr(), W, H)
-for _ in range(repeat):
-    v.launch(li, args, sp)
-torch.cuda.synchronize()
-print("launched", kernel, "level", li, v.level(li), v.info(li))
+for i in (range(len(v)) if li is None else [li]):
+    for _ in range(repeat):
+        v.launch(i, args, sp)
+    torch.cuda.synchronize()
+    print("launched", kernel, "level", i, v.level(i), v.info(i))
