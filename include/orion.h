@@ -247,6 +247,26 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
                                   void *dev_aux, void *stream, orion_step_report *out,
                                   long long *h2d_bytes, long long *d2h_bytes);
 
+/* A whole iterative stencil run end to end from HOST buffers -- the Rodinia driver shape
+ * (copy the grid in, iterate, copy it out), the iterations being the ones
+ * Fig. 9 tunes across (P:L651-P:L653).  Kernels of kind hotspot ("hotspot_f32",
+ * "hotspot2_f32") and srad ("srad_f32", "srad_f32_tile") only, whole grids only
+ * (a->row_begin = a->src_row_begin = a->dst_row_begin = 0, a->row_end = a->src_row_end =
+ * a->height).
+ *   a->src  host initial grid (fp32, width x height, row-major; pinned for async copies)
+ *   a->aux  hotspot: host power map (same shape); srad: ignored
+ *   a->dst  host buffer receiving the grid after `iterations` launches
+ *   dev_a, dev_b  caller-owned device grids (ping-pong), width x height fp32 each
+ *   dev_aux hotspot: device power map buffer (filled here); srad: the device float q0sqr
+ *   roi     srad only: {r1, r2, c1, c2} of the ROI statistics run before every iteration
+ * Copies in, runs `iterations` orion_tune_step iterations on `stream` (hotspot2_f32 advances
+ * two time steps per iteration), copies the final grid out and synchronises the stream.
+ * Bytes copied are returned in *h2d_bytes / *d2h_bytes.  ORION_E_INVALID on other kernels,
+ * partial row ranges or missing buffers. */
+orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterations, void *dev_a, void *dev_b,
+                                 void *dev_aux, const int *roi, void *stream, long long *h2d_bytes,
+                                 long long *d2h_bytes);
+
 /* Pipelined end-to-end iterations from HOST buffers.  The pipe owns `depth` slots of device
  * staging buffers (width x max_rows elements each for src, dst and -- stencil -- aux;
  * allocated here, never in submit) and three non-blocking streams: the H2D copy of frame n,

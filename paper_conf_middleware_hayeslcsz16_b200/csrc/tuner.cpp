@@ -341,6 +341,48 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
     return ORION_OK;
 }
 
+orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterations, void *dev_a, void *dev_b,
+                                 void *dev_aux, const int *roi, void *stream, long long *h2d, long long *d2h)
+{
+    if (!t || !a || !dev_a || !dev_b || iterations < 1 || !a->src || !a->dst)
+        return fail(ORION_E_INVALID, "orion_tune_run_host: bad argument");
+    const KernelDef &def = *t->v->def;
+    const bool srad = def.kind == K_SRAD;
+    if (def.kind != K_STENCIL && !srad) return fail(ORION_E_INVALID, "orion_tune_run_host: stencil kernels only");
+    if (a->row_begin != 0 || a->row_end != a->height || a->src_row_begin != 0 || a->src_row_end != a->height ||
+        a->dst_row_begin != 0 || a->width < 1 || a->height < 1)
+        return fail(ORION_E_INVALID, "orion_tune_run_host: whole grids only (rows [0, height))");
+    if (!dev_aux || (!srad && !a->aux) || (srad && !roi))
+        return fail(ORION_E_INVALID, "orion_tune_run_host: missing aux / roi");
+    const size_t bytes = (size_t)a->width * (size_t)a->height * 4;
+    const Driver &D = drv();
+    CUstream s = (CUstream)stream;
+    ORION_TRY(ensure_context(t->v->device));
+    ORION_CU(D.cuMemcpyHtoDAsync((CUdeviceptr)dev_a, a->src, bytes, s));
+    size_t in_bytes = bytes;
+    if (!srad) {
+        ORION_CU(D.cuMemcpyHtoDAsync((CUdeviceptr)dev_aux, a->aux, bytes, s));
+        in_bytes += bytes;
+    }
+    void *cur = dev_a, *nxt = dev_b;
+    for (int it = 0; it < iterations; ++it) {
+        if (srad)
+            ORION_TRY(orion_srad_roi_stats(t->v->device, cur, a->width, a->height, roi[0], roi[1], roi[2], roi[3],
+                                           dev_aux, stream));
+        orion_args da = *a;
+        da.src = cur;
+        da.dst = nxt;
+        da.aux = dev_aux;
+        ORION_TRY(orion_tune_step(t, &da, stream, nullptr));
+        std::swap(cur, nxt);
+    }
+    ORION_CU(D.cuMemcpyDtoHAsync(a->dst, (CUdeviceptr)cur, bytes, s));
+    ORION_CU(D.cuStreamSynchronize(s));
+    if (h2d) *h2d = (long long)in_bytes;
+    if (d2h) *d2h = (long long)bytes;
+    return ORION_OK;
+}
+
 }  // extern "C"
 
 // ---- pipelined host-buffer iterations --------------------------------------------------------

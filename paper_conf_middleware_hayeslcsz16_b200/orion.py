@@ -128,6 +128,8 @@ def lib() -> ctypes.CDLL:
                 "orion_tune_step_host": [V, P(Args), V, V, V, V, P(StepReport), P(ctypes.c_longlong),
                                          P(ctypes.c_longlong)],
                 "orion_tune_split": [V, P(Args), I, V, P(StepReport)],
+                "orion_tune_run_host": [V, P(Args), I, V, V, V, P(I), V, P(ctypes.c_longlong),
+                                        P(ctypes.c_longlong)],
                 "orion_host_pipe_create": [V, I, I, I, P(V)],
                 "orion_host_pipe_submit": [V, P(Args), P(StepReport), P(ctypes.c_longlong), P(ctypes.c_longlong)],
                 "orion_host_pipe_drain": [V],
@@ -359,6 +361,15 @@ class Tuner:
                                           ctypes.byref(r), ctypes.byref(hi), ctypes.byref(ho)),
                "orion_tune_step_host")
         return r, hi.value, ho.value
+
+    def run_host(self, args: Args, iterations: int, dev_a: int, dev_b: int, dev_aux: int, roi=None, stream=None):
+        """orion_tune_run_host: a whole stencil run from host grids (copy in, iterate, copy out)."""
+        hi, ho = ctypes.c_longlong(), ctypes.c_longlong()
+        r = (ctypes.c_int * 4)(*roi) if roi is not None else None
+        _check(lib().orion_tune_run_host(self.h, ctypes.byref(args), iterations, ctypes.c_void_p(dev_a),
+                                         ctypes.c_void_p(dev_b), ctypes.c_void_p(dev_aux), r, _s(stream),
+                                         ctypes.byref(hi), ctypes.byref(ho)), "orion_tune_run_host")
+        return hi.value, ho.value
 
     def ladder(self):
         d, n = ctypes.c_int(), ctypes.c_int()
