@@ -140,14 +140,19 @@ typedef struct orion_variants orion_variants;   /* opaque, library-owned */
  * the kernel's PTX is compiled once (at library build time) and assembled by ptxas once
  * per distinct register cap; every variant is loaded on `device`, its padding recomputed
  * from the ACTUAL register count, the carveout pinned when padding is used, and its
- * realised CTAs/SM checked with cuOccupancyMaxActiveBlocksPerMultiprocessor
- * (-> ORION_E_OCCUPANCY_MISMATCH).  Every variant is launched once (warm-up, defeats lazy
+ * realised CTAs/SM checked twice: with cuOccupancyMaxActiveBlocksPerMultiprocessor and by a
+ * residency probe launch of the function itself (every CTA counts the CTAs resident on its
+ * SM; the driver may run a padded launch in a larger carveout configuration than requested,
+ * which the API does not model).  A level whose planned configuration does not measure k is
+ * retried in each larger configuration; none -> ORION_E_OCCUPANCY_MISMATCH.  The probe
+ * launches (148 x 32 CTAs, ~1 ms) run on the legacy default stream during the build.  Every variant is launched once (warm-up, defeats lazy
  * loading) only when orion_launch is first called with it. */
 orion_status orion_build_variants(int device, const char *kernel_id, int block_threads,
                                   const orion_level *levels, int n, orion_variants **out);
 orion_status orion_variants_count(const orion_variants *v, int *n);
 /* The realised level (pad recomputed from actual registers) of variant `level_idx`. */
 orion_status orion_variant_level(const orion_variants *v, int level_idx, orion_level *out);
+/* verified_ctas_per_sm = the residency MEASURED by the probe launch (equal to the level's k). */
 orion_status orion_variant_info(const orion_variants *v, int level_idx, int *regs, int *spill_store_bytes,
                                 int *spill_load_bytes, int *local_bytes, int *verified_ctas_per_sm);
 /* The kernel's natural resources (what orion_kernel_probe returned when building). */

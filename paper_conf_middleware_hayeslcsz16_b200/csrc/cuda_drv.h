@@ -21,7 +21,8 @@ namespace orion {
     X(cuOccupancyMaxActiveBlocksPerMultiprocessor) X(cuEventCreate) X(cuEventDestroy)             \
     X(cuEventRecord) X(cuEventSynchronize) X(cuEventElapsedTime) X(cuMemcpyHtoDAsync)             \
     X(cuMemcpyDtoHAsync) X(cuStreamSynchronize) X(cuGetErrorString) X(cuGetErrorName)            \
-    X(cuMemAlloc) X(cuMemFree) X(cuStreamCreate) X(cuStreamDestroy) X(cuStreamWaitEvent)
+    X(cuMemAlloc) X(cuMemFree) X(cuStreamCreate) X(cuStreamDestroy) X(cuStreamWaitEvent)          \
+    X(cuMemsetD32) X(cuMemcpyDtoH) X(cuCtxSynchronize)
 
 struct Driver {
 #define ORION_DECL(f) decltype(&::f) f = nullptr;

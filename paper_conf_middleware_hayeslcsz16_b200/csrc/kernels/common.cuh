@@ -11,6 +11,33 @@
 
 #define ORION_DEVICE __device__ __forceinline__
 
+// Residency probe (build time only, a.probe != NULL): thread 0 of each CTA counts the CTAs
+// resident on its SM (probe[smid]), records the maximum (probe[1024 + smid]) and holds the
+// CTA -- all its warps waiting at a barrier, with the function's real registers and shared
+// memory allocated -- for 20 us; the kernel then returns without touching its buffers.  orion_build_variants launches a full
+// grid this way to MEASURE the CTAs/SM each occupancy variant actually gets.
+ORION_DEVICE bool orion_probe(const orion_kargs &a)
+{
+    if (a.probe == nullptr) return false;
+    if (threadIdx.x == 0 && threadIdx.y == 0) {
+        unsigned smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        smid &= 1023u;
+        const unsigned c = atomicAdd(a.probe + smid, 1u) + 1u;
+        atomicMax(a.probe + 1024 + smid, c);
+        unsigned long long t0, t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        do {
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        } while (t - t0 < 20000ull);
+        atomicSub(a.probe + smid, 1u);
+    }
+    __syncthreads();   // every warp stays resident (registers are granted per warp) until then
+    return true;
+}
+#define ORION_PROBE(a) \
+    if (orion_probe(a)) return
+
 ORION_DEVICE int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
 
 // Squared RGB distance, |a - b|^2 with a fixed operation order.

@@ -93,9 +93,9 @@ __device__ __forceinline__ void hotspot_body(const orion_kargs &a)
 }
 
 // T = 256 threads (32 x 8 warps): 128 columns x 8 strips of 16 rows per CTA.
-extern "C" __global__ void __launch_bounds__(256) orion_hotspot_f32_256(orion_kargs a) { hotspot_body<8, 16>(a); }
+extern "C" __global__ void __launch_bounds__(256) orion_hotspot_f32_256(orion_kargs a) { ORION_PROBE(a); hotspot_body<8, 16>(a); }
 // T = 128 threads (32 x 4 warps): 128 columns x 4 strips of 16 rows per CTA.
-extern "C" __global__ void __launch_bounds__(128) orion_hotspot_f32_128(orion_kargs a) { hotspot_body<4, 16>(a); }
+extern "C" __global__ void __launch_bounds__(128) orion_hotspot_f32_128(orion_kargs a) { ORION_PROBE(a); hotspot_body<4, 16>(a); }
 
 // ---- two explicit steps per launch (temporal blocking) -------------------------------------
 // T2 = step(step(T0)) with the intermediate T1 kept in registers: per 2 cell-steps the kernel
@@ -208,4 +208,4 @@ __device__ __forceinline__ void hotspot2_body(const orion_kargs &a)
 }
 
 // T = 256 threads (32 x 8 warps): 128 columns x 8 strips of 16 rows per CTA; 2 steps per launch.
-extern "C" __global__ void __launch_bounds__(256) orion_hotspot2_f32_256(orion_kargs a) { hotspot2_body<8, 16>(a); }
+extern "C" __global__ void __launch_bounds__(256) orion_hotspot2_f32_256(orion_kargs a) { ORION_PROBE(a); hotspot2_body<8, 16>(a); }

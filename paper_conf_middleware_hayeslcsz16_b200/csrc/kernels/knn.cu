@@ -73,8 +73,8 @@ __device__ __forceinline__ void knn_body(const orion_kargs &a)
 }
 
 // T = 128 threads (32 x 4), 16-row tiles.
-extern "C" __global__ void __launch_bounds__(128) orion_knn_f4_128(orion_kargs a) { knn_body<32, 4, 4>(a); }
+extern "C" __global__ void __launch_bounds__(128) orion_knn_f4_128(orion_kargs a) { ORION_PROBE(a); knn_body<32, 4, 4>(a); }
 // T = 256 threads (32 x 8), 32-row tiles.
-extern "C" __global__ void __launch_bounds__(256) orion_knn_f4_256(orion_kargs a) { knn_body<32, 8, 4>(a); }
+extern "C" __global__ void __launch_bounds__(256) orion_knn_f4_256(orion_kargs a) { ORION_PROBE(a); knn_body<32, 8, 4>(a); }
 // T = 64 threads (8 x 8), the SDK's CTA shape, 32-row tiles.
-extern "C" __global__ void __launch_bounds__(64) orion_knn_f4_64(orion_kargs a) { knn_body<8, 8, 4>(a); }
+extern "C" __global__ void __launch_bounds__(64) orion_knn_f4_64(orion_kargs a) { ORION_PROBE(a); knn_body<8, 8, 4>(a); }

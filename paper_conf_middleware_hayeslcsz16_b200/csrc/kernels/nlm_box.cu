@@ -389,8 +389,8 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 }  // namespace
 
 // One pair per pass: 3 planar planes + 1 H buffer = 75 732 B of shared memory.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kargs a) { nlm_box_body<1, false>(a); }
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<1, false>(a); }
 // Up to three pairs per pass: 3 planar planes + 3 H buffers = 108 756 B of shared memory.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_box3_f4_128(orion_kargs a) { nlm_box_body<3, false>(a); }
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_box3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<3, false>(a); }
 // Integer (fixed-point, exact) box sums, up to three pairs per pass.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_boxi3_f4_128(orion_kargs a) { nlm_box_body<3, true>(a); }
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_boxi3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<3, true>(a); }

@@ -130,6 +130,7 @@ __constant__ int kPass3[10][3] = {
 // 3 planar planes + 3 H buffers = 108 756 B of shared memory; 2 CTAs x 8 warps per SM.
 extern "C" __global__ void __launch_bounds__(256) orion_nlm_box256_f4_256(orion_kargs a)
 {
+    ORION_PROBE(a);
     extern __shared__ float4 smem4[];
     float *pr = reinterpret_cast<float *>(smem4);
     float *pg = pr + PR * PW;

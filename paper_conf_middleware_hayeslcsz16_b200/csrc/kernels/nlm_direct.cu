@@ -18,5 +18,6 @@
 
 extern "C" __global__ void __launch_bounds__(128) orion_nlm_direct_f4_128(orion_kargs a)
 {
+    ORION_PROBE(a);
     nlm_direct_body<32, 4, false>(a);
 }

@@ -6,9 +6,11 @@
 
 extern "C" __global__ void __launch_bounds__(128) orion_nlm_regheavy_f4_128(orion_kargs a)
 {
+    ORION_PROBE(a);
     nlm_direct_body<32, 4, true>(a);
 }
 extern "C" __global__ void __launch_bounds__(64) orion_nlm_regheavy_f4_64(orion_kargs a)
 {
+    ORION_PROBE(a);
     nlm_direct_body<8, 8, true>(a);
 }

@@ -90,6 +90,7 @@ constexpr int CW = TW + 1, CH = TH + 1;       // c tile: x0 .. x0+TW, y0 .. y0+T
 // derivative arrays to DRAM instead); then J' is formed.
 extern "C" __global__ void __launch_bounds__(256) orion_srad_f32_256(orion_kargs a)
 {
+    ORION_PROBE(a);
     extern __shared__ float4 smem4[];
     float *js = reinterpret_cast<float *>(smem4);   // JH x JW
     float *cs = js + JH * JW;                       // CH x CW
@@ -289,6 +290,7 @@ __device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys,
 // T = 256 threads (32 x 8 warps), output tile 124 x 128.
 extern "C" __global__ void __launch_bounds__(256) orion_srad4_f32_256(orion_kargs a)
 {
+    ORION_PROBE(a);
     const int w = threadIdx.y;
     if ((a.width & 3) == 0) {
         const int ys = a.row_begin + blockIdx.y * 128 + w * 16;

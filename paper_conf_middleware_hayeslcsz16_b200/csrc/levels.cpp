@@ -147,6 +147,12 @@ bool realise(const orion_device_limits &d, int T, int regs, int smem_static, int
     return false;
 }
 
+const int *carveout_configs_kb(int *n)
+{
+    *n = (int)(sizeof kCarveoutKB / sizeof kCarveoutKB[0]);
+    return kCarveoutKB;
+}
+
 int level_carveout_pct(const orion_device_limits &d, const orion_level &L)
 {
     return L.carveout_kb > 0 ? carveout_pct_for_kb(d, L.carveout_kb) : -1;

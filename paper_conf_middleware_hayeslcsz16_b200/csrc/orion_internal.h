@@ -42,6 +42,10 @@ int pad_for_level(const orion_device_limits &d, int T, int regs, int smem_static
                   int carveout_pct);
 int carveout_pct_for_kb(const orion_device_limits &d, int kb);
 int level_carveout_pct(const orion_device_limits &d, const orion_level &L);
+// Per-SM shared-memory budget a carveout preference requests (pct < 0: the maximum).
+int carveout_pref_bytes(const orion_device_limits &d, int pct);
+// The unified L1 / shared-memory configurations (KB), ascending.
+const int *carveout_configs_kb(int *n);
 
 // ---- kernel registry + code generation (registry.cpp) -------------------------------------
 enum KernelKind { K_KNN = 0, K_NLM = 1, K_STENCIL = 2, K_SRAD = 3 };

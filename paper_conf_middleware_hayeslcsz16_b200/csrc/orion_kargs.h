@@ -14,6 +14,9 @@ typedef struct {
     int dst_row_begin;               /* global row of dst's first row                               */
     int iparam0;                     /* denoise: lerp count threshold (cnt >= iparam0 -> lerpC)     */
     float fparam[8];                 /* denoise: -Noise*log2e, lerpC, wthr ; stencil: sdc,rx,ry,rz,amb */
+    unsigned *probe;                 /* NULL in every real launch.  Non-NULL: residency probe only --
+                                        the CTA records how many CTAs share its SM and exits
+                                        (orion_probe in kernels/common.cuh)                        */
 } orion_kargs;
 
 #endif

@@ -13,6 +13,8 @@
 #include <algorithm>
 #include <cmath>
 #include <cstring>
+#include <string>
+#include <vector>
 
 #include "orion_internal.h"
 
@@ -79,6 +81,47 @@ orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const
     return ORION_OK;
 }
 
+// Device scratch of the residency probe: 1024 live counters + 1024 maxima (per %smid).
+struct ProbeBuffer {
+    CUdeviceptr p = 0;
+    orion_status alloc()
+    {
+        if (drv().cuMemAlloc(&p, 2048 * sizeof(unsigned)) != CUDA_SUCCESS) {
+            p = 0;
+            return fail(ORION_E_CUDA, "cuMemAlloc (residency probe)");
+        }
+        return ORION_OK;
+    }
+    ~ProbeBuffer()
+    {
+        if (p) drv().cuMemFree(p);
+    }
+};
+
+// Launch `fn` as a residency probe (kargs.probe set: every CTA only counts its SM's resident
+// CTAs, then holds for 20 us) over sm_count x 32 CTAs, and return the largest number of CTAs
+// ever resident together on one SM.
+orion_status measure_residency(const orion_variants &v, const KernelDef &def, CUfunction fn, int dyn_bytes,
+                               const ProbeBuffer &buf, int *out)
+{
+    const Driver &D = drv();
+    ORION_CU(D.cuMemsetD32(buf.p, 0u, 2048));
+    orion_kargs k;
+    std::memset(&k, 0, sizeof k);
+    k.probe = reinterpret_cast<unsigned *>(buf.p);
+    void *params[] = {&k};
+    const unsigned grid = (unsigned)(v.dev.sm_count * v.dev.max_blocks_per_sm);
+    ORION_CU(D.cuLaunchKernel(fn, grid, 1, 1, (unsigned)def.bx, (unsigned)def.by, 1, (unsigned)dyn_bytes, nullptr,
+                              params, nullptr));
+    ORION_CU(D.cuCtxSynchronize());
+    unsigned host[1024];
+    ORION_CU(D.cuMemcpyDtoH(host, buf.p + 1024 * sizeof(unsigned), sizeof host));
+    unsigned m = 0;
+    for (unsigned x : host) m = std::max(m, x);
+    *out = (int)m;
+    return ORION_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -100,6 +143,8 @@ orion_status orion_build_variants(int device, const char *kernel_id, int block_t
     const Driver &D = drv();
     const int T = def->threads;
     const int need = def->dyn_need();
+    ProbeBuffer probe;
+    ORION_TRY(probe.alloc());
     for (int i = 0; i < n; ++i) {
         const orion_level &L = levels[i];
         if (L.ctas_per_sm < 1 || L.reg_cap < 0 || L.reg_cap > 255)
@@ -115,35 +160,58 @@ orion_status orion_build_variants(int device, const char *kernel_id, int block_t
         ORION_CU(D.cuFuncGetAttribute(&w.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, w.fn));
         ORION_CU(D.cuFuncGetAttribute(&w.local_bytes, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, w.fn));
         ORION_CU(D.cuFuncGetAttribute(&static_smem, CU_FUNC_ATTRIBUTE_SHARED_SIZE_BYTES, w.fn));
-        // the level's carveout: its configuration when it names one, else the maximum
-        // whenever padding turns out to be needed at the actual register count
-        int pct = level_carveout_pct(v->dev, L);
-        int pad = pad_for_level(v->dev, T, w.regs, static_smem, need, L.ctas_per_sm, pct);
-        if (pad > 0 && pct < 0) pct = 100;
-        if (pad < 0)
-            return fail(ORION_E_INFEASIBLE, "level " + std::to_string(L.ctas_per_sm) + " CTAs/SM not realisable at " +
-                                                std::to_string(w.regs) + " registers");
-        w.dyn_bytes = need + pad;
-        w.carveout_pct = pct;
-        ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, w.dyn_bytes));
-        if (pct >= 0) ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, pct));
-        ORION_CU(D.cuOccupancyMaxActiveBlocksPerMultiprocessor(&w.verified, w.fn, T, (size_t)w.dyn_bytes));
-        if (w.verified != L.ctas_per_sm && pct < 0) {
-            // the driver picked a smaller carveout than the calculator assumes: pin it
-            w.carveout_pct = pct = 100;
-            ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, 100));
-            ORION_CU(D.cuOccupancyMaxActiveBlocksPerMultiprocessor(&w.verified, w.fn, T, (size_t)w.dyn_bytes));
+        // Realise level k: the planned carveout first, then every larger configuration.  A
+        // candidate is accepted when both the driver's occupancy API AND the measured
+        // residency (a probe launch of this very function, orion_probe in common.cuh) give k:
+        // the driver treats the carveout preference as a hint and may run a padded launch in a
+        // larger configuration than requested (measured on B200: an 8 KB preference runs in
+        // 16 or 64 KB), which the occupancy API does not model.
+        std::vector<int> pcts{level_carveout_pct(v->dev, L)};
+        {
+            int nc = 0;
+            const int *kb = carveout_configs_kb(&nc);
+            for (int c = 0; c < nc; ++c)
+                if (kb[c] > std::max(L.carveout_kb, 0) && (long long)kb[c] * 1024 <= v->dev.smem_per_sm)
+                    pcts.push_back(kb[c] * 1024 >= v->dev.smem_per_sm ? 100 : carveout_pct_for_kb(v->dev, kb[c]));
         }
-        if (w.verified != L.ctas_per_sm)
+        int pct = -1, pad = -1, api = 0, measured = 0;
+        bool ok = false;
+        std::string tried;
+        for (int cand : pcts) {
+            pct = cand;
+            pad = pad_for_level(v->dev, T, w.regs, static_smem, need, L.ctas_per_sm, pct);
+            if (pad > 0 && pct < 0) {   // padding needed at the actual register count: pin the maximum
+                pct = 100;
+                pad = pad_for_level(v->dev, T, w.regs, static_smem, need, L.ctas_per_sm, pct);
+            }
+            if (pad < 0) continue;
+            w.dyn_bytes = need + pad;
+            ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, w.dyn_bytes));
+            if (pct >= 0) ORION_CU(D.cuFuncSetAttribute(w.fn, CU_FUNC_ATTRIBUTE_PREFERRED_SHARED_MEMORY_CARVEOUT, pct));
+            ORION_CU(D.cuOccupancyMaxActiveBlocksPerMultiprocessor(&api, w.fn, T, (size_t)w.dyn_bytes));
+            if (api != L.ctas_per_sm) {
+                tried += " pct " + std::to_string(pct) + ": api " + std::to_string(api) + ";";
+                continue;
+            }
+            ORION_TRY(measure_residency(*v, *def, w.fn, w.dyn_bytes, probe, &measured));
+            tried += " pct " + std::to_string(pct) + ": measured " + std::to_string(measured) + ";";
+            if (measured == L.ctas_per_sm) {
+                ok = true;
+                break;
+            }
+        }
+        if (!ok)
             return fail(ORION_E_OCCUPANCY_MISMATCH, std::string(def->entry) + ": level " +
-                                                        std::to_string(L.ctas_per_sm) + " realised as " +
-                                                        std::to_string(w.verified) + " CTAs/SM");
+                                                        std::to_string(L.ctas_per_sm) + " not realisable at " +
+                                                        std::to_string(w.regs) + " registers (" + tried + ")");
+        w.carveout_pct = pct;
+        w.verified = measured;
         w.realised = L;
         w.realised.smem_pad_bytes = pad;
         int limiter = 0;
         ctas_per_sm(v->dev, T, w.regs, static_smem, w.dyn_bytes, pct, &limiter);
         w.realised.limiter = limiter;
-        w.realised.carveout_kb = pct < 0 ? 0 : (pct >= 100 ? v->dev.smem_per_sm / 1024 : L.carveout_kb);
+        w.realised.carveout_kb = pct < 0 ? 0 : carveout_pref_bytes(v->dev, pct) / 1024;
         w.realised.warps_per_sm = L.ctas_per_sm * warps_of(v->dev, T);
         w.realised.occupancy_permille = w.realised.warps_per_sm * 1000 / (v->dev.max_threads_per_sm / v->dev.warp_size);
     }

@@ -23,9 +23,11 @@ METRICS = [
     "smsp__issue_active.avg.pct_of_peak_sustained_active",
     "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
     "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
+    "launch__shared_mem_config_size",
+    "launch__shared_mem_per_block_dynamic",
 ]
 SHORT = ["us", "regs", "lim_reg", "lim_smem", "occ_theo%", "occ_ach%", "local_ld_MB", "local_st_MB", "dram_rd_MB",
-         "dram_wr_MB", "issue%", "fma%", "long_sb"]
+         "dram_wr_MB", "issue%", "fma%", "long_sb", "cfg_KB", "dyn_KB"]
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
@@ -41,22 +43,27 @@ def summarise(kernel, rnd):
     rows = [r for r in csv.reader(l for l in open(path) if l.startswith('"'))]
     hdr, data = rows[0], rows[1:]
     iid, iname, ival, iunit = hdr.index("ID"), hdr.index("Metric Name"), hdr.index("Metric Value"), hdr.index("Metric Unit")
-    per = {}
+    ik = hdr.index("Kernel Name")
+    per, names = {}, {}
     for r in data:
+        if "_gen_" in r[ik] or "_stats" in r[ik]:     # the input generator / SRAD statistics
+            continue
         per.setdefault(int(r[iid]), {})[r[iname]] = (r[ival], r[iunit])
+        names[int(r[iid])] = r[ik]
 
     def val(m, name):
         v, unit = m.get(name, ("nan", ""))
         x = float(v.replace(",", ""))
-        scale = {"byte": 1e-6, "Kbyte": 1e-3, "Mbyte": 1.0, "Gbyte": 1e3, "nsecond": 1e-3, "usecond": 1.0,
-                 "msecond": 1e3}.get(unit, 1.0)
-        return x * scale
+        scale = {"byte": 1e-6, "Kbyte": 1e-3, "Mbyte": 1.0, "Gbyte": 1e3, "nsecond": 1e-3, "ns": 1e-3,
+                 "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3}.get(unit, 1.0)
+        kb = name.startswith("launch__shared_mem")      # reported in KB, not MB
+        return x * scale * (1e3 if kb else 1.0)
 
-    lines = [f"# ncu per-level evidence: {kernel} (one launch per level, MIN_CARVEOUT realisation, "
-             f"--clock-control none; times are cold, single-launch)",
+    lines = [f"# ncu per-level evidence: {kernel} = {names[min(per)]} (one launch per level in level order, "
+             f"MIN_CARVEOUT realisation, --clock-control none; times are cold, single-launch)",
              "level " + " ".join(f"{s:>11s}" for s in SHORT)]
-    for k in sorted(per):
-        lines.append(f"{k:5d} " + " ".join(f"{val(per[k], m):11.2f}" for m in METRICS))
+    for lvl, k in enumerate(sorted(per)):
+        lines.append(f"{lvl:5d} " + " ".join(f"{val(per[k], m):11.2f}" for m in METRICS))
     dst = os.path.join(ROOT, "profiles", f"ncu_levels_{rnd}_{kernel}.txt")
     open(dst, "w").write("\n".join(lines) + "\n")
     print("\n".join(lines))

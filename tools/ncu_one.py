@@ -17,7 +17,8 @@ threads = int(sys.argv[5]) if len(sys.argv) > 5 else 0
 repeat = int(sys.argv[6]) if len(sys.argv) > 6 else 1
 torch.cuda.set_device(0)
 sp = torch.cuda.current_stream().cuda_stream
-v, res = O.build_all_levels(0, kernel, threads, mode=O.REALISE_MIN_CARVEOUT)
+mode = O.REALISE_MAX_SMEM if os.environ.get("ORION_REALISE") == "max" else O.REALISE_MIN_CARVEOUT
+v, res = O.build_all_levels(0, kernel, threads, mode=mode)
 if lev == "all":
     li = None
 elif lev == "orig":
