@@ -71,9 +71,11 @@ typedef struct {
     int reg_cap;             /* ptxas --maxrregcount for this level; 0 = uncapped (natural) */
     int smem_pad_bytes;      /* extra dynamic shared memory that caps residency at k */
     int limiter;             /* ORION_LIM_* bits                                            */
-    int carveout_kb;         /* per-SM shared-memory configuration the level is realised with
+    int carveout_kb;         /* per-SM shared-memory configuration requested for the level
                                 (8 .. 228 KB; the rest of the 256 KB array is L1); 0 = left to
-                                the driver (no padding needed)                               */
+                                the driver.  For padded levels it is the configuration the
+                                residency probe measured k in; unpadded levels may run in a
+                                larger one chosen by the driver, which does not change k     */
 } orion_level;
 
 /* How a level's CTA count is realised (the paper's small- vs large-cache axis, P:L757-P:L761,
