@@ -16,17 +16,19 @@
  *
  * Two forms:
  *   oracle_hotspot_f64 -- the definition in double precision;
- *   oracle_hotspot_f32 -- the same definition evaluated in fp32 with every
- *     operation rounded once, in the order written above (no contraction; this
- *     file is compiled with -ffp-contract=off):
- *       a = ((S + N) - (T + T)) * ry;  b = ((E + W) - (T + T)) * rx;
- *       c = (amb - T) * rz;            T' = T + (((P + a) + b) + c) * sdc
+ *   oracle_hotspot_f32 -- the same definition evaluated in fp32, every operation
+ *     rounded once, in the order written above, with the products that feed a sum
+ *     fused (reading R-HS-FP; explicit fmaf, the file is compiled with
+ *     -ffp-contract=off so nothing else is contracted):
+ *       a = fma(T, -2, S + N);   b = fma(T, -2, E + W);   d = amb - T;
+ *       acc = fma(rz, d, fma(rx, b, fma(ry, a, P)));      T' = fma(sdc, acc, T)
  *
  * Pins (tests/test_oracle_stencil.py): uniform T = amb, P = 0 is a fixed point;
  * the discrete Neumann cosine modes are eigenvectors with a closed-form
  * eigenvalue (checked after many steps); heat conservation with rz = 0, P = 0;
  * the maximum principle; f32 form within the fp32 error bound of f64.
  */
+#include <math.h>
 #include <stddef.h>
 #include <stdlib.h>
 #include <string.h>
@@ -82,12 +84,11 @@ int oracle_hotspot_f32(const float *t0, const float *power, int W, int H, int st
                 float Wv = a[(size_t)y * W + clampi(x - 1, 0, W - 1)];
                 float E = a[(size_t)y * W + clampi(x + 1, 0, W - 1)];
                 float P = power[(size_t)y * W + x];
-                float t2 = T + T;
-                float av = ((S + N) - t2) * ry;
-                float bv = ((E + Wv) - t2) * rx;
-                float cv = (amb - T) * rz;
-                float acc = ((P + av) + bv) + cv;
-                b[(size_t)y * W + x] = T + acc * sdc;
+                float av = fmaf(T, -2.0f, S + N);
+                float bv = fmaf(T, -2.0f, E + Wv);
+                float dv = amb - T;
+                float acc = fmaf(rz, dv, fmaf(rx, bv, fmaf(ry, av, P)));
+                b[(size_t)y * W + x] = fmaf(sdc, acc, T);
             }
         float *t = a; a = b; b = t;
     }

@@ -2,9 +2,10 @@
 // (Table 2, Rodinia [6] P:L1147; update rule per DESIGN.md reading
 // R-O3, constants per reading R-A15):
 //   T' = T + sdc * ( P + (S + N - 2T)*ry + (E + W - 2T)*rx + (amb - T)*rz )
-// with clamp-to-edge neighbours, evaluated in fp32 in exactly this order (one
-// rounding per operation, no contraction):
-//   t2 = T+T; a = ((S+N)-t2)*ry; b = ((E+W)-t2)*rx; c = (amb-T)*rz; T' = T + (((P+a)+b)+c)*sdc
+// with clamp-to-edge neighbours, evaluated in fp32 in exactly this order, one rounding per
+// operation with the products that feed a sum fused (reading R-HS-FP; 9 operations):
+//   a = fma(T,-2,S+N); b = fma(T,-2,E+W); d = amb-T; acc = fma(rz,d,fma(rx,b,fma(ry,a,P)));
+//   T' = fma(sdc, acc, T)
 //
 // HBM-bound: 12 algorithmic bytes per cell-step (read T and P, write T').  Each warp
 // owns 128 consecutive columns (4 per lane, 16-byte vector loads and stores) and walks
@@ -17,12 +18,11 @@
 
 ORION_DEVICE float hs_cell(float T, float N, float S, float E, float Wv, float P, const float (&c)[5])
 {
-    const float t2 = __fadd_rn(T, T);
-    const float av = __fmul_rn(__fsub_rn(__fadd_rn(S, N), t2), c[2]);
-    const float bv = __fmul_rn(__fsub_rn(__fadd_rn(E, Wv), t2), c[1]);
-    const float cv = __fmul_rn(__fsub_rn(c[4], T), c[3]);
-    const float acc = __fadd_rn(__fadd_rn(__fadd_rn(P, av), bv), cv);
-    return __fadd_rn(T, __fmul_rn(acc, c[0]));
+    const float av = __fmaf_rn(T, -2.0f, __fadd_rn(S, N));
+    const float bv = __fmaf_rn(T, -2.0f, __fadd_rn(E, Wv));
+    const float dv = __fsub_rn(c[4], T);
+    const float acc = __fmaf_rn(c[3], dv, __fmaf_rn(c[1], bv, __fmaf_rn(c[2], av, P)));
+    return __fmaf_rn(c[0], acc, T);
 }
 
 template <int BY, int RY>
@@ -112,100 +112,158 @@ struct Row4 {
     float xo;      // T one further out: cx0-2 (lane 0), cx0+129 (lane 31)
 };
 
+// The rows a warp walks are streamed through a ring in shared memory: fetched NB-1 rows
+// ahead with cp.async (LDGSTS: global -> shared without registers), so the bytes in flight
+// per SM no longer depend on the register budget of the occupancy level.  Each lane copies
+// its own 16 bytes of the T0 and P rows (edge lanes also their outer columns) into its warp's
+// ring slot and later reads back exactly what it copied, so no warp barrier is needed.  The
+// strip is peeled so the loop body is uniform, and rows advance by pointer increments.
+namespace {
+constexpr int H2_NB = 4;                    // ring slots per warp (NB-1 rows in flight)
+constexpr int H2_SLOT = 136 + 136;          // floats: T0 segment [base-4, base+132), P segment
+}  // namespace
+
+__device__ __forceinline__ void cp_async16(float *sdst, const float *gsrc)
+{
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+                 "l"(gsrc));
+}
+__device__ __forceinline__ void cp_async4(float *sdst, const float *gsrc)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+                 "l"(gsrc));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
 template <int BY, int RY>
 __device__ __forceinline__ void hotspot2_body(const orion_kargs &a)
 {
-    const float *tin = (const float *)a.src;
-    const float *pw = (const float *)a.aux;
-    float *tout = (float *)a.dst;
+    extern __shared__ float4 smem4[];
     const int W = a.width, H = a.height;
     const int lane = threadIdx.x;
     const int ys = a.row_begin + (blockIdx.y * BY + threadIdx.y) * RY;
     if (ys >= a.row_end) return;
     const int ye = min(ys + RY, a.row_end);
     const float c[5] = {a.fparam[0], a.fparam[1], a.fparam[2], a.fparam[3], a.fparam[4]};
-    const size_t sb = (size_t)a.src_row_begin, db = (size_t)a.dst_row_begin;
     const int cx = (blockIdx.x * 32 + lane) * 4;
     const int cxl = min(cx, W - 4);
     const int base = blockIdx.x * 128;
     const bool west_edge = base == 0, east_edge = base + 128 >= W;
     const bool edge_lane = (lane == 0 && !west_edge) || (lane == 31 && !east_edge);
-    // the extra column of an edge lane and the one beyond it (valid only on edge lanes)
     const int xx = lane == 0 ? base - 1 : base + 128;
     const int xo = lane == 0 ? base - 2 : base + 129;
+    const int xoc = clampi(xo, 0, W - 1);
+    const bool wclamp = cx == 0, eclamp = cx + 4 >= W;
+    const float *t0 = (const float *)a.src - (size_t)a.src_row_begin * (size_t)W;
+    const float *p0 = (const float *)a.aux - (size_t)a.src_row_begin * (size_t)W;
+    float *ring = reinterpret_cast<float *>(smem4) + threadIdx.y * (H2_NB * H2_SLOT);
+    // slot offsets: own float4 at 4 + 4*lane; lane 0's outer columns at 3 (xx) and 2 (xo);
+    // lane 31's at 132 (xx) and 133 (xo); the P segment follows at +136
+    const int own = 4 + 4 * lane, oxx = lane == 0 ? 3 : 132, oxo = lane == 0 ? 2 : 133;
 
-    auto load = [&](int y) {
+    auto load = [&](const float *row) {
         Row4 r;
-        const float *row = tin + ((size_t)y - sb) * (size_t)W;
         r.v = __ldg(reinterpret_cast<const float4 *>(row + cxl));
         r.xw = r.xe = r.xo = 0.0f;
         if (edge_lane) {
             r.xw = r.xe = __ldg(row + xx);
-            r.xo = __ldg(row + clampi(xo, 0, W - 1));
+            r.xo = __ldg(row + xoc);
         }
         return r;
     };
-    // one explicit step of the lane's 4 cells and (edge lanes) of its extra cell
-    auto step = [&](const Row4 &N, const Row4 &T, const Row4 &S, float4 P, float Pe, Row4 &out) {
+    auto prow = [&](const float *row, float4 &P, float &Pe) {
+        P = __ldg(reinterpret_cast<const float4 *>(row + cxl));
+        Pe = edge_lane ? __ldg(row + xx) : 0.0f;
+    };
+    auto step = [&](const Row4 &N, const Row4 &T, const Row4 &S, float4 P, float Pe) {
         float Wv = __shfl_up_sync(0xffffffffu, T.v.w, 1);
         float Ev = __shfl_down_sync(0xffffffffu, T.v.x, 1);
         if (lane == 0) Wv = west_edge ? T.v.x : T.xw;
         if (lane == 31) Ev = east_edge ? T.v.w : T.xe;
-        if (cx + 4 >= W) Ev = T.v.w;
-        if (cx == 0) Wv = T.v.x;
+        if (eclamp) Ev = T.v.w;
+        if (wclamp) Wv = T.v.x;
+        Row4 out;
         out.v.x = hs_cell(T.v.x, N.v.x, S.v.x, T.v.y, Wv, P.x, c);
         out.v.y = hs_cell(T.v.y, N.v.y, S.v.y, T.v.z, T.v.x, P.y, c);
         out.v.z = hs_cell(T.v.z, N.v.z, S.v.z, T.v.w, T.v.y, P.z, c);
         out.v.w = hs_cell(T.v.w, N.v.w, S.v.w, Ev, T.v.z, P.w, c);
-        // extra cell: lane 0 at base-1 (E = own column base, W = base-2 clamped);
-        // lane 31 at base+128 (W = own column base+127, E = base+129 clamped)
         const float te = T.xw;
         const float ee = lane == 0 ? T.v.x : (xo > W - 1 ? te : T.xo);
         const float we = lane == 0 ? (xo < 0 ? te : T.xo) : T.v.w;
         out.xw = out.xe = hs_cell(te, N.xw, S.xw, ee, we, Pe, c);
         out.xo = 0.0f;
+        return out;
     };
-    auto prow = [&](int y, float4 &P, float &Pe) {
-        const float *row = pw + ((size_t)y - sb) * (size_t)W;
-        P = __ldg(reinterpret_cast<const float4 *>(row + cxl));
-        Pe = edge_lane ? __ldg(row + xx) : 0.0f;
+    auto rowp = [&](const float *b, int y) { return b + (size_t)clampi(y, 0, H - 1) * (size_t)W; };
+    // ring slot q holds T0(clamp(ys+2+q)) and P(clamp(ys+1+q))
+    auto issue = [&](int q) {
+        float *sl = ring + (q % H2_NB) * H2_SLOT;
+        const float *tr = rowp(t0, ys + 2 + q), *pr = rowp(p0, ys + 1 + q);
+        cp_async16(sl + own, tr + cxl);
+        cp_async16(sl + 136 + own, pr + cxl);
+        if (edge_lane) {
+            cp_async4(sl + oxx, tr + xx);
+            cp_async4(sl + oxo, tr + xoc);
+            cp_async4(sl + 136 + oxx, pr + xx);
+        }
     };
 
-    const int r_lo = max(ys - 1, 0), r_hi = min(ye, H - 1);
-    Row4 t0p = load(max(r_lo - 1, 0)), t0c = load(r_lo);
-    Row4 ua, ub, uc;                 // T1 rows r-2, r-1, r
-    float4 Pb = make_float4(0.f, 0.f, 0.f, 0.f);
-    float Peb = 0.0f;                // P of row r-1 (what T2(r-1) needs)
-    bool have_b = false, have_a = false;
-    float *orow_base = tout + (size_t)cx;
-    for (int r = r_lo; r <= r_hi; ++r) {
-        const Row4 t0n = load(min(r + 1, H - 1));
-        float4 P;
-        float Pe;
-        prow(r, P, Pe);
-        step(t0p, t0c, t0n, P, Pe, uc);     // T1(r)
-        t0p = t0c;
-        t0c = t0n;
-        const int y = r - 1;                 // T2(y) needs T1(clamp(y-1)), T1(y), T1(r)
-        if (have_b && y >= ys && y < ye) {
-            Row4 o;
-            step(have_a ? ua : ub, ub, uc, Pb, Peb, o);
-            if (cx < W) *reinterpret_cast<float4 *>(orow_base + ((size_t)y - db) * (size_t)W) = o.v;
-        }
-        ua = ub;
-        have_a = have_b && (y >= 0);
-        ub = uc;
-        have_b = true;
-        Pb = P;
-        Peb = Pe;
+    const int yb = min(ye, H - 1);                 // rows whose south T1 row is distinct
+    const int nq = yb - ys;                        // loop iterations
+#pragma unroll
+    for (int q = 0; q < H2_NB - 1; ++q) {
+        if (q < nq) issue(q);
+        cp_async_commit();
     }
-    // the bottom row of the image: its south T1 neighbour is itself
-    if (ye == H && H - 1 >= ys) {
-        Row4 o;
-        step(have_a ? ua : ub, ub, ub, Pb, Peb, o);
-        if (cx < W) *reinterpret_cast<float4 *>(orow_base + ((size_t)(H - 1) - db) * (size_t)W) = o.v;
+    // prologue: T1 of rows clamp(ys-1) (ua) and ys (ub)
+    const bool top = ys == 0;
+    Row4 tm2 = load(rowp(t0, ys - 2)), tm1 = load(rowp(t0, ys - 1));
+    Row4 tc0 = load(rowp(t0, ys)), tc1 = load(rowp(t0, ys + 1));
+    float4 Pa, Pc;
+    float Pea, Pec;
+    prow(rowp(p0, ys - 1), Pa, Pea);
+    prow(rowp(p0, ys), Pc, Pec);
+    Row4 ua = top ? step(tc0, tc0, tc1, Pc, Pec) : step(tm2, tm1, tc0, Pa, Pea);
+    Row4 ub = step(tm1, tc0, tc1, Pc, Pec);
+    float *orow = (float *)a.dst + (size_t)cx + ((size_t)ys - (size_t)a.dst_row_begin) * (size_t)W;
+    for (int q = 0; q < nq; ++q) {
+        if (q + H2_NB - 1 < nq) issue(q + H2_NB - 1);
+        cp_async_commit();
+        cp_async_wait<H2_NB - 1>();                // slot q has landed (this lane's copies)
+        const float *sl = ring + (q % H2_NB) * H2_SLOT;
+        Row4 tc2;
+        tc2.v = *reinterpret_cast<const float4 *>(sl + own);
+        float4 Pn = *reinterpret_cast<const float4 *>(sl + 136 + own);
+        float Pen = 0.0f;
+        tc2.xw = tc2.xe = tc2.xo = 0.0f;
+        if (edge_lane) {
+            tc2.xw = tc2.xe = sl[oxx];
+            tc2.xo = sl[oxo];
+            Pen = sl[136 + oxx];
+        }
+        const Row4 uc = step(tc0, tc1, tc2, Pn, Pen);   // T1(y+1), y = ys + q
+        const Row4 o = step(ua, ub, uc, Pc, Pec);       // T2(y)
+        if (cx < W) *reinterpret_cast<float4 *>(orow) = o.v;
+        orow += W;
+        ua = ub;
+        ub = uc;
+        tc0 = tc1;
+        tc1 = tc2;
+        Pc = Pn;
+        Pec = Pen;
+    }
+    cp_async_wait<0>();
+    if (ye == H) {                                 // bottom image row: its south T1 row is itself
+        const Row4 o = step(ua, ub, ub, Pc, Pec);
+        if (cx < W) *reinterpret_cast<float4 *>(orow) = o.v;
     }
 }
 
 // T = 256 threads (32 x 8 warps): 128 columns x 8 strips of 16 rows per CTA; 2 steps per launch.
-extern "C" __global__ void __launch_bounds__(256) orion_hotspot2_f32_256(orion_kargs a) { ORION_PROBE(a); hotspot2_body<8, 16>(a); }
+extern "C" __global__ void __launch_bounds__(256) orion_hotspot2_f32_256(orion_kargs a)
+{
+    ORION_PROBE(a);
+    hotspot2_body<8, 16>(a);
+}

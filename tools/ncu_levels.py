@@ -33,7 +33,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def run(kernel, W, H, threads="0"):
     out = os.path.join(ROOT, "gpurun_out", f"levels_{kernel}.csv")
-    cmd = ["ncu", "--clock-control", "none", "--csv", "--metrics", ",".join(METRICS), "-k", "regex:orion_",
+    cmd = ["ncu", "--clock-control", "none", "--nvtx", "--nvtx-include", "measure/", "--csv", "--metrics", ",".join(METRICS), "-k", "regex:orion_",
            "--log-file", out, sys.executable, os.path.join(ROOT, "tools", "ncu_one.py"), kernel, "all", W, H, threads]
     subprocess.run(cmd, check=True)
 

@@ -19,6 +19,6 @@ for spec in "nlm_f4 -1 2048 2048 nlm_box3" "knn_f4 orig 2048 2048 knn" "nlm_f4_r
             "hotspot_f32 3 8192 8192 hotspot_f32" "hotspot2_f32 2 8192 8192 hotspot2" "srad_f32 2 8192 8192 srad4" \
             "nlm_f4_w8 -1 2048 2048 nlm_box256"; do
   set -- $spec
-  timeout 600 ncu --set full --clock-control none --import-source on -k regex:orion_$5 -c 1 -f -o $OUT/prof_$1 \
+  timeout 600 ncu --set full --clock-control none --import-source on --nvtx --nvtx-include "measure/" -k regex:orion_$5 -c 1 -f -o $OUT/prof_$1 \
       python tools/ncu_one.py $1 $2 $3 $4 > $OUT/ncu_$1.log 2>&1
 done
