@@ -185,10 +185,30 @@ extern "C" __global__ void __launch_bounds__(1024) orion_srad_stats(const float 
 // and lane 31 only supplies the coefficient lane 30's last cell needs as c_E (31V output
 // columns per warp: 3 % of the arithmetic instead of a divergent extra cell).  It walks a strip
 // of rows top to bottom with J rows y .. y+2 and the coefficient row y in registers, the next
-// two rows in flight: every J row is read once per strip, every coefficient computed once.
+// three rows in flight through a cp.async ring in shared memory (4 slots per warp, 16.9 KB
+// per CTA): every J row is read once per strip, every coefficient computed once.
 // W / E neighbours come by shuffle; lane 0 fetches column x0-1, lane 31 column x0+32V.
 // CTA = 8 warps over a 124 x 128 tile: V = 4 -> 8 strips of 16 rows; V = 1 -> 4 column
 // groups of 31 x 2 strips of 64 rows.
+namespace {
+constexpr int SRAD_NB = 4;      // ring slots per warp
+constexpr int SRAD_SLOT = 132;  // floats per slot: 32 lanes x up to 4 columns + 2 outer columns (+pad)
+}  // namespace
+
+__device__ __forceinline__ void srad_cp16(float *sdst, const float *gsrc)
+{
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+                 "l"(gsrc));
+}
+__device__ __forceinline__ void srad_cp4(float *sdst, const float *gsrc)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+                 "l"(gsrc));
+}
+__device__ __forceinline__ void srad_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void srad_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
 namespace {
 template <int V>
 struct SRow {
@@ -258,32 +278,62 @@ __device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys,
         }
     };
 
-    // rows are fetched through a pointer that stops at the last image row (clamp to edge)
-    int rn = ys + 3;                                            // next row to fetch
-    const float *pn = J + (size_t)min(rn, H - 1) * (size_t)W;
-    auto fetch = [&]() {
-        const SRow<V> r = load(pn);
+    // rows y+2, y+3, ... stream through the warp's ring of SRAD_NB slots in shared memory
+    // (cp.async, SRAD_NB-1 rows in flight without holding registers); slot q holds
+    // J(clamp(ys+2+q)).  Each lane reads back exactly the words it copied.
+    extern __shared__ float4 srad_ring4[];
+    float *ring = reinterpret_cast<float *>(srad_ring4) + threadIdx.y * (SRAD_NB * SRAD_SLOT);
+    const int own = V * lane, oxa = 32 * V + (lane == 0 ? 0 : 1);
+    const float *pn = J + (size_t)min(ys + 2, H - 1) * (size_t)W;
+    int rn = ys + 2;                                            // row pn points at (unclamped)
+    auto issue = [&](int q) {
+        float *sl = ring + (q % SRAD_NB) * SRAD_SLOT;
+        if constexpr (V == 4)
+            srad_cp16(sl + own, pn + cxl);
+        else
+            srad_cp4(sl + own, pn + cxl);
+        if (lane == 0 || lane == 31) srad_cp4(sl + oxa, pn + xa);
         if (rn < H - 1) pn += W;
         ++rn;
+    };
+    auto slot_row = [&](int q) {
+        const float *sl = ring + (q % SRAD_NB) * SRAD_SLOT;
+        SRow<V> r;
+        if constexpr (V == 4) {
+            const float4 t = *reinterpret_cast<const float4 *>(sl + own);
+            r.v[0] = t.x;
+            r.v[1] = t.y;
+            r.v[2] = t.z;
+            r.v[3] = t.w;
+        } else {
+            r.v[0] = sl[own];
+        }
+        r.xa = (lane == 0 || lane == 31) ? sl[oxa] : 0.0f;
         return r;
     };
+    const int yb = min(ye, H - 1);                              // rows with a distinct south row
+    const int nq = yb - ys;
+#pragma unroll
+    for (int q = 0; q < SRAD_NB - 1; ++q) {
+        if (q < nq) issue(q);
+        srad_commit();
+    }
     SRow<V> j0 = load(J + (size_t)ys * (size_t)W);
     SRow<V> j1 = load(J + (size_t)min(ys + 1, H - 1) * (size_t)W);
-    SRow<V> j2 = load(J + (size_t)min(ys + 2, H - 1) * (size_t)W);
-    SRow<V> j3 = fetch();
     CRow<V> c0 = coeff_row(load(J + (size_t)max(ys - 1, 0) * (size_t)W), j0, j1);
-    const int yb = min(ye, H - 1);                              // rows with a distinct south row
-#pragma unroll 4
-    for (int y = ys; y < yb; ++y) {
-        const SRow<V> j4 = fetch();                             // two rows in flight
+#pragma unroll 1
+    for (int q = 0; q < nq; ++q) {
+        if (q + SRAD_NB - 1 < nq) issue(q + SRAD_NB - 1);
+        srad_commit();
+        srad_wait<SRAD_NB - 1>();
+        const SRow<V> j2 = slot_row(q);                         // J(y+2), y = ys + q
         const CRow<V> c1 = coeff_row(j0, j1, j2);               // c of row y+1
-        update_row(y, j0, c0, c1);
+        update_row(ys + q, j0, c0, c1);
         j0 = j1;
         j1 = j2;
-        j2 = j3;
-        j3 = j4;
         c0 = c1;
     }
+    srad_wait<0>();
     if (ye == H) update_row(H - 1, j0, c0, c0);               // last image row: c_S = own c
 }
 

@@ -72,8 +72,9 @@ static const KernelDef kKernels[] = {
     {"hotspot2_f32", 256, "orion_hotspot2_f32_256", "hotspot", 32, 8, 128, 128, 2, K_STENCIL, 0, 8 * 4 * 272 * 4, 4, 2},
     // srad: J tile (32+3)^2 + coefficient tile (32+1)^2 floats; reads 2 rows below the tile
     {"srad_f32_tile", 256, "orion_srad_f32_256", "srad", 32, 8, 32, 32, 2, K_SRAD, 0, (35 * 35 + 33 * 33) * 4},
-    // srad, register-sliding: 124 x 128 tile; float4 lanes (width % 4 == 0) or scalar lanes
-    {"srad_f32", 256, "orion_srad4_f32_256", "srad", 32, 8, 124, 128, 2, K_SRAD, 0, 0},
+    // srad, register-sliding: 124 x 128 tile; float4 lanes (width % 4 == 0) or scalar lanes;
+    // rows stream through a 4-slot cp.async ring per warp (8 x 4 x 132 floats)
+    {"srad_f32", 256, "orion_srad4_f32_256", "srad", 32, 8, 124, 128, 2, K_SRAD, 0, 8 * 4 * 132 * 4},
 };
 
 const KernelDef *find_kernel(const char *id, int threads)
