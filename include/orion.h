@@ -207,6 +207,12 @@ typedef struct {
     float slowdown_tol;           /* Fig. 9 "Slowdown > .02?"                              */
     float worse_eps;              /* Fig. 9 "Worse runtime?" margin (paper: 0)                      */
     int expected_iterations;      /* canTune (Fig. 8 line 05): 0 = unknown (assume enough)          */
+    int async_timing;             /* 0 (default, the paper's P:L653 loop): an exploring iteration
+                                     synchronises on its event pair before returning.  1: it only
+                                     records the pair; later iterations poll it (cuEventQuery) and,
+                                     until it has completed, repeat the level being measured without
+                                     timing it -- no host synchronisation anywhere, the measured
+                                     launch runs back to back with its neighbours                   */
 } orion_tuner_cfg;
 
 orion_status orion_tuner_default_cfg(orion_tuner_cfg *cfg);
@@ -224,7 +230,8 @@ typedef struct {
     int level_idx;        /* variant launched this iteration                                 */
     int phase;            /* 0 = exploring (timed, synchronised), 1 = final (no host sync)   */
     int final_level_idx;  /* -1 until the final kernel is set                                */
-    float ms;             /* measured kernel ms while exploring, else -1                     */
+    float ms;             /* measured kernel ms of this iteration while exploring, else -1;
+                             async_timing: the measurement that completed during this call    */
 } orion_step_report;
 
 /* One application iteration under Fig. 9 (P:L605-P:L643, P:L651-P:L653, P:L687-P:L689):

@@ -22,7 +22,7 @@ namespace orion {
     X(cuEventRecord) X(cuEventSynchronize) X(cuEventElapsedTime) X(cuMemcpyHtoDAsync)             \
     X(cuMemcpyDtoHAsync) X(cuStreamSynchronize) X(cuGetErrorString) X(cuGetErrorName)            \
     X(cuMemAlloc) X(cuMemFree) X(cuStreamCreate) X(cuStreamDestroy) X(cuStreamWaitEvent)          \
-    X(cuMemsetD32) X(cuMemcpyDtoH) X(cuCtxSynchronize)
+    X(cuMemsetD32) X(cuMemcpyDtoH) X(cuCtxSynchronize) X(cuEventQuery)
 
 struct Driver {
 #define ORION_DECL(f) decltype(&::f) f = nullptr;

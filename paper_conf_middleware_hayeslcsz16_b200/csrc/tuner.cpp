@@ -139,6 +139,7 @@ struct Fig9 {
 orion_status check_cfg(const orion_tuner_cfg *c)
 {
     if (!c || c->samples_per_level < 1 || c->slowdown_tol < 0.0f || c->worse_eps < 0.0f ||
+        (c->async_timing != 0 && c->async_timing != 1) ||
         (c->select_mode != ORION_SELECT_FASTEST && c->select_mode != ORION_SELECT_LOWEST_WITHIN_TOL))
         return fail(ORION_E_INVALID, "bad tuner cfg");
     return ORION_OK;
@@ -161,6 +162,10 @@ struct orion_tuner {
     int pending_level = -1;      // level being sampled (samples_per_level > 1)
     int samples = 0;
     float sample_best = 0.0f;
+    // async_timing: the one measured launch whose event pair has not been read yet
+    bool inflight = false;
+    int inflight_level = -1;
+    double inflight_work = 0.0;
 };
 
 extern "C" {
@@ -175,6 +180,7 @@ orion_status orion_tuner_default_cfg(orion_tuner_cfg *c)
     c->slowdown_tol = 0.02f;
     c->worse_eps = 0.0f;
     c->expected_iterations = 0;
+    c->async_timing = 0;
     return ORION_OK;
 }
 
@@ -232,10 +238,59 @@ void orion_tuner_destroy(orion_tuner *t)
     delete t;
 }
 
+// Feed one completed measurement (ms of a launch over `work` output elements) to Fig. 9,
+// through the samples_per_level filter (the fastest of the samples is observed).
+static void feed_sample(orion_tuner *t, int lvl, float ms, double work)
+{
+    Fig9 &f = t->f;
+    // work-normalised runtime: ns per output element, so iterations of
+    // different sizes -- the bands of a split frame -- compare fairly
+    const float per = work > 0 ? (float)(ms * 1e6 / work) : ms;
+    const float m = (t->samples == 0) ? per : std::min(t->sample_best, per);
+    t->samples += 1;
+    t->sample_best = m;
+    if (t->samples >= f.cfg.samples_per_level) {
+        f.observe(lvl, m);            // best of the samples feeds Fig. 9
+        t->pending_level = -1;
+        t->samples = 0;
+    } else {
+        t->pending_level = lvl;
+    }
+}
+
 orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, orion_step_report *out)
 {
     if (!t || !a) return fail(ORION_E_INVALID, "orion_tune_step: NULL");
     Fig9 &f = t->f;
+    CUstream s = (CUstream)stream;
+    const Driver &D = drv();
+    const double work = (double)(a->row_end - a->row_begin) * (double)a->width;
+    float ms = -1.0f;
+    auto report = [&](int lvl, int phase) {
+        if (out) {
+            out->iteration = f.iter;
+            out->level_idx = lvl;
+            out->phase = phase;
+            out->final_level_idx = f.final_idx;
+            out->ms = ms;
+        }
+        f.iter += 1;
+        return ORION_OK;
+    };
+    if (t->inflight) {                    // async_timing: is the measured launch done?
+        const CUresult q = D.cuEventQuery(t->e1);
+        if (q == CUDA_SUCCESS) {
+            ORION_CU(D.cuEventElapsedTime(&ms, t->e0, t->e1));
+            t->inflight = false;
+            feed_sample(t, t->inflight_level, ms, t->inflight_work);
+        } else if (q == CUDA_ERROR_NOT_READY) {
+            // not yet: run the level being measured again, untimed (never block the host)
+            ORION_TRY(orion_launch(t->v, t->inflight_level, a, stream));
+            return report(t->inflight_level, 0);
+        } else {
+            ORION_CU(q);
+        }
+    }
     bool measure = false;
     int lvl;
     if (t->pending_level >= 0) {          // still sampling a level (samples_per_level > 1)
@@ -244,41 +299,23 @@ orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, 
     } else {
         lvl = f.choose(&measure);
     }
-    CUstream s = (CUstream)stream;
-    const Driver &D = drv();
-    float ms = -1.0f;
     if (measure) {
         ORION_CU(D.cuEventRecord(t->e0, s));
         ORION_TRY(orion_launch(t->v, lvl, a, stream));
         ORION_CU(D.cuEventRecord(t->e1, s));
-        ORION_CU(D.cuEventSynchronize(t->e1));
-        ORION_CU(D.cuEventElapsedTime(&ms, t->e0, t->e1));
-        // work-normalised runtime: ns per output element, so iterations of
-        // different sizes -- the bands of a split frame -- compare fairly
-        const double work = (double)(a->row_end - a->row_begin) * (double)a->width;
-        const float per = work > 0 ? (float)(ms * 1e6 / work) : ms;
-        const float m = (t->samples == 0) ? per : std::min(t->sample_best, per);
-        t->samples += 1;
-        t->sample_best = m;
-        if (t->samples >= f.cfg.samples_per_level) {
-            f.observe(lvl, m);            // best of the samples feeds Fig. 9
-            t->pending_level = -1;
-            t->samples = 0;
+        if (f.cfg.async_timing) {
+            t->inflight = true;
+            t->inflight_level = lvl;
+            t->inflight_work = work;
         } else {
-            t->pending_level = lvl;
+            ORION_CU(D.cuEventSynchronize(t->e1));
+            ORION_CU(D.cuEventElapsedTime(&ms, t->e0, t->e1));
+            feed_sample(t, lvl, ms, work);
         }
     } else {
         ORION_TRY(orion_launch(t->v, lvl, a, stream));
     }
-    if (out) {
-        out->iteration = f.iter;
-        out->level_idx = lvl;
-        out->phase = measure ? 0 : 1;
-        out->final_level_idx = f.final_idx;
-        out->ms = ms;
-    }
-    f.iter += 1;
-    return ORION_OK;
+    return report(lvl, measure ? 0 : 1);
 }
 
 orion_status orion_tune_split(orion_tuner *t, const orion_args *a, int bands, void *stream, orion_step_report *reports)

@@ -84,7 +84,7 @@ class TunerCfg(ctypes.Structure):
     _fields_ = [("maxlive_threshold", ctypes.c_int), ("samples_per_level", ctypes.c_int),
                 ("select_mode", ctypes.c_int), ("allow_direction_switch", ctypes.c_int),
                 ("slowdown_tol", ctypes.c_float), ("worse_eps", ctypes.c_float),
-                ("expected_iterations", ctypes.c_int)]
+                ("expected_iterations", ctypes.c_int), ("async_timing", ctypes.c_int)]
 
 
 class StepReport(ctypes.Structure):

@@ -14,7 +14,7 @@ python bench.py --workload c4 --steps 20 --warmup 15 --rounds 3 --cpu-seconds 5 
 python bench.py --workload c5 --steps 10 --warmup 5 > $OUT/bench_c5.log 2>&1
 python bench.py --workload srad --steps 100 --warmup 12 --cpu-seconds 5 > $OUT/bench_srad.log 2>&1
 [ -n "$SKIP_NCU" ] && exit 0
-ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
+ncu --metrics gpu__time_duration.sum --clock-control none --nvtx --nvtx-include "timed/" --csv --log-file $OUT/launches.csv \
     python bench.py --steps 20 --warmup 5 --rounds 3 --no-cpu-baseline --no-carveout-axis > $OUT/bench_under_ncu.log 2>&1
 for spec in "nlm_f4 -1 2048 2048 nlm_box3" "knn_f4 orig 2048 2048 knn" "nlm_f4_regheavy orig 4096 4096 nlm_regheavy" \
             "hotspot_f32 3 8192 8192 hotspot_f32" "hotspot2_f32 2 8192 8192 hotspot2" "srad_f32 2 8192 8192 srad4" \
