@@ -190,7 +190,9 @@ orion_status orion_launch(orion_variants *v, int level_idx, const orion_args *a,
 /* Exhaustive occupancy sweep (Fig. 11's Orion-Min / Orion-Max methodology, P:L747-P:L755):
  * `rounds` rounds, each launching every level once in round-robin order (interleaving
  * cancels clock drift), each launch timed with a CUDA event pair on `stream`; writes the
- * median ms per level into ms_median[n levels].  Synchronises the stream. */
+ * median ms per level into ms_median[n levels].  A level whose (timed) warm-up launch is
+ * shorter than 0.2 ms is timed over a batch of up to 64 back-to-back launches per sample and
+ * reported per launch.  Synchronises the stream. */
 orion_status orion_sweep(orion_variants *v, const orion_args *a, void *stream, int rounds, float *ms_median);
 
 /* ---- runtime adaptation (question 2) ------------------------------------------------------ */

@@ -282,8 +282,6 @@ orion_status orion_sweep(orion_variants *v, const orion_args *a, void *stream, i
     const Driver &D = drv();
     const int n = (int)v->vars.size();
     CUstream s = (CUstream)stream;
-    // warm every variant once (module lazy loading, instruction cache)
-    for (int i = 0; i < n; ++i) ORION_TRY(launch_fn(*v->def, v->vars[i].fn, v->vars[i].dyn_bytes, k, s));
     std::vector<CUevent> ev((size_t)2 * n * rounds, nullptr);
     orion_status st = ORION_OK;
     for (auto &e : ev)
@@ -291,13 +289,30 @@ orion_status orion_sweep(orion_variants *v, const orion_args *a, void *stream, i
             st = fail(ORION_E_CUDA, "cuEventCreate");
             break;
         }
+    // warm every variant once (module lazy loading, instruction cache) and time that launch:
+    // a level whose launch is shorter than kMinSampleMs is timed over a batch of back-to-back
+    // launches per sample (per-launch ms = batch ms / batch), so event overhead and launch
+    // jitter do not decide between microsecond-scale levels
+    constexpr float kMinSampleMs = 0.2f;
+    std::vector<int> batch((size_t)n, 1);
+    for (int i = 0; i < n && st == ORION_OK; ++i) {
+        float w = 0.0f;
+        if (D.cuEventRecord(ev[0], s) != CUDA_SUCCESS) st = fail(ORION_E_CUDA, "cuEventRecord");
+        if (st == ORION_OK) st = launch_fn(*v->def, v->vars[i].fn, v->vars[i].dyn_bytes, k, s);
+        if (st == ORION_OK && (D.cuEventRecord(ev[1], s) != CUDA_SUCCESS || D.cuEventSynchronize(ev[1]) != CUDA_SUCCESS ||
+                               D.cuEventElapsedTime(&w, ev[0], ev[1]) != CUDA_SUCCESS))
+            st = fail(ORION_E_CUDA, "sweep warm-up timing");
+        if (st == ORION_OK && w > 0.0f && w < kMinSampleMs)
+            batch[(size_t)i] = std::min(64, (int)std::ceil(kMinSampleMs / w));
+    }
     if (st == ORION_OK) {
         for (int r = 0; r < rounds && st == ORION_OK; ++r)
             for (int q = 0; q < n && st == ORION_OK; ++q) {
                 const int i = (q + r) % n;   // rotate the start so no level is always first
                 const size_t e = (size_t)2 * (r * n + i);
                 if (D.cuEventRecord(ev[e], s) != CUDA_SUCCESS) st = fail(ORION_E_CUDA, "cuEventRecord");
-                if (st == ORION_OK) st = launch_fn(*v->def, v->vars[i].fn, v->vars[i].dyn_bytes, k, s);
+                for (int b = 0; b < batch[(size_t)i] && st == ORION_OK; ++b)
+                    st = launch_fn(*v->def, v->vars[i].fn, v->vars[i].dyn_bytes, k, s);
                 if (st == ORION_OK && D.cuEventRecord(ev[e + 1], s) != CUDA_SUCCESS)
                     st = fail(ORION_E_CUDA, "cuEventRecord");
             }
@@ -313,7 +328,8 @@ orion_status orion_sweep(orion_variants *v, const orion_args *a, void *stream, i
                     }
                 }
                 std::sort(t.begin(), t.end());
-                ms_median[i] = (rounds % 2) ? t[rounds / 2] : 0.5f * (t[rounds / 2 - 1] + t[rounds / 2]);
+                ms_median[i] = ((rounds % 2) ? t[rounds / 2] : 0.5f * (t[rounds / 2 - 1] + t[rounds / 2])) /
+                               (float)batch[(size_t)i];
             }
         }
     }
