@@ -318,17 +318,33 @@ __device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys,
         if (q < nq) issue(q);
         srad_commit();
     }
-    SRow<V> j0 = load(J + (size_t)ys * (size_t)W);
-    SRow<V> j1 = load(J + (size_t)min(ys + 1, H - 1) * (size_t)W);
-    CRow<V> c0 = coeff_row(load(J + (size_t)max(ys - 1, 0) * (size_t)W), j0, j1);
-#pragma unroll 1
-    for (int q = 0; q < nq; ++q) {
+    SRow<V> j0 = load(J + (size_t)ys * (size_t)W), j1 = load(J + (size_t)min(ys + 1, H - 1) * (size_t)W), j2;
+    CRow<V> c0 = coeff_row(load(J + (size_t)max(ys - 1, 0) * (size_t)W), j0, j1), c1;
+    // one output row y = ys + q: N = J(y), T = J(y+1), S = J(y+2) (from the ring, written into
+    // S), cT = c(y), cS = c(y+1) (written).  The row registers rotate through three variables and
+    // the coefficient rows through two, so six consecutive rows are written out with permuted
+    // arguments -- no register moves between rows.
+    auto row = [&](int q, const SRow<V> &N, const SRow<V> &T, SRow<V> &S, const CRow<V> &cT, CRow<V> &cS) {
         if (q + SRAD_NB - 1 < nq) issue(q + SRAD_NB - 1);
         srad_commit();
         srad_wait<SRAD_NB - 1>();
-        const SRow<V> j2 = slot_row(q);                         // J(y+2), y = ys + q
-        const CRow<V> c1 = coeff_row(j0, j1, j2);               // c of row y+1
-        update_row(ys + q, j0, c0, c1);
+        S = slot_row(q);
+        cS = coeff_row(N, T, S);
+        update_row(ys + q, N, cT, cS);
+    };
+    int q = 0;
+#pragma unroll 1
+    for (; q + 6 <= nq; q += 6) {
+        row(q, j0, j1, j2, c0, c1);
+        row(q + 1, j1, j2, j0, c1, c0);
+        row(q + 2, j2, j0, j1, c0, c1);
+        row(q + 3, j0, j1, j2, c1, c0);
+        row(q + 4, j1, j2, j0, c0, c1);
+        row(q + 5, j2, j0, j1, c1, c0);
+    }
+#pragma unroll 1
+    for (; q < nq; ++q) {                                       // the last < 6 rows
+        row(q, j0, j1, j2, c0, c1);
         j0 = j1;
         j1 = j2;
         c0 = c1;
