@@ -228,32 +228,58 @@ __device__ __forceinline__ void hotspot2_body(const orion_kargs &a)
     Row4 ua = top ? step(tc0, tc0, tc1, Pc, Pec) : step(tm2, tm1, tc0, Pa, Pea);
     Row4 ub = step(tm1, tc0, tc1, Pc, Pec);
     float *orow = (float *)a.dst + (size_t)cx + ((size_t)ys - (size_t)a.dst_row_begin) * (size_t)W;
-    for (int q = 0; q < nq; ++q) {
+    // one output row y = ys + q: T0 rows y, y+1 (A, B) and y+2 (C, from the ring), T1 rows
+    // clamp(y-1), y (X, Y) and y+1 (Z, computed), P rows y (Pc) and y+1 (Pn, from the ring).
+    // T0 and T1 rows rotate through three variables and P rows through two, so six consecutive
+    // rows are written out with permuted arguments -- no register moves between rows.
+    struct PRow {
+        float4 v;
+        float e;
+    };
+    PRow pa{Pc, Pec}, pb;
+    Row4 tcx;
+    auto row = [&](int q, const Row4 &A, const Row4 &B, Row4 &C, const Row4 &X, const Row4 &Y, Row4 &Z,
+                   const PRow &Pcur, PRow &Pnext) {
         if (q + H2_NB - 1 < nq) issue(q + H2_NB - 1);
         cp_async_commit();
         cp_async_wait<H2_NB - 1>();                // slot q has landed (this lane's copies)
         const float *sl = ring + (q % H2_NB) * H2_SLOT;
-        Row4 tc2;
-        tc2.v = *reinterpret_cast<const float4 *>(sl + own);
-        float4 Pn = *reinterpret_cast<const float4 *>(sl + 136 + own);
-        float Pen = 0.0f;
-        tc2.xw = tc2.xe = tc2.xo = 0.0f;
+        C.v = *reinterpret_cast<const float4 *>(sl + own);
+        Pnext.v = *reinterpret_cast<const float4 *>(sl + 136 + own);
+        Pnext.e = 0.0f;
+        C.xw = C.xe = C.xo = 0.0f;
         if (edge_lane) {
-            tc2.xw = tc2.xe = sl[oxx];
-            tc2.xo = sl[oxo];
-            Pen = sl[136 + oxx];
+            C.xw = C.xe = sl[oxx];
+            C.xo = sl[oxo];
+            Pnext.e = sl[136 + oxx];
         }
-        const Row4 uc = step(tc0, tc1, tc2, Pn, Pen);   // T1(y+1), y = ys + q
-        const Row4 o = step(ua, ub, uc, Pc, Pec);       // T2(y)
+        Z = step(A, B, C, Pnext.v, Pnext.e);       // T1(y+1)
+        const Row4 o = step(X, Y, Z, Pcur.v, Pcur.e);   // T2(y)
         if (cx < W) *reinterpret_cast<float4 *>(orow) = o.v;
         orow += W;
-        ua = ub;
-        ub = uc;
-        tc0 = tc1;
-        tc1 = tc2;
-        Pc = Pn;
-        Pec = Pen;
+    };
+    Row4 uz;
+    int q = 0;
+#pragma unroll 1
+    for (; q + 6 <= nq; q += 6) {
+        row(q, tc0, tc1, tcx, ua, ub, uz, pa, pb);
+        row(q + 1, tc1, tcx, tc0, ub, uz, ua, pb, pa);
+        row(q + 2, tcx, tc0, tc1, uz, ua, ub, pa, pb);
+        row(q + 3, tc0, tc1, tcx, ua, ub, uz, pb, pa);
+        row(q + 4, tc1, tcx, tc0, ub, uz, ua, pa, pb);
+        row(q + 5, tcx, tc0, tc1, uz, ua, ub, pb, pa);
     }
+#pragma unroll 1
+    for (; q < nq; ++q) {                          // the last < 6 rows
+        row(q, tc0, tc1, tcx, ua, ub, uz, pa, pb);
+        tc0 = tc1;
+        tc1 = tcx;
+        ua = ub;
+        ub = uz;
+        pa = pb;
+    }
+    Pc = pa.v;
+    Pec = pa.e;
     cp_async_wait<0>();
     if (ye == H) {                                 // bottom image row: its south T1 row is itself
         const Row4 o = step(ua, ub, ub, Pc, Pec);
