@@ -595,6 +595,9 @@ def run_ours(args):
                                                           - len(explore_ms)) * ms_step) / (args.warmup + args.steps)),
                   "speedup_max_vs_nvcc": ms[orig] / ms[best], "speedup_min_vs_nvcc": ms[orig] / ms[worst]},
         "vs_maxocc": ms[kmax] / t_final,
+        "paper_context": {"note": "context only, not a target: the paper's best speedup over nvcc (particles, "
+                                  "Table 3) on GTX680 / Tesla C2075; imageDenoising 1.08-1.12, hotspot 1.12-1.18",
+                          "paper_max_speedup_vs_nvcc": 1.61, "this_run_vs_nvcc": ms[orig] / t_final},
         "vs_nvcc_default": ms[orig] / t_final,
         "build_seconds": round(t_build, 2),
         "realise": "min_carveout" if realise == O.REALISE_MIN_CARVEOUT else "max_smem",
