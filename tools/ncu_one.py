@@ -1,8 +1,8 @@
 """Launch ONE kernel variant once on a synthetic frame (for ncu --set full captures).
 
 usage: python tools/ncu_one.py KERNEL LEVEL W H [THREADS] [REPEAT]
-  LEVEL = index into the level list (-1 = max occupancy, 'orig' = natural build, 'all' = every
-  level once, in order).  Levels are realised as bench.py realises them (MIN_CARVEOUT).
+  LEVEL = index into the level list (-1 = max occupancy, 'orig' = natural build, 'best' = the
+  sweep's fastest level, 'all' = every level once, in order).  Levels are realised as bench.py realises them (MIN_CARVEOUT).
 """
 import os
 import sys
@@ -19,7 +19,7 @@ torch.cuda.set_device(0)
 sp = torch.cuda.current_stream().cuda_stream
 mode = O.REALISE_MAX_SMEM if os.environ.get("ORION_REALISE") == "max" else O.REALISE_MIN_CARVEOUT
 v, res = O.build_all_levels(0, kernel, threads, mode=mode)
-if lev == "all":
+if lev in ("all", "best"):
     li = None
 elif lev == "orig":
     li = max((i for i, l in enumerate(v.planned) if l.reg_cap == 0), key=lambda i: v.planned[i].ctas_per_sm)
@@ -45,6 +45,9 @@ else:
     O.generate_rgba(0, a.data_ptr(), W, H, sigma=0.13, stream=sp)
     args = O.denoise_args(kernel, a.data_ptr(), b.data_ptr(), W, H)
 torch.cuda.synchronize()
+if lev == "best":   # the exhaustive sweep's fastest level (what the tuner should settle on)
+    ms = v.sweep(args, sp, rounds=5)
+    li = min(range(len(ms)), key=lambda i: ms[i])
 torch.cuda.nvtx.range_push("measure")   # ncu --nvtx --nvtx-include "measure/": skips the build's probe launches
 for i in (range(len(v)) if li is None else [li]):
     for _ in range(repeat):
