@@ -306,6 +306,21 @@ orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, 
 orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final);
 void orion_tuner_destroy(orion_tuner *t);
 
+/* ---- CUDA graph replay of settled iterations (launch-bound loops) ------------------------- */
+
+typedef struct orion_graph orion_graph;   /* opaque, library-owned (a CUgraphExec) */
+
+/* Once Fig. 9 has set the final kernel ("run final kernel" every later iteration), the
+ * iterations are plain launches of one variant: capture `n` of them -- args[i] for iteration i,
+ * e.g. a ring of frames; device pointers, geometry as for orion_launch -- into a CUDA graph on
+ * a library stream.  Each orion_graph_launch then replays the n launches on `stream` with one
+ * host call (no per-launch host work: what bounds small frames such as C1's 64x64).  The
+ * tuner's iteration counter advances by n per replay.  ORION_E_STATE while the tuner is still
+ * exploring; ORION_E_INVALID on n < 1 or bad args. */
+orion_status orion_tuner_capture(orion_tuner *t, const orion_args *args, int n, orion_graph **out);
+orion_status orion_graph_launch(orion_graph *g, void *stream);
+void orion_graph_destroy(orion_graph *g);
+
 /* Host-only replay of Fig. 8 + Fig. 9 on a synthetic per-level runtime table (no GPU):
  * levels[n] as from orion_levels, natural_regs = MAXLIVE proxy, ms_of_level[n] = the runtime
  * each level would take; runs `iterations` iterations writing the level index run at each

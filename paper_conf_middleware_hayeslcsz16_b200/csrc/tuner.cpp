@@ -12,6 +12,7 @@
 // LOWEST_WITHIN_TOL mode, the lowest occupancy within slowdown_tol of the best (R-A4).
 #include <algorithm>
 #include <map>
+#include <memory>
 
 #include "orion_internal.h"
 
@@ -558,6 +559,67 @@ orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *
     if (!t) return fail(ORION_E_INVALID, "orion_tuner_final: NULL");
     if (final_level_idx) *final_level_idx = t->f.final_idx;
     if (iterations_to_final) *iterations_to_final = t->f.final_iter;
+    return ORION_OK;
+}
+
+}  // extern "C"
+
+struct orion_graph {
+    orion_tuner *t = nullptr;
+    CUgraph graph = nullptr;
+    CUgraphExec exec = nullptr;
+    int n = 0;
+};
+
+extern "C" {
+
+void orion_graph_destroy(orion_graph *g)
+{
+    if (!g) return;
+    if (drv().ok) {
+        if (g->exec) drv().cuGraphExecDestroy(g->exec);
+        if (g->graph) drv().cuGraphDestroy(g->graph);
+    }
+    delete g;
+}
+
+orion_status orion_tuner_capture(orion_tuner *t, const orion_args *args, int n, orion_graph **out)
+{
+    if (!t || !args || n < 1 || !out) return fail(ORION_E_INVALID, "orion_tuner_capture: bad argument");
+    *out = nullptr;
+    if (t->f.final_idx < 0 || t->inflight) return fail(ORION_E_STATE, "orion_tuner_capture: the tuner is still exploring");
+    ORION_TRY(ensure_context(t->v->device));
+    const Driver &D = drv();
+    CUstream s = nullptr;
+    ORION_CU(D.cuStreamCreate(&s, CU_STREAM_NON_BLOCKING));
+    std::unique_ptr<orion_graph, void (*)(orion_graph *)> g(new orion_graph(), orion_graph_destroy);
+    g->t = t;
+    g->n = n;
+    orion_status st = ORION_OK;
+    if (D.cuStreamBeginCapture(s, CU_STREAM_CAPTURE_MODE_THREAD_LOCAL) != CUDA_SUCCESS)
+        st = fail(ORION_E_CUDA, "cuStreamBeginCapture");
+    const long long before = g_launches.load();
+    for (int i = 0; i < n && st == ORION_OK; ++i) st = orion_launch(t->v, t->f.final_idx, &args[i], s);
+    g_launches.store(before);   // captured, not launched: replays are counted
+    CUgraph graph = nullptr;
+    const CUresult end = D.cuStreamEndCapture(s, &graph);   // always end the capture
+    g->graph = graph;
+    if (st == ORION_OK && end != CUDA_SUCCESS) st = fail(ORION_E_CUDA, "cuStreamEndCapture");
+    if (st == ORION_OK && D.cuGraphInstantiate(&g->exec, g->graph, 0) != CUDA_SUCCESS)
+        st = fail(ORION_E_CUDA, "cuGraphInstantiate");
+    D.cuStreamDestroy(s);
+    if (st != ORION_OK) return st;
+    *out = g.release();
+    return ORION_OK;
+}
+
+orion_status orion_graph_launch(orion_graph *g, void *stream)
+{
+    if (!g || !g->exec) return fail(ORION_E_INVALID, "orion_graph_launch: NULL");
+    ORION_TRY(ensure_context(g->t->v->device));
+    ORION_CU(drv().cuGraphLaunch(g->exec, (CUstream)stream));
+    g_launches.fetch_add(g->n);
+    g->t->f.iter += g->n;
     return ORION_OK;
 }
 

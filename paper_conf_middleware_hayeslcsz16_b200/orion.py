@@ -128,6 +128,8 @@ def lib() -> ctypes.CDLL:
                 "orion_tune_step_host": [V, P(Args), V, V, V, V, P(StepReport), P(ctypes.c_longlong),
                                          P(ctypes.c_longlong)],
                 "orion_tune_split": [V, P(Args), I, V, P(StepReport)],
+                "orion_tuner_capture": [V, P(Args), I, P(V)],
+                "orion_graph_launch": [V, V],
                 "orion_tune_run_host": [V, P(Args), I, V, V, V, P(I), V, P(ctypes.c_longlong),
                                         P(ctypes.c_longlong)],
                 "orion_host_pipe_create": [V, I, I, I, P(V)],
@@ -145,7 +147,8 @@ def lib() -> ctypes.CDLL:
                 f = getattr(L, name)
                 f.argtypes = args
                 f.restype = ctypes.c_int
-            for name in ("orion_variants_destroy", "orion_tuner_destroy", "orion_host_pipe_destroy"):
+            for name in ("orion_variants_destroy", "orion_tuner_destroy", "orion_host_pipe_destroy",
+                         "orion_graph_destroy"):
                 getattr(L, name).argtypes = [V]
                 getattr(L, name).restype = None
             L.orion_status_str.restype = ctypes.c_char_p
@@ -371,6 +374,10 @@ class Tuner:
                                          ctypes.byref(hi), ctypes.byref(ho)), "orion_tune_run_host")
         return hi.value, ho.value
 
+    def capture(self, args_list: list, stream=None) -> "Graph":
+        """orion_tuner_capture: the settled kernel's launches for args_list[i] as one CUDA graph."""
+        return Graph(self, args_list)
+
     def ladder(self):
         d, n = ctypes.c_int(), ctypes.c_int()
         buf = (ctypes.c_int * 64)()
@@ -385,6 +392,31 @@ class Tuner:
     def close(self):
         if getattr(self, "h", None):
             lib().orion_tuner_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Graph:
+    """orion_graph handle: replay n settled iterations with one host call."""
+
+    def __init__(self, tuner: "Tuner", args_list: list):
+        self.tuner = tuner
+        arr = (Args * len(args_list))(*args_list)
+        h = ctypes.c_void_p()
+        _check(lib().orion_tuner_capture(tuner.h, arr, len(args_list), ctypes.byref(h)), "orion_tuner_capture")
+        self.h, self.n = h, len(args_list)
+
+    def launch(self, stream=None):
+        _check(lib().orion_graph_launch(self.h, _s(stream)), "orion_graph_launch")
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().orion_graph_destroy(self.h)
             self.h = None
 
     def __del__(self):

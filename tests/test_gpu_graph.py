@@ -1,0 +1,54 @@
+"""orion_tuner_capture / orion_graph_launch: once Fig. 9 has set the final kernel (PAPER.md
+P:L643), n settled iterations replay as one CUDA graph -- bit-identical to launching them one
+by one, counted as n launches, refused while the tuner is still exploring."""
+import numpy as np
+import pytest
+
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
+
+
+@pytest.fixture(scope="module")
+def knn():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return O.build_all_levels(0, "knn_f4", mode=O.REALISE_MIN_CARVEOUT)[0]
+
+
+def test_graph_replay_matches_direct_launches(knn):
+    W = H = 64
+    n = 6
+    sp = torch.cuda.current_stream().cuda_stream
+    srcs = [torch.from_numpy(synth.noisy_rgba(W, H, seed=10 + f, sigma=0.2)).cuda() for f in range(n)]
+    dsts = [torch.zeros_like(s) for s in srcs]
+    args = [O.denoise_args("knn_f4", srcs[f].data_ptr(), dsts[f].data_ptr(), W, H) for f in range(n)]
+    tuner = O.Tuner(knn)
+    with pytest.raises(O.OrionError) as e:          # still exploring
+        tuner.capture(args)
+    assert e.value.status == -7
+    it = 0
+    while tuner.final()[0] < 0:
+        tuner.step(args[it % n], sp)
+        it += 1
+        assert it < 200
+    final = tuner.final()[0]
+    ref = []
+    for f in range(n):
+        knn.launch(final, args[f], sp)
+    torch.cuda.synchronize()
+    ref = [d.cpu().numpy().copy() for d in dsts]
+    for d in dsts:
+        d.zero_()
+    g = tuner.capture(args)
+    c0 = O.launch_count()
+    for _ in range(3):
+        g.launch(sp)
+    torch.cuda.synchronize()
+    assert O.launch_count() - c0 == 3 * n
+    for f in range(n):
+        assert np.array_equal(dsts[f].cpu().numpy(), ref[f])
+    g.close()
