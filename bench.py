@@ -648,18 +648,51 @@ def run_c5(args):
                        b.src_end, b.row_begin)
     ms = variants.sweep(a, sp, rounds=max(3, args.rounds // 3))
     tuner = O.Tuner(variants)
+    # the exchange: the kernels' fan-out stores into every rank's symmetric-memory image
+    # (compute + gather in one kernel over NVLink), else chunked NCCL all-gathers
+    mode, fan, fan_note = ("none" if world == 1 and args.c5_mode != "fanout" else args.c5_mode), None, None
+    if mode == "fanout" and world == 1 and not dist.is_initialized():
+        # P = 1 with an explicit fan-out: a one-rank NCCL group exercises the symmetric-memory path
+        import socket
+        with socket.socket() as so:
+            so.bind(("127.0.0.1", 0))
+            port = so.getsockname()[1]
+        dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", world_size=1, rank=0,
+                                device_id=dev)
+    if mode in ("auto", "fanout"):
+        try:
+            fan = shard.FanoutImage((H, W, 4), dev)
+            a = O.with_fanout(type(a).from_buffer_copy(a), fan.ptrs)
+            mode = "fanout"
+        except Exception as ex:   # no symmetric memory on this group / backend
+            if mode == "fanout":
+                raise
+            mode, fan_note = "gather", f"fan-out unavailable ({type(ex).__name__}); chunked all-gather used"
     for _ in range(args.warmup):
         tuner.step(a, sp)
-        if world > 1:
+        if mode == "fanout":
+            fan.barrier()
+        elif world > 1:
             shard.gather_bands(out, full)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
            torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    chunks = max(1, args.c5_chunks) if world > 1 else 1
+    chunks = max(1, args.c5_chunks) if mode == "gather" else 1
     n0 = O.launch_count()
-    if chunks == 1:
+    if mode == "fanout":
+        with ClockSampler(local) as clk:
+            for e0, e1, e2 in ev:
+                e0.record(stream)
+                tuner.step(a, sp)            # stores its band into every rank's image
+                e1.record(stream)
+                fan.barrier()                # every rank's stores have landed
+                e2.record(stream)
+            torch.cuda.synchronize()
+        comp = sum(e0.elapsed_time(e1) for e0, e1, _ in ev)
+        gat = sum(e1.elapsed_time(e2) for _, e1, e2 in ev)
+    elif chunks == 1:
         with ClockSampler(local) as clk:
             for e0, e1, e2 in ev:
                 e0.record(stream)
@@ -723,9 +756,12 @@ def run_c5(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": wl["name"], "kernel": "nlm_f4", "width": W, "height": H,
-                       "rows_per_rank": b.rows_per_rank, "halo_rows": 6, "collective": (f"all_gather of {chunks} row chunks on a side stream, overlapped with the next chunk's kernel"
-                                      if chunks > 1 else "all_gather_into_tensor (NCCL)")
-                       if world > 1 else "none (P=1)", "l2": "4 GiB frame >> L2",
+                       "rows_per_rank": b.rows_per_rank, "halo_rows": 6,
+                       "collective": ("kernel fan-out stores into every rank's symmetric-memory image over NVLink "
+                                      "+ device barrier" if mode == "fanout" else
+                                      f"all_gather of {chunks} row chunks on a side stream, overlapped with the "
+                                      f"next chunk's kernel" if chunks > 1 else "all_gather_into_tensor (NCCL)")
+                       if world > 1 else "none (P=1)", "collective_note": fan_note, "l2": "4 GiB frame >> L2",
                        "parallelism": f"row-sharded x{world}"},
             "compute_only": {"value": H * W * args.steps / (comp * 1e-3) / 1e6, "unit": "Mpix/s",
                              "ms_per_step": comp / args.steps},
@@ -762,6 +798,8 @@ def main():
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
     ap.add_argument("--kernel", default="", help="override the workload's kernel id (same family)")
     ap.add_argument("--c5-chunks", type=int, default=4, help="C5: row chunks per band whose all-gathers overlap compute")
+    ap.add_argument("--c5-mode", default="auto", choices=("auto", "fanout", "gather"),
+                    help="C5 exchange: kernel fan-out into symmetric memory (auto: when available) or all-gather")
     ap.add_argument("--graph", default="auto", choices=("auto", "on", "off"),
                     help="replay the K settled iterations as one CUDA graph (orion_tuner_capture); "
                          "auto = on for the launch-bound C1 frames")

@@ -172,7 +172,13 @@ void orion_variants_destroy(orion_variants *v);
  *             window taps), as in the SDK imageDenoising sample (reading R-O2).
  *  hotspot:   src = T (float), aux = power (same rows as src), dst = T'; fparam[0..4] =
  *             sdc (step/Cap), rx = 1/Rx, ry = 1/Ry, rz = 1/Rz, amb (reading R-O3/R-A15).
- *             src must hold rows row_begin-1 .. row_end (clamped). */
+ *             src must hold rows row_begin-1 .. row_end (clamped).
+ *  fan-out (kernels "knn_f4", "nlm_f4", "nlm_f4_i", "nlm_f4_w8", "nlm_f4_g1"): every output
+ *             pixel is also stored into fanout[0 .. n_fanout) -- full width x height images
+ *             (global row y at y * width), device pointers in this GPU's memory or a peer's
+ *             reachable over NVLink (P2P / symmetric memory) -- so a row-sharded frame is
+ *             gathered by the kernel's own epilogue as each tile completes (C5).  n_fanout = 0:
+ *             no fan-out; > 8, or > 0 for other kernels -> ORION_E_INVALID. */
 typedef struct {
     const void *src;
     void *dst;
@@ -182,6 +188,8 @@ typedef struct {
     int src_row_begin, src_row_end;
     int dst_row_begin;
     float fparam[8];
+    void *fanout[8];
+    int n_fanout;
 } orion_args;
 
 /* Launch variant `level_idx` (realising its occupancy level) on `stream` (async). */

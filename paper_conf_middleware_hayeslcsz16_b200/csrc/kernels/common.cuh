@@ -65,6 +65,29 @@ ORION_DEVICE void load_tile_clamped(float4 *tile, const orion_kargs &a, int gx0,
     }
 }
 
+// Output pixel (x, y) (global row y) into dst (rows from dst_row_begin).
+ORION_DEVICE void store_out(const orion_kargs &a, int x, int y, float4 o)
+{
+    ((float4 *)a.dst)[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = o;
+}
+
+// Fan-out of this thread's output column x, rows [y0, y1) (already in dst, written by this
+// same thread): copied into every fan-out image (full images, row y at y * width) -- the
+// gather of a row-sharded frame written straight into each rank's buffer over NVLink peer
+// memory (C5) as each tile completes.  A compact rolled loop after the unrolled epilogue, so
+// the kernel's hot code does not grow when fan-out is used.
+ORION_DEVICE void fanout_column(const orion_kargs &a, int x, int y0, int y1)
+{
+    if (a.nfan == 0) return;
+    const float4 *src = (const float4 *)a.dst + (size_t)(y0 - a.dst_row_begin) * (size_t)a.width + x;
+#pragma unroll 1
+    for (int y = y0; y < y1; ++y, src += a.width) {
+        const float4 o = *src;
+#pragma unroll 1
+        for (int f = 0; f < a.nfan; ++f) ((float4 *)a.fan[f])[(size_t)y * (size_t)a.width + x] = o;
+    }
+}
+
 // Final SDK imageDenoising blend: clr = acc/sw; out = clr + (c00 - clr) * q.
 ORION_DEVICE float4 lerp_out(float4 c00, float ax, float ay, float az, float sw, int cnt,
                              const orion_kargs &a)

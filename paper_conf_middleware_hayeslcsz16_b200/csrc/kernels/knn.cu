@@ -62,14 +62,12 @@ __device__ __forceinline__ void knn_body(const orion_kargs &a)
     }
     const int x = x0 + tx;
     if (x >= a.width) return;
-    float4 *dst = (float4 *)a.dst;
 #pragma unroll
     for (int p = 0; p < PY; ++p) {
         const int y = y0 + ty * PY + p;
-        if (y < a.row_end)
-            dst[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] =
-                lerp_out(c00[p], ax[p], ay[p], az[p], sw[p], cnt[p], a);
+        if (y < a.row_end) store_out(a, x, y, lerp_out(c00[p], ax[p], ay[p], az[p], sw[p], cnt[p], a));
     }
+    fanout_column(a, x, y0 + ty * PY, min(y0 + ty * PY + PY, a.row_end));
 }
 
 // T = 128 threads (32 x 4), 16-row tiles.

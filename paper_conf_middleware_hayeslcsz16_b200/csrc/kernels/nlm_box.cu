@@ -374,7 +374,6 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
     }
     const int x = x0 + t;
     if (t >= TW || x >= a.width) return;
-    float4 *dst = (float4 *)a.dst;
 #pragma unroll
     for (int r = 0; r < TH; ++r) {
         const int y = y0 + r;
@@ -382,8 +381,9 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
         const int pc = (r + 6) * PW + t + 9;
         const float4 c00 = make_float4(prg[pc].x, prg[pc].y, pb[pc], 0.0f);
         const int c = (int)((A.cnt[r >> 2] >> (8 * (r & 3))) & 0xffu);
-        dst[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = lerp_out(c00, A.axy[r].x, A.axy[r].y, A.azs[r].x, A.azs[r].y, c, a);
+        store_out(a, x, y, lerp_out(c00, A.axy[r].x, A.axy[r].y, A.azs[r].x, A.azs[r].y, c, a));
     }
+    fanout_column(a, x, y0, min(y0 + TH, a.row_end));
 }
 
 }  // namespace

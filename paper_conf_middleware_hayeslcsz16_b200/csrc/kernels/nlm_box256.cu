@@ -188,7 +188,6 @@ extern "C" __global__ void __launch_bounds__(256) orion_nlm_box256_f4_256(orion_
     }
     const int x = x0 + t;
     if (t >= TW || x >= a.width) return;
-    float4 *dst = (float4 *)a.dst;
 #pragma unroll
     for (int r = 0; r < RH; ++r) {
         if (h && r == 0) continue;               // row 11 belongs to the upper half
@@ -197,7 +196,7 @@ extern "C" __global__ void __launch_bounds__(256) orion_nlm_box256_f4_256(orion_
         const int pc = (r0 + r + 6) * PW + t + 9;
         const float4 c00 = make_float4(pr[pc], pg[pc], pb[pc], 0.0f);
         const int c = (int)((A.cnt[r >> 2] >> (8 * (r & 3))) & 0xffu);
-        dst[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] =
-            lerp_out(c00, A.axy[r].x, A.axy[r].y, A.azs[r].x, A.azs[r].y, c, a);
+        store_out(a, x, y, lerp_out(c00, A.axy[r].x, A.axy[r].y, A.azs[r].x, A.azs[r].y, c, a));
     }
+    fanout_column(a, x, y0 + r0 + (h ? 1 : 0), min(y0 + r0 + RH, a.row_end));
 }

@@ -63,6 +63,7 @@ struct KernelDef {
     int smem_bytes;         // > 0: explicit dynamic shared-memory need (overrides smem_tile)
     int width_align;        // > 1: the image width must be a multiple of this
     int steps_per_launch;   // stencil steps one launch performs (0 / 1 = one)
+    int fanout;             // 1: the kernel's epilogue honours orion_args.fanout (store_out)
     int dyn_need() const
     {
         if (smem_bytes > 0) return smem_bytes;

@@ -17,6 +17,8 @@ typedef struct {
     unsigned *probe;                 /* NULL in every real launch.  Non-NULL: residency probe only --
                                         the CTA records how many CTAs share its SM and exits
                                         (orion_probe in kernels/common.cuh)                        */
+    void *fan[8];                    /* denoisers: extra full-image outputs (global row y at y*width), */
+    int nfan;                        /* e.g. every rank's gather buffer over NVLink peer memory        */
 } orion_kargs;
 
 #endif

@@ -46,22 +46,22 @@ static const char *module_ptx(const char *module)
 // id, T, entry, module, bx, by, tile_w, tile_h, halo, kind, smem_tile, smem_bytes.  The first row of
 // each id is its default CTA size.
 static const KernelDef kKernels[] = {
-    {"knn_f4", 128, "orion_knn_f4_128", "knn", 32, 4, 32, 16, 3, K_KNN, 1, 0},
-    {"knn_f4", 256, "orion_knn_f4_256", "knn", 32, 8, 32, 32, 3, K_KNN, 1, 0},
-    {"knn_f4", 64, "orion_knn_f4_64", "knn", 8, 8, 8, 32, 3, K_KNN, 1, 0},
+    {"knn_f4", 128, "orion_knn_f4_128", "knn", 32, 4, 32, 16, 3, K_KNN, 1, 0, 1, 1, 1},
+    {"knn_f4", 256, "orion_knn_f4_256", "knn", 32, 8, 32, 32, 3, K_KNN, 1, 0, 1, 1, 1},
+    {"knn_f4", 64, "orion_knn_f4_64", "knn", 8, 8, 8, 32, 3, K_KNN, 1, 0, 1, 1, 1},
     // nlm_box: 3 planar (122+18) x (23+12) fp32 planes (pitch 141) + 32 x 129 floats of H_o
     // up to 3 offset pairs per pass: 3 H_o buffers (2 CTAs/SM) -- the C2 / C5 default
     {"nlm_f4", 128, "orion_nlm_box3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
-     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4},
+     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},
     // same, integer (fixed-point, exact) box sums
     {"nlm_f4_i", 128, "orion_nlm_boxi3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
-     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4},
+     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},
     // same tile, 256 threads (8 warps per CTA)
     {"nlm_f4_w8", 256, "orion_nlm_box256_f4_256", "nlm_box256", 256, 1, 122, 23, 6, K_NLM, 0,
-     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4},
+     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},
     // one offset pair per pass: 1 H_o buffer (3 CTAs/SM)
     {"nlm_f4_g1", 128, "orion_nlm_box_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
-     3 * 35 * 141 * 4 + 32 * 129 * 4},
+     3 * 35 * 141 * 4 + 32 * 129 * 4, 1, 1, 1},
     {"nlm_f4_direct", 128, "orion_nlm_direct_f4_128", "nlm_direct", 32, 4, 32, 4, 6, K_NLM, 1, 0},
     {"nlm_f4_regheavy", 128, "orion_nlm_regheavy_f4_128", "nlm_regheavy", 32, 4, 32, 4, 6, K_NLM, 1, 0},
     {"nlm_f4_regheavy", 64, "orion_nlm_regheavy_f4_64", "nlm_regheavy", 8, 8, 8, 8, 6, K_NLM, 1, 0},

@@ -42,7 +42,13 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
     if (def.width_align > 1 && a->width % def.width_align)
         return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + " needs width % " +
                                          std::to_string(def.width_align) + " == 0");
+    if (a->n_fanout < 0 || a->n_fanout > 8 || (a->n_fanout > 0 && !def.fanout))
+        return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + ": bad n_fanout");
+    for (int f = 0; f < a->n_fanout; ++f)
+        if (!a->fanout[f]) return fail(ORION_E_INVALID, "orion_launch: NULL fanout buffer");
     std::memset(k, 0, sizeof *k);
+    for (int f = 0; f < a->n_fanout; ++f) k->fan[f] = a->fanout[f];
+    k->nfan = a->n_fanout;
     k->src = a->src;
     k->dst = a->dst;
     k->aux = a->aux;

@@ -77,7 +77,19 @@ class Args(ctypes.Structure):
                 ("width", ctypes.c_int), ("height", ctypes.c_int),
                 ("row_begin", ctypes.c_int), ("row_end", ctypes.c_int),
                 ("src_row_begin", ctypes.c_int), ("src_row_end", ctypes.c_int),
-                ("dst_row_begin", ctypes.c_int), ("fparam", ctypes.c_float * 8)]
+                ("dst_row_begin", ctypes.c_int), ("fparam", ctypes.c_float * 8),
+                ("fanout", ctypes.c_void_p * 8), ("n_fanout", ctypes.c_int)]
+
+
+def with_fanout(a: Args, ptrs) -> Args:
+    """Add fan-out outputs (full-image device pointers, e.g. every rank's gather buffer) to a."""
+    ptrs = list(ptrs)
+    if len(ptrs) > 8:
+        raise ValueError("at most 8 fan-out buffers")
+    for i, p in enumerate(ptrs):
+        a.fanout[i] = p
+    a.n_fanout = len(ptrs)
+    return a
 
 
 class TunerCfg(ctypes.Structure):

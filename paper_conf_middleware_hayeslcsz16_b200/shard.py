@@ -7,6 +7,13 @@ its own Orion tuner on that slab (per-GPU tuning), and one NCCL
 ``all_gather_into_tensor`` over NVLink collects the output bands -- the only
 inter-GPU exchange of the configuration.
 
+Two ways to gather: (1) NCCL all-gathers of row chunks on a side stream, overlapping
+the next chunk's kernel (``gather_rows``); (2) the kernels' fan-out epilogue
+(``orion_args.fanout``): with the full images in symmetric memory (``FanoutImage``), each
+rank's kernel stores every output pixel straight into every rank's image over NVLink as
+its tiles complete, and a device-side barrier closes the step -- compute and exchange in
+one kernel, no collective call.
+
 Host-side logic only (partitioning, halo arithmetic, the gather glue); all pixel
 work happens in liborion's kernels.  The gather glue takes any process group, so
 it is exercised with ``gloo`` on CPU tensors in tests/test_shard.py.
@@ -80,3 +87,21 @@ def gather_bands(out_band, full_out, group=None):
         return full_out
     dist.all_gather_into_tensor(full_out, out_band.contiguous(), group=group)
     return full_out
+
+
+class FanoutImage:
+    """The full output image of a row-sharded frame in symmetric memory: every rank holds one,
+    and ``ptrs`` are all ranks' device addresses (peer memory over NVLink), in rank order --
+    the fan-out list of ``orion.with_fanout``.  ``barrier()`` (device-side, on the current
+    stream) orders every rank's stores before anyone reads its image."""
+
+    def __init__(self, shape, device, group=None):
+        import torch
+        import torch.distributed as dist
+        import torch.distributed._symmetric_memory as symm_mem
+        self.tensor = symm_mem.empty(*shape, dtype=torch.float32, device=device)
+        self.handle = symm_mem.rendezvous(self.tensor, group or dist.group.WORLD)
+        self.ptrs = [int(p) for p in self.handle.buffer_ptrs]
+
+    def barrier(self):
+        self.handle.barrier()
