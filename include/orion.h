@@ -312,6 +312,11 @@ void orion_host_pipe_destroy(orion_host_pipe *p);
 /* Current ladder: *direction, ladder level indices (ladder[0] = original) -> out[]. */
 orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, int capacity, int *n_out);
 orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final);
+/* Checkpoint / resume of the tuner's decision: a final level recorded from an
+ * earlier run (orion_tuner_final, keyed by the caller on kernel id, device and shape) is set
+ * directly, so a restarted application skips the Fig. 9 exploration.  ORION_E_INVALID for an
+ * index outside the variants; ORION_E_STATE while an async measurement is in flight. */
+orion_status orion_tuner_resume(orion_tuner *t, int final_level_idx);
 void orion_tuner_destroy(orion_tuner *t);
 
 /* ---- CUDA graph replay of settled iterations (launch-bound loops) ------------------------- */

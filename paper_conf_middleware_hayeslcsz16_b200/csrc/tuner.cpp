@@ -554,6 +554,19 @@ orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, 
     return ORION_OK;
 }
 
+orion_status orion_tuner_resume(orion_tuner *t, int final_level_idx)
+{
+    if (!t) return fail(ORION_E_INVALID, "orion_tuner_resume: NULL");
+    if (final_level_idx < 0 || final_level_idx >= (int)t->v->vars.size())
+        return fail(ORION_E_INVALID, "orion_tuner_resume: level index out of range");
+    if (t->inflight) return fail(ORION_E_STATE, "orion_tuner_resume: a measurement is in flight");
+    t->f.final_idx = final_level_idx;
+    t->f.final_iter = t->f.iter;
+    t->pending_level = -1;
+    t->samples = 0;
+    return ORION_OK;
+}
+
 orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final)
 {
     if (!t) return fail(ORION_E_INVALID, "orion_tuner_final: NULL");

@@ -141,6 +141,7 @@ def lib() -> ctypes.CDLL:
                                          P(ctypes.c_longlong)],
                 "orion_tune_split": [V, P(Args), I, V, P(StepReport)],
                 "orion_tuner_capture": [V, P(Args), I, P(V)],
+                "orion_tuner_resume": [V, I],
                 "orion_graph_launch": [V, V],
                 "orion_tune_run_host": [V, P(Args), I, V, V, V, P(I), V, P(ctypes.c_longlong),
                                         P(ctypes.c_longlong)],
@@ -385,6 +386,10 @@ class Tuner:
                                          ctypes.c_void_p(dev_b), ctypes.c_void_p(dev_aux), r, _s(stream),
                                          ctypes.byref(hi), ctypes.byref(ho)), "orion_tune_run_host")
         return hi.value, ho.value
+
+    def resume(self, final_level_idx: int):
+        """orion_tuner_resume: adopt a final level recorded by an earlier run (skip exploration)."""
+        _check(lib().orion_tuner_resume(self.h, final_level_idx), "orion_tuner_resume")
 
     def capture(self, args_list: list, stream=None) -> "Graph":
         """orion_tuner_capture: the settled kernel's launches for args_list[i] as one CUDA graph."""

@@ -52,3 +52,21 @@ def test_graph_replay_matches_direct_launches(knn):
     for f in range(n):
         assert np.array_equal(dsts[f].cpu().numpy(), ref[f])
     g.close()
+
+
+def test_resume_skips_exploration(knn):
+    W = H = 64
+    sp = torch.cuda.current_stream().cuda_stream
+    src = torch.from_numpy(synth.noisy_rgba(W, H, seed=2, sigma=0.2)).cuda()
+    dst = torch.zeros_like(src)
+    a = O.denoise_args("knn_f4", src.data_ptr(), dst.data_ptr(), W, H)
+    t = O.Tuner(knn)
+    with pytest.raises(O.OrionError):
+        t.resume(len(knn))
+    t.resume(len(knn) - 1)
+    r = t.step(a, sp)
+    assert r.phase == 1 and r.level_idx == len(knn) - 1 and t.final()[0] == len(knn) - 1
+    g = t.capture([a])                       # settled: capturable at once
+    g.launch(sp)
+    torch.cuda.synchronize()
+    g.close()
