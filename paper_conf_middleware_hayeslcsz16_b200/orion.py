@@ -352,16 +352,26 @@ def default_cfg(**kw) -> TunerCfg:
 class Tuner:
     """orion_tuner handle: Fig. 8 ladder + Fig. 9 walk across iterations."""
 
-    def __init__(self, variants: Variants, cfg: TunerCfg | None = None):
+    def __init__(self, variants: Variants, cfg: TunerCfg | None = None, trace: str | None = None):
+        """trace: optional JSONL path -- one record per orion_tune_step (iteration, level index,
+        its CTAs/SM, phase, measured ms, final level): the tuner's per-iteration log."""
         self.variants = variants
         h = ctypes.c_void_p()
         _check(lib().orion_tuner_create(variants.h, ctypes.byref(cfg or default_cfg()), ctypes.byref(h)),
                "orion_tuner_create")
         self.h = h
+        self._trace = open(trace, "a") if trace else None
 
     def step(self, args: Args, stream=None) -> StepReport:
         r = StepReport()
         _check(lib().orion_tune_step(self.h, ctypes.byref(args), _s(stream), ctypes.byref(r)), "orion_tune_step")
+        if self._trace is not None:
+            import json
+            self._trace.write(json.dumps({"iteration": r.iteration, "level_idx": r.level_idx,
+                                          "ctas_per_sm": self.variants.level(r.level_idx).ctas_per_sm,
+                                          "phase": "explore" if r.phase == 0 else "final",
+                                          "ms": r.ms if r.ms >= 0 else None,
+                                          "final_level_idx": r.final_level_idx}) + "\n")
         return r
 
     def split(self, args: Args, bands: int, stream=None) -> list[StepReport]:
@@ -407,6 +417,9 @@ class Tuner:
         return f.value, it.value
 
     def close(self):
+        if getattr(self, "_trace", None) is not None:
+            self._trace.close()
+            self._trace = None
         if getattr(self, "h", None):
             lib().orion_tuner_destroy(self.h)
             self.h = None

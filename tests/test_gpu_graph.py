@@ -70,3 +70,21 @@ def test_resume_skips_exploration(knn):
     g.launch(sp)
     torch.cuda.synchronize()
     g.close()
+
+
+def test_trace_jsonl(knn, tmp_path):
+    import json
+    W = H = 64
+    sp = torch.cuda.current_stream().cuda_stream
+    src = torch.from_numpy(synth.noisy_rgba(W, H, seed=4, sigma=0.2)).cuda()
+    dst = torch.zeros_like(src)
+    a = O.denoise_args("knn_f4", src.data_ptr(), dst.data_ptr(), W, H)
+    path = tmp_path / "trace.jsonl"
+    t = O.Tuner(knn, trace=str(path))
+    for _ in range(12):
+        t.step(a, sp)
+    t.close()
+    recs = [json.loads(line) for line in open(path)]
+    assert [r["iteration"] for r in recs] == list(range(12))
+    assert recs[0]["phase"] == "explore" and recs[0]["ms"] is not None
+    assert all(r["ctas_per_sm"] >= 1 for r in recs)
