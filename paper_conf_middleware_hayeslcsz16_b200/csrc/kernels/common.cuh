@@ -94,7 +94,12 @@ ORION_DEVICE float4 lerp_out(float4 c00, float ax, float ay, float az, float sw,
 {
     const float lerpc = a.fparam[1];
     const float q = (cnt >= a.iparam0) ? lerpc : __fsub_rn(1.0f, lerpc);
-    float cx = __fdiv_rn(ax, sw), cy = __fdiv_rn(ay, sw), cz = __fdiv_rn(az, sw);
+    // acc / sw as acc * (1/sw) with one MUFU reciprocal (rcp.approx, <= 1 ulp): sw >= 1 always
+    // (the centre weight is exactly 1), so the quotient is within 2 ulp of the IEEE division
+    // -- far inside the 1e-5 tolerance -- and the epilogue needs no division subroutine.
+    float rs;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(rs) : "f"(sw));
+    float cx = __fmul_rn(ax, rs), cy = __fmul_rn(ay, rs), cz = __fmul_rn(az, rs);
     float4 o;
     o.x = __fmaf_rn(__fsub_rn(c00.x, cx), q, cx);
     o.y = __fmaf_rn(__fsub_rn(c00.y, cy), q, cy);

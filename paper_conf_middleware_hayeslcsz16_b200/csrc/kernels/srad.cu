@@ -61,6 +61,39 @@ ORION_DEVICE float srad_update(float Jc, const SradCell &k, float cS, float cE, 
     return __fmaf_rn(lam4, __fmaf_rn(k.c, k.dnw, __fmaf_rn(cS, k.ds, __fmul_rn(cE, k.de))), Jc);
 }
 
+// The same two functions for a pair of horizontally adjacent cells on the packed fp32x2 pipe
+// (FADD2 / FMUL2 / FFMA2: two independent IEEE .rn operations per instruction, bit-identical
+// to the scalar forms above, operation by operation).  dW / dE of a pair are not register
+// pairs of the row, so they are scalar FSUBs written straight into pairs; every other step is
+// one packed instruction for both cells.
+struct SradPair {
+    float2 c, dnw, ds, de;
+};
+ORION_DEVICE float2 f2(float v) { return make_float2(v, v); }
+ORION_DEVICE float2 neg(float2 v) { return make_float2(-v.x, -v.y); }
+ORION_DEVICE SradPair srad_coeff2(float2 Jc, float2 N, float2 S, float2 dW, float2 dE, float iqden, float nq)
+{
+    const float2 dN = __fadd2_rn(N, neg(Jc)), dS = __fadd2_rn(S, neg(Jc));
+    const float2 g2 = __ffma2_rn(dE, dE, __ffma2_rn(dW, dW, __ffma2_rn(dS, dS, __fmul2_rn(dN, dN))));
+    const float2 dnw = __fadd2_rn(dN, dW);
+    const float2 sd = __fadd2_rn(__fadd2_rn(dnw, dS), dE);
+    const float2 num = __ffma2_rn(__fmul2_rn(f2(-0.0625f), sd), sd, __fmul2_rn(f2(0.5f), g2));
+    const float2 den = __ffma2_rn(f2(0.25f), sd, Jc);
+    const float2 dd = __fmul2_rn(den, den);
+    const float2 qsqr = __fmul2_rn(num, make_float2(rcp_approx(dd.x), rcp_approx(dd.y)));
+    const float2 t = __fadd2_rn(f2(1.0f), __ffma2_rn(qsqr, f2(iqden), f2(nq)));
+    SradPair r;
+    r.c = make_float2(__saturatef(rcp_approx(t.x)), __saturatef(rcp_approx(t.y)));
+    r.dnw = dnw;
+    r.ds = dS;
+    r.de = dE;
+    return r;
+}
+ORION_DEVICE float2 srad_update2(float2 Jc, const SradPair &k, float2 cS, float2 cE, float lam4)
+{
+    return __ffma2_rn(f2(lam4), __ffma2_rn(k.c, k.dnw, __ffma2_rn(cS, k.ds, __fmul2_rn(cE, k.de))), Jc);
+}
+
 struct SradConsts {
     float lam4, iqden, nq;
 };
@@ -219,6 +252,10 @@ template <int V>
 struct CRow {
     SradCell k[V];
 };
+template <>
+struct CRow<4> {
+    SradPair p[2];   // cells (0, 1) and (2, 3)
+};
 }  // namespace
 
 template <int V>
@@ -256,19 +293,42 @@ __device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys,
         if (lane == 31) Ev = T.xa;
         if (east_clamp) Ev = T.v[V - 1];
         CRow<V> c;
+        if constexpr (V == 4) {
+            const float *t = T.v;
+            c.p[0] = srad_coeff2(make_float2(t[0], t[1]), make_float2(N.v[0], N.v[1]), make_float2(S.v[0], S.v[1]),
+                                 make_float2(__fsub_rn(Wv, t[0]), __fsub_rn(t[0], t[1])),
+                                 make_float2(__fsub_rn(t[1], t[0]), __fsub_rn(t[2], t[1])), kc.iqden, kc.nq);
+            c.p[1] = srad_coeff2(make_float2(t[2], t[3]), make_float2(N.v[2], N.v[3]), make_float2(S.v[2], S.v[3]),
+                                 make_float2(__fsub_rn(t[1], t[2]), __fsub_rn(t[2], t[3])),
+                                 make_float2(__fsub_rn(t[3], t[2]), __fsub_rn(Ev, t[3])), kc.iqden, kc.nq);
+        } else {
 #pragma unroll
-        for (int k = 0; k < V; ++k)
-            c.k[k] = srad_coeff(T.v[k], N.v[k], S.v[k], k == 0 ? Wv : T.v[k - 1], k == V - 1 ? Ev : T.v[k + 1],
-                                kc.iqden, kc.nq);
+            for (int k = 0; k < V; ++k)
+                c.k[k] = srad_coeff(T.v[k], N.v[k], S.v[k], k == 0 ? Wv : T.v[k - 1], k == V - 1 ? Ev : T.v[k + 1],
+                                    kc.iqden, kc.nq);
+        }
         return c;
     };
     auto update_row = [&](int y, const SRow<V> &T, const CRow<V> &c0, const CRow<V> &c1) {
-        float cE = __shfl_down_sync(0xffffffffu, c0.k[0].c, 1);
-        if (east_clamp) cE = c0.k[V - 1].c;
         float o[V];
+        if constexpr (V == 4) {
+            float cE = __shfl_down_sync(0xffffffffu, c0.p[0].c.x, 1);
+            if (east_clamp) cE = c0.p[1].c.y;
+            const float2 lo = srad_update2(make_float2(T.v[0], T.v[1]), c0.p[0], c1.p[0].c,
+                                           make_float2(c0.p[0].c.y, c0.p[1].c.x), kc.lam4);
+            const float2 hi = srad_update2(make_float2(T.v[2], T.v[3]), c0.p[1], c1.p[1].c,
+                                           make_float2(c0.p[1].c.y, cE), kc.lam4);
+            o[0] = lo.x;
+            o[1] = lo.y;
+            o[2] = hi.x;
+            o[3] = hi.y;
+        } else {
+            float cE = __shfl_down_sync(0xffffffffu, c0.k[0].c, 1);
+            if (east_clamp) cE = c0.k[V - 1].c;
 #pragma unroll
-        for (int k = 0; k < V; ++k)
-            o[k] = srad_update(T.v[k], c0.k[k], c1.k[k].c, k == V - 1 ? cE : c0.k[k + 1].c, kc.lam4);
+            for (int k = 0; k < V; ++k)
+                o[k] = srad_update(T.v[k], c0.k[k], c1.k[k].c, k == V - 1 ? cE : c0.k[k + 1].c, kc.lam4);
+        }
         if (writer) {
             float *orow = Jo + (size_t)y * (size_t)W;
             if constexpr (V == 4)

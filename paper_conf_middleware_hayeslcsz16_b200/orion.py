@@ -18,7 +18,7 @@ import threading
 from dataclasses import dataclass
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "liborion.so")
+LIB_PATH = os.environ.get("ORION_LIB") or os.path.join(_HERE, "liborion.so")  # ORION_LIB: A/B experiments
 
 ORION_OK = 0
 STATUS = {0: "ORION_OK", -1: "ORION_E_INVALID", -2: "ORION_E_CAPACITY", -3: "ORION_E_INFEASIBLE",
