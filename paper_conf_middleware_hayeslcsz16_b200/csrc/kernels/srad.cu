@@ -224,7 +224,7 @@ extern "C" __global__ void __launch_bounds__(1024) orion_srad_stats(const float 
 // CTA = 8 warps over a 124 x 128 tile: V = 4 -> 8 strips of 16 rows; V = 1 -> 4 column
 // groups of 31 x 2 strips of 64 rows.
 namespace {
-constexpr int SRAD_NB = 4;      // ring slots per warp
+constexpr int SRAD_NB = 6;      // ring slots per warp (a multiple of the 6-row loop body: static slots)
 constexpr int SRAD_SLOT = 132;  // floats per slot: 32 lanes x up to 4 columns + 2 outer columns (+pad)
 }  // namespace
 
@@ -346,8 +346,7 @@ __device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys,
     const int own = V * lane, oxa = 32 * V + (lane == 0 ? 0 : 1);
     const float *pn = J + (size_t)min(ys + 2, H - 1) * (size_t)W;
     int rn = ys + 2;                                            // row pn points at (unclamped)
-    auto issue = [&](int q) {
-        float *sl = ring + (q % SRAD_NB) * SRAD_SLOT;
+    auto issue = [&](float *sl) {
         if constexpr (V == 4)
             srad_cp16(sl + own, pn + cxl);
         else
@@ -356,8 +355,7 @@ __device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys,
         if (rn < H - 1) pn += W;
         ++rn;
     };
-    auto slot_row = [&](int q) {
-        const float *sl = ring + (q % SRAD_NB) * SRAD_SLOT;
+    auto slot_row = [&](const float *sl) {
         SRow<V> r;
         if constexpr (V == 4) {
             const float4 t = *reinterpret_cast<const float4 *>(sl + own);
@@ -375,7 +373,7 @@ __device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys,
     const int nq = yb - ys;
 #pragma unroll
     for (int q = 0; q < SRAD_NB - 1; ++q) {
-        if (q < nq) issue(q);
+        if (q < nq) issue(ring + q * SRAD_SLOT);
         srad_commit();
     }
     SRow<V> j0 = load(J + (size_t)ys * (size_t)W), j1 = load(J + (size_t)min(ys + 1, H - 1) * (size_t)W), j2;
@@ -384,46 +382,55 @@ __device__ __forceinline__ void srad_strip(const orion_kargs &a, int x0, int ys,
     // S), cT = c(y), cS = c(y+1) (written).  The row registers rotate through three variables and
     // the coefficient rows through two, so six consecutive rows are written out with permuted
     // arguments -- no register moves between rows.
-    auto row = [&](int q, const SRow<V> &N, const SRow<V> &T, SRow<V> &S, const CRow<V> &cT, CRow<V> &cS) {
-        if (q + SRAD_NB - 1 < nq) issue(q + SRAD_NB - 1);
+    auto row = [&](int q, float *sl_read, float *sl_issue, const SRow<V> &N, const SRow<V> &T, SRow<V> &S,
+                   const CRow<V> &cT, CRow<V> &cS) {
+        if (q + SRAD_NB - 1 < nq) issue(sl_issue);
         srad_commit();
         srad_wait<SRAD_NB - 1>();
-        S = slot_row(q);
+        S = slot_row(sl_read);
         cS = coeff_row(N, T, S);
         update_row(ys + q, N, cT, cS);
     };
     int q = 0;
 #pragma unroll 1
-    for (; q + 6 <= nq; q += 6) {
-        row(q, j0, j1, j2, c0, c1);
-        row(q + 1, j1, j2, j0, c1, c0);
-        row(q + 2, j2, j0, j1, c0, c1);
-        row(q + 3, j0, j1, j2, c1, c0);
-        row(q + 4, j1, j2, j0, c0, c1);
-        row(q + 5, j2, j0, j1, c1, c0);
+#define SR_S(k) (ring + (k) * SRAD_SLOT)
+#define SR_I(k) SR_S(((k) + SRAD_NB - 1) % SRAD_NB)
+    for (; q + 6 <= nq; q += 6) {                               // slot of row q + k is k
+        row(q, SR_S(0), SR_I(0), j0, j1, j2, c0, c1);
+        row(q + 1, SR_S(1), SR_I(1), j1, j2, j0, c1, c0);
+        row(q + 2, SR_S(2), SR_I(2), j2, j0, j1, c0, c1);
+        row(q + 3, SR_S(3), SR_I(3), j0, j1, j2, c1, c0);
+        row(q + 4, SR_S(4), SR_I(4), j1, j2, j0, c0, c1);
+        row(q + 5, SR_S(5), SR_I(5), j2, j0, j1, c1, c0);
     }
 #pragma unroll 1
     for (; q < nq; ++q) {                                       // the last < 6 rows
-        row(q, j0, j1, j2, c0, c1);
+        row(q, SR_S(q % SRAD_NB), SR_I(q % SRAD_NB), j0, j1, j2, c0, c1);
         j0 = j1;
         j1 = j2;
         c0 = c1;
     }
+#undef SR_S
+#undef SR_I
     srad_wait<0>();
     if (ye == H) update_row(H - 1, j0, c0, c0);               // last image row: c_S = own c
 }
 
-// T = 256 threads (32 x 8 warps), output tile 124 x 128.
+// T = 256 threads (32 x 8 warps), output tile 124 x (8 * SRAD_RY).  Longer strips amortise the
+// strip prologue (three J rows and one coefficient row computed before the first output row).
+#ifndef SRAD_RY
+#define SRAD_RY 32
+#endif
 extern "C" __global__ void __launch_bounds__(256) orion_srad4_f32_256(orion_kargs a)
 {
     ORION_PROBE(a);
     const int w = threadIdx.y;
     if ((a.width & 3) == 0) {
-        const int ys = a.row_begin + blockIdx.y * 128 + w * 16;
-        if (ys < a.row_end) srad_strip<4>(a, blockIdx.x * 124, ys, min(ys + 16, a.row_end));
+        const int ys = a.row_begin + blockIdx.y * (8 * SRAD_RY) + w * SRAD_RY;
+        if (ys < a.row_end) srad_strip<4>(a, blockIdx.x * 124, ys, min(ys + SRAD_RY, a.row_end));
     } else {
         const int x0 = blockIdx.x * 124 + (w & 3) * 31;
-        const int ys = a.row_begin + blockIdx.y * 128 + (w >> 2) * 64;
-        if (ys < a.row_end && x0 < a.width) srad_strip<1>(a, x0, ys, min(ys + 64, a.row_end));
+        const int ys = a.row_begin + blockIdx.y * (8 * SRAD_RY) + (w >> 2) * (4 * SRAD_RY);
+        if (ys < a.row_end && x0 < a.width) srad_strip<1>(a, x0, ys, min(ys + 4 * SRAD_RY, a.row_end));
     }
 }

@@ -74,7 +74,7 @@ static const KernelDef kKernels[] = {
     {"srad_f32_tile", 256, "orion_srad_f32_256", "srad", 32, 8, 32, 32, 2, K_SRAD, 0, (35 * 35 + 33 * 33) * 4},
     // srad, register-sliding: 124 x 128 tile; float4 lanes (width % 4 == 0) or scalar lanes;
     // rows stream through a 4-slot cp.async ring per warp (8 x 4 x 132 floats)
-    {"srad_f32", 256, "orion_srad4_f32_256", "srad", 32, 8, 124, 128, 2, K_SRAD, 0, 8 * 4 * 132 * 4},
+    {"srad_f32", 256, "orion_srad4_f32_256", "srad", 32, 8, 124, 256, 2, K_SRAD, 0, 8 * 6 * 132 * 4},
 };
 
 const KernelDef *find_kernel(const char *id, int threads)
