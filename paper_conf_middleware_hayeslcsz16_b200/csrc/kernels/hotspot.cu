@@ -335,3 +335,126 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2_f32_256(orion_k
     ORION_PROBE(a);
     hotspot2_body<8, H2_ROWS>(a);
 }
+
+// ---- two steps per launch, halo lanes (hotspot2h) ------------------------------------------
+// The same two-step update with the warp's column halo carried by whole lanes instead of edge
+// lanes: a warp loads 128 consecutive columns [base-4, base+124) as float4 lanes and writes the
+// 120 columns [base, base+120) of lanes 1..30.  Lane 0's last and lane 31's first T1 cells are
+// exactly the step-1 halo the outer T2 cells need (their own neighbours are in-lane or one
+// shuffle away), so there are no scalar outer-column loads, no extra T1 cell and no per-lane
+// edge copies: per row two 16-byte cp.async, two 16-byte ring reads, four shuffles.  6.7 % of
+// the lanes' cells are recomputed halo (the neighbouring warp's), traded for half the
+// memory-pipe instructions of hotspot2_f32.  Clamp-to-edge: the lane holding column 0 takes
+// its own value as W, the lane holding column W-1 its own value as E; lanes past either edge
+// load clamped columns, write nothing and feed no written cell.  Bit-identical to one-step
+// launches (every cell is hs_cell4's operation sequence, = hs_cell's).
+namespace {
+constexpr int H2H_NB = 6;                   // ring slots per warp: the 6-row body's static slots
+constexpr int H2H_SLOT = 256;               // floats: T0 segment (128) + P segment (128)
+}  // namespace
+
+template <int RY, bool BOTTOM>
+__device__ __forceinline__ void hotspot2h_strip(const orion_kargs &a, int ys, int ye)
+{
+    extern __shared__ float4 smem4[];
+    const int W = a.width, H = a.height;
+    const int lane = threadIdx.x;
+    const float c[5] = {a.fparam[0], a.fparam[1], a.fparam[2], a.fparam[3], a.fparam[4]};
+    const int base = blockIdx.x * 120;
+    const int cx = base - 4 + 4 * lane;            // the lane's first column (lane 0: halo)
+    const int cxl = clampi(cx, 0, W - 4);
+    const bool writer = lane >= 1 && lane <= 30 && cx < W;
+    const bool wclamp = cx == 0, eclamp = cx + 4 >= W;
+    const float *t0 = (const float *)a.src - (size_t)a.src_row_begin * (size_t)W;
+    const float *p0 = (const float *)a.aux - (size_t)a.src_row_begin * (size_t)W;
+    float *ring = reinterpret_cast<float *>(smem4) + threadIdx.y * (H2H_NB * H2H_SLOT);
+    const int own = 4 * lane;
+
+    auto step = [&c, wclamp, eclamp](const float4 &N, const float4 &T, const float4 &S, const float4 &P) {
+        float Wv = __shfl_up_sync(0xffffffffu, T.w, 1);
+        float Ev = __shfl_down_sync(0xffffffffu, T.x, 1);
+        if (wclamp) Wv = T.x;
+        if (eclamp) Ev = T.w;
+        return hs_cell4(T, N, S, Ev, Wv, P, c);
+    };
+    auto rowp = [&](const float *b, int y) { return b + (size_t)clampi(y, 0, H - 1) * (size_t)W + cxl; };
+    auto load = [&](const float *p) { return __ldg(reinterpret_cast<const float4 *>(p)); };
+    // issue() runs for q = 0, 1, ... in order: slot q % NB gets T0(clamp(ys+2+q)) and P(ys+1+q)
+    const float *tn = rowp(t0, ys + 2), *pn = rowp(p0, ys + 1);
+    int rt = ys + 2;
+    auto issue = [&](float *sl) {
+        cp_async16(sl + own, tn);
+        cp_async16(sl + 128 + own, pn);
+        if (!BOTTOM || rt < H - 1) tn += W;
+        pn += W;
+        ++rt;
+    };
+    const int yb = min(ye, H - 1);
+    const int nq = yb - ys;
+#pragma unroll
+    for (int q = 0; q < H2H_NB - 1; ++q) {
+        if (q < nq) issue(ring + q * H2H_SLOT);
+        cp_async_commit();
+    }
+    const bool top = ys == 0;
+    const float4 tm2 = load(rowp(t0, ys - 2)), tm1 = load(rowp(t0, ys - 1));
+    float4 tc0 = load(rowp(t0, ys)), tc1 = load(rowp(t0, ys + 1)), tcx;
+    const float4 Pa = load(rowp(p0, ys - 1));
+    float4 pa = load(rowp(p0, ys)), pb;
+    float4 ua = top ? step(tc0, tc0, tc1, pa) : step(tm2, tm1, tc0, Pa);
+    float4 ub = step(tm1, tc0, tc1, pa), uz;
+    float *orow = (float *)a.dst + (size_t)cx + ((size_t)ys - (size_t)a.dst_row_begin) * (size_t)W;
+    auto row = [&](int q, const float *sl_read, float *sl_issue, const float4 &A, const float4 &B, float4 &C,
+                   const float4 &X, const float4 &Y, float4 &Z, const float4 &Pcur, float4 &Pnext) {
+        if (q + H2H_NB - 1 < nq) issue(sl_issue);
+        cp_async_commit();
+        cp_async_wait<H2H_NB - 1>();
+        C = *reinterpret_cast<const float4 *>(sl_read + own);
+        Pnext = *reinterpret_cast<const float4 *>(sl_read + 128 + own);
+        Z = step(A, B, C, Pnext);                  // T1(y+1)
+        const float4 o = step(X, Y, Z, Pcur);      // T2(y)
+        if (writer) *reinterpret_cast<float4 *>(orow) = o;
+        orow += W;
+    };
+    int q = 0;
+#define H2H_S(k) (ring + (k) * H2H_SLOT)
+#define H2H_I(k) H2H_S(((k) + H2H_NB - 1) % H2H_NB)
+#pragma unroll 1
+    for (; q + 6 <= nq; q += 6) {                  // slot of row q + k is k
+        row(q, H2H_S(0), H2H_I(0), tc0, tc1, tcx, ua, ub, uz, pa, pb);
+        row(q + 1, H2H_S(1), H2H_I(1), tc1, tcx, tc0, ub, uz, ua, pb, pa);
+        row(q + 2, H2H_S(2), H2H_I(2), tcx, tc0, tc1, uz, ua, ub, pa, pb);
+        row(q + 3, H2H_S(3), H2H_I(3), tc0, tc1, tcx, ua, ub, uz, pb, pa);
+        row(q + 4, H2H_S(4), H2H_I(4), tc1, tcx, tc0, ub, uz, ua, pa, pb);
+        row(q + 5, H2H_S(5), H2H_I(5), tcx, tc0, tc1, uz, ua, ub, pb, pa);
+    }
+#pragma unroll 1
+    for (; q < nq; ++q) {
+        row(q, H2H_S(q % H2H_NB), H2H_I(q % H2H_NB), tc0, tc1, tcx, ua, ub, uz, pa, pb);
+        tc0 = tc1;
+        tc1 = tcx;
+        ua = ub;
+        ub = uz;
+        pa = pb;
+    }
+#undef H2H_S
+#undef H2H_I
+    cp_async_wait<0>();
+    if (ye == H) {
+        const float4 o = step(ua, ub, ub, pa);
+        if (writer) *reinterpret_cast<float4 *>(orow) = o;
+    }
+}
+
+// T = 256 threads (32 x 8 warps): 120 output columns x 8 strips of H2_ROWS rows per CTA.
+extern "C" __global__ void __launch_bounds__(256) orion_hotspot2h_f32_256(orion_kargs a)
+{
+    ORION_PROBE(a);
+    const int ys = a.row_begin + (blockIdx.y * 8 + threadIdx.y) * H2_ROWS;
+    if (ys >= a.row_end) return;
+    const int ye = min(ys + H2_ROWS, a.row_end);
+    if (ye + 1 < a.height)
+        hotspot2h_strip<H2_ROWS, false>(a, ys, ye);
+    else
+        hotspot2h_strip<H2_ROWS, true>(a, ys, ye);
+}

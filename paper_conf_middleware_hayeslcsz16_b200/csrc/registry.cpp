@@ -70,6 +70,9 @@ static const KernelDef kKernels[] = {
     // two steps per launch (temporal blocking): reads 2 rows beyond its strip; width % 4 == 0
     // the rows each warp walks stream through a 6-slot cp.async ring: 8 warps x 6 x 272 floats
     {"hotspot2_f32", 256, "orion_hotspot2_f32_256", "hotspot", 32, 8, 128, 256, 2, K_STENCIL, 0, 8 * 6 * 272 * 4, 4, 2},
+    // two steps per launch with whole halo lanes: 120 output columns per warp, 6-slot ring of
+    // 8 warps x 6 x 256 floats
+    {"hotspot2h_f32", 256, "orion_hotspot2h_f32_256", "hotspot", 32, 8, 120, 256, 2, K_STENCIL, 0, 8 * 6 * 256 * 4, 4, 2},
     // srad: J tile (32+3)^2 + coefficient tile (32+1)^2 floats; reads 2 rows below the tile
     {"srad_f32_tile", 256, "orion_srad_f32_256", "srad", 32, 8, 32, 32, 2, K_SRAD, 0, (35 * 35 + 33 * 33) * 4},
     // srad, register-sliding: 124 x 128 tile; float4 lanes (width % 4 == 0) or scalar lanes;

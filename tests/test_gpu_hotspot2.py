@@ -1,4 +1,5 @@
-"""hotspot2_f32 (two explicit steps per launch, the intermediate step kept in registers):
+"""hotspot2_f32 / hotspot2h_f32 (two explicit steps per launch, the intermediate step kept in
+registers; edge lanes vs whole halo lanes):
 bit-identical to two launches of the one-step kernel and to the oracle's fp32 form, at every
 occupancy level, on ragged heights and at the image borders."""
 import numpy as np
@@ -13,11 +14,11 @@ pytestmark = pytest.mark.gpu
 from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
 
 
-@pytest.fixture(scope="module")
-def v2():
+@pytest.fixture(scope="module", params=["hotspot2_f32", "hotspot2h_f32"])
+def v2(request):
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
-    return O.build_all_levels(0, "hotspot2_f32", mode=O.REALISE_MIN_CARVEOUT)[0]
+    return O.build_all_levels(0, request.param, mode=O.REALISE_MIN_CARVEOUT)[0]
 
 
 def run(v, level, t0, pw, launches):
@@ -33,7 +34,8 @@ def run(v, level, t0, pw, launches):
     return a.cpu().numpy()
 
 
-@pytest.mark.parametrize("shape", [(300, 203), (128, 1), (132, 2), (260, 3), (512, 129), (4, 37)])
+@pytest.mark.parametrize("shape", [(300, 203), (128, 1), (132, 2), (260, 3), (512, 129), (4, 37), (120, 9),
+                                   (124, 40), (244, 33), (8, 70)])
 def test_two_steps_bit_exact_vs_oracle_fp32(v2, shape):
     W, H = shape
     t0, pw = synth.thermal_inputs(W, H, seed=5)

@@ -82,7 +82,8 @@ def test_query_limits_match_b200(dev):
 @pytest.mark.parametrize("kernel,threads", [("knn_f4", 128), ("knn_f4", 64), ("knn_f4", 256), ("nlm_f4", 128),
                                             ("nlm_f4_g1", 128), ("nlm_f4_direct", 128), ("nlm_f4_regheavy", 128),
                                             ("hotspot_f32", 256),
-                                            ("hotspot_f32", 128)])
+                                            ("hotspot_f32", 128), ("hotspot2_f32", 256), ("hotspot2h_f32", 256),
+                                            ("srad_f32", 256)])
 def test_every_level_realised_and_verified(dev, kernel, threads):
     v, res = variants(kernel, threads)
     planned = O.levels(O.b200_limits(), res)
@@ -240,6 +241,29 @@ def test_hotspot_full_size_crops(dev):
         cy0, cy1, cx0, cx1 = max(0, y0 - 1), min(H, y1 + 1), max(0, x0 - 1), min(W, x1 + 1)
         ref = oracle.hotspot(t0[cy0:cy1, cx0:cx1], pw[cy0:cy1, cx0:cx1], 1, precision="f32")
         assert np.array_equal(g[y0:y1, x0:x1], ref[y0 - cy0:y1 - cy0, x0 - cx0:x1 - cx0])
+
+
+@pytest.mark.parametrize("kernel", ["hotspot2_f32", "hotspot2h_f32"])
+def test_hotspot2_full_size_crops(dev, kernel):
+    # C3 size, one two-step launch at the level bench.py settles on and at max occupancy,
+    # checked on crops whose 2-cell margin makes the interior exact (every column block border
+    # of both kernels falls inside some crop: 120 / 128-column warps)
+    W = H = 8192
+    v, _ = variants(kernel)
+    t = torch.empty((H, W), device="cuda")
+    p = torch.empty((H, W), device="cuda")
+    o = torch.empty((H, W), device="cuda")
+    O.generate_thermal(0, t.data_ptr(), p.data_ptr(), W, H, seed=1, stream=stream())
+    t0, pw = synth.thermal_inputs(W, H, seed=1)
+    for lvl in (1 if len(v) > 1 else 0, len(v) - 1):
+        v.launch(lvl, O.hotspot_args(t.data_ptr(), o.data_ptr(), p.data_ptr(), W, H), stream())
+        torch.cuda.synchronize()
+        g = o.cpu().numpy()
+        for (y0, y1, x0, x1) in ((0, 40, 0, 40), (H - 40, H, W - 40, W), (4000, 4040, 110, 140),
+                                 (255, 290, 230, 262), (0, 30, 8100, W), (8150, H, 3830, 3850)):
+            cy0, cy1, cx0, cx1 = max(0, y0 - 2), min(H, y1 + 2), max(0, x0 - 2), min(W, x1 + 2)
+            ref = oracle.hotspot(t0[cy0:cy1, cx0:cx1], pw[cy0:cy1, cx0:cx1], 2, precision="f32")
+            assert np.array_equal(g[y0:y1, x0:x1], ref[y0 - cy0:y1 - cy0, x0 - cx0:x1 - cx0]), (lvl, y0, x0)
 
 
 def test_row_sharded_bit_identical_to_full(dev):
