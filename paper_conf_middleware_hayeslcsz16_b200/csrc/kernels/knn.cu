@@ -76,3 +76,8 @@ extern "C" __global__ void __launch_bounds__(128) orion_knn_f4_128(orion_kargs a
 extern "C" __global__ void __launch_bounds__(256) orion_knn_f4_256(orion_kargs a) { ORION_PROBE(a); knn_body<32, 8, 4>(a); }
 // T = 64 threads (8 x 8), the SDK's CTA shape, 32-row tiles.
 extern "C" __global__ void __launch_bounds__(64) orion_knn_f4_64(orion_kargs a) { ORION_PROBE(a); knn_body<8, 8, 4>(a); }
+// One pixel per thread (PY = 1): 4x the threads of the strip kernels for the same frame and a
+// quarter of the serial tap chain per thread -- small, launch- and latency-bound frames (C1:
+// 64 x 64 = 32 CTAs instead of 8).  Same per-pixel tap order, so the same bits.
+extern "C" __global__ void __launch_bounds__(128) orion_knn1_f4_128(orion_kargs a) { ORION_PROBE(a); knn_body<32, 4, 1>(a); }
+extern "C" __global__ void __launch_bounds__(64) orion_knn1_f4_64(orion_kargs a) { ORION_PROBE(a); knn_body<8, 8, 1>(a); }

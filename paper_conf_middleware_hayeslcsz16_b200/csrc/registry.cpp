@@ -49,6 +49,9 @@ static const KernelDef kKernels[] = {
     {"knn_f4", 128, "orion_knn_f4_128", "knn", 32, 4, 32, 16, 3, K_KNN, 1, 0, 1, 1, 1},
     {"knn_f4", 256, "orion_knn_f4_256", "knn", 32, 8, 32, 32, 3, K_KNN, 1, 0, 1, 1, 1},
     {"knn_f4", 64, "orion_knn_f4_64", "knn", 8, 8, 8, 32, 3, K_KNN, 1, 0, 1, 1, 1},
+    // one pixel per thread: small (launch-bound) frames
+    {"knn_f4_p1", 128, "orion_knn1_f4_128", "knn", 32, 4, 32, 4, 3, K_KNN, 1, 0, 1, 1, 1},
+    {"knn_f4_p1", 64, "orion_knn1_f4_64", "knn", 8, 8, 8, 8, 3, K_KNN, 1, 0, 1, 1, 1},
     // nlm_box: 3 planar (122+18) x (23+12) fp32 planes (pitch 141) + 32 x 129 floats of H_o
     // up to 3 offset pairs per pass: 3 H_o buffers (2 CTAs/SM) -- the C2 / C5 default
     {"nlm_f4", 128, "orion_nlm_box3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,

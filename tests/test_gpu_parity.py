@@ -79,7 +79,8 @@ def test_query_limits_match_b200(dev):
         assert getattr(d, f) == getattr(n, f), f
 
 
-@pytest.mark.parametrize("kernel,threads", [("knn_f4", 128), ("knn_f4", 64), ("knn_f4", 256), ("nlm_f4", 128),
+@pytest.mark.parametrize("kernel,threads", [("knn_f4", 128), ("knn_f4", 64), ("knn_f4", 256), ("knn_f4_p1", 128),
+                                            ("nlm_f4", 128),
                                             ("nlm_f4_g1", 128), ("nlm_f4_direct", 128), ("nlm_f4_regheavy", 128),
                                             ("hotspot_f32", 256),
                                             ("hotspot_f32", 128), ("hotspot2_f32", 256), ("hotspot2h_f32", 256),
@@ -115,11 +116,12 @@ def test_generator_bit_identical(dev):
     assert np.array_equal(t0.cpu().numpy(), rt) and np.array_equal(pw.cpu().numpy(), rp)
 
 
-@pytest.mark.parametrize("threads", [128, 64, 256])
-def test_knn_c1_all_levels(dev, threads):
+@pytest.mark.parametrize("kernel,threads", [("knn_f4", 128), ("knn_f4", 64), ("knn_f4", 256), ("knn_f4_p1", 128),
+                                            ("knn_f4_p1", 64)])
+def test_knn_c1_all_levels(dev, kernel, threads):
     # C1: KNN 64x64 RGBA, radius 3, all feasible occupancy levels vs the oracle
     img = synth.noisy_rgba(64, 64, seed=1, sigma=0.2)
-    outs = run_denoise("knn_f4", img, threads)
+    outs = run_denoise(kernel, img, threads)
     for o in outs[1:]:
         assert np.array_equal(o, outs[0])                               # bit-exact across levels
     out, alt, amb = oracle.denoise("knn", img)
@@ -133,6 +135,8 @@ def test_knn_ragged_and_degenerate(dev, shape):
     v, _ = variants("knn_f4")
     outs = run_denoise("knn_f4", img, level=len(v) - 1) + run_denoise("knn_f4", img, level=0)
     assert np.array_equal(outs[0], outs[1])
+    v1, _ = variants("knn_f4_p1")                     # one pixel per thread: the same bits
+    assert np.array_equal(run_denoise("knn_f4_p1", img, level=len(v1) - 1)[0], outs[0])
     out, alt, amb = oracle.denoise("knn", img)
     check_vs_oracle(outs[0], out, alt, amb)
 
