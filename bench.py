@@ -45,8 +45,8 @@ WORKLOADS = {
     # register-heavy direct NLM: 2401 patch terms x 6 + 49 x 6 per-offset terms + blend
     "c4": dict(kernel="nlm_f4_regheavy", W=4096, H=4096, sigma=0.13, unit="Mpix/s",
                name="register-heavy NLM 4096x4096 RGBA, maxrregcount caps", insts=2401 * 6 + 49 * 6 + 10, bytes=32),
-    # thermal stencil: two explicit steps per launch (hotspot2h_f32), 12 B per cell per launch
-    "c3": dict(kernel="hotspot2h_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
+    # thermal stencil: four explicit steps per launch (hotspot4h_f32), 12 B per cell per launch
+    "c3": dict(kernel="hotspot4h_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
                insts=12, bytes=12),
     # NEXT-4: a second Rodinia stencil (srad), 8 B/cell-iteration (read J, write J')
     "srad": dict(kernel="srad_f32", W=8192, H=8192, unit="Mcell-steps/s", name="SRAD 8192x8192 fp32 (NEXT-4)",
@@ -428,7 +428,7 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     final, iters_to_final = tuner.final()
-    spl = 2 if kernel.startswith("hotspot2") else 1        # stencil steps per launch (temporal blocking)
+    spl = O.STEPS_PER_LAUNCH.get(kernel, 1)                # stencil steps per launch (temporal blocking)
     units_per_step = W * H * spl
     value = world * units_per_step * args.steps / (total_ms * 1e-3) / 1e6
     ms_step = total_ms / args.steps

@@ -125,7 +125,8 @@ orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int bloc
  * "nlm_f4_g1" (1 pair per pass), "nlm_f4_direct", "nlm_f4_regheavy" (T = 128 / 64),
  * "hotspot_f32" (T = 256 / 128), "hotspot2_f32" (two stencil steps per launch, edge lanes fetch
  * the outer columns; width % 4 == 0), "hotspot2h_f32" (two steps per launch, whole halo lanes:
- * 120 output columns per warp; width % 4 == 0; the C3 default),
+ * 120 output columns per warp; width % 4 == 0), "hotspot4h_f32" (four steps per launch, the same
+ * halo-lane warps as a 4-stage register pipeline; width % 4 == 0; the C3 default),
  * "srad_f32" (register-sliding, any width), "srad_f32_tile" (shared-memory form, same bits).
  * block_threads = 0 selects the kernel's default CTA size.  Fills the natural resources
  * (compiles the kernel's PTX once, uncapped, with the embedded ptxas). */
@@ -276,7 +277,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
 /* A whole iterative stencil run end to end from HOST buffers -- the Rodinia driver shape
  * (copy the grid in, iterate, copy it out), the iterations being the ones
  * Fig. 9 tunes across (P:L651-P:L653).  Kernels of kind hotspot ("hotspot_f32",
- * "hotspot2_f32", "hotspot2h_f32") and srad ("srad_f32", "srad_f32_tile") only, whole grids only
+ * "hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32") and srad ("srad_f32", "srad_f32_tile") only, whole grids only
  * (a->row_begin = a->src_row_begin = a->dst_row_begin = 0, a->row_end = a->src_row_end =
  * a->height).
  *   a->src  host initial grid (fp32, width x height, row-major; pinned for async copies)
@@ -286,7 +287,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
  *   dev_aux hotspot: device power map buffer (filled here); srad: the device float q0sqr
  *   roi     srad only: {r1, r2, c1, c2} of the ROI statistics run before every iteration
  * Copies in, runs `iterations` orion_tune_step iterations on `stream` (hotspot2_f32 / hotspot2h_f32 advance
- * two time steps per iteration), copies the final grid out and synchronises the stream.
+ * two time steps per iteration, hotspot4h_f32 four), copies the final grid out and synchronises the stream.
  * Bytes copied are returned in *h2d_bytes / *d2h_bytes.  ORION_E_INVALID on other kernels,
  * partial row ranges or missing buffers. */
 orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterations, void *dev_a, void *dev_b,

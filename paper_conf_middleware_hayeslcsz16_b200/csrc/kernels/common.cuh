@@ -65,6 +65,21 @@ ORION_DEVICE void load_tile_clamped(float4 *tile, const orion_kargs &a, int gx0,
     }
 }
 
+// cp.async (LDGSTS) of 8 / 4 bytes global -> shared: no registers, every copy of a thread in
+// flight at once (one memory latency for a whole staged tile instead of one per unrolled
+// batch of register loads).  Completed by cp_async_wait_all() + a barrier.
+ORION_DEVICE void cpa8(void *sdst, const void *gsrc)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+                 "l"(gsrc) : "memory");
+}
+ORION_DEVICE void cpa4(void *sdst, const void *gsrc)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+                 "l"(gsrc) : "memory");
+}
+ORION_DEVICE void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+
 // Output pixel (x, y) (global row y) into dst (rows from dst_row_begin).
 ORION_DEVICE void store_out(const orion_kargs &a, int x, int y, float4 o)
 {

@@ -458,3 +458,152 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2h_f32_256(orion_
     else
         hotspot2h_strip<H2_ROWS, true>(a, ys, ye);
 }
+
+// ---- S steps per launch, halo lanes (hotspot4h: S = 4) -------------------------------------
+// hotspot2h's layout carried to S <= 4 steps: a warp loads 128 consecutive columns
+// [base-4, base+124) as float4 lanes and writes the 120 columns of lanes 1..30.  Step s's valid
+// columns shrink by one per side per step and lanes 0 / 31 hold 4 halo columns each, so 4 steps
+// fit.  Vertically the warp walks its strip of HS_ROWS rows as a pipeline over iterations
+// t = ys-S .. ye-1+S: T0 row t arrives from the ring, then step s computes its row t-s from step
+// s-1's rows t-s-1 .. t-s+1 (kept in registers, 3 float4 per step; stage s only from iteration
+// 2s on, earlier rows being outside what stage s+1 needs), and step S's row t-S is the output.
+// Per launch the kernel reads T0 and P once and writes T_S once: 12 B of DRAM per cell for S
+// cell-steps (+ S/HS_ROWS re-read halo rows).  Strips touching row 0 or H-1 take the EDGE form,
+// which clamps each step's N / S neighbour at rows 0 / H-1 to the cell itself (the T0 rows
+// beyond the grid are clamped loads); warps holding column 0 or W-1 take the CEDGE form (the
+// clamped E / W neighbour).  Every cell is hs_cell4's operation sequence with clamp-to-edge
+// neighbours: bit-identical to S one-step launches.
+//
+// The ring: slot q holds the T0 and P rows of iteration q, fetched D = NB-S-1 iterations ahead
+// by cp.async, and lives until step S has read its P row, S iterations later, so the power rows
+// need no registers.  The loop body is NB rows (NB % 3 == 0: the step windows rotate with period
+// 3), so every slot offset is a compile-time constant.  Measured on C3 (8192^2, A/B on one box):
+// power rows in registers 0.1599 ms per launch, from the ring 0.1559; a 12-row body 0.176
+// (instruction-cache bound); 32-row strips 0.1623 (more halo recompute); odd warps walking
+// upwards (halo rows read by both neighbours at the same time: 549 instead of 604 MB of DRAM
+// reads) 0.1600 -- the kernel is bound by issue and latency at 4 warps per scheduler, not DRAM.
+#ifndef HS_ROWS
+#define HS_ROWS 64
+#endif
+namespace {
+constexpr int HS_SLOT = 256;                // floats: T0 row segment (128) + P row segment (128)
+}  // namespace
+
+template <int S, int NB, bool EDGE, bool CEDGE>
+__device__ __forceinline__ void hotspotS_strip(const orion_kargs &a, int ys, int ye)
+{
+    static_assert(S >= 1 && S <= 4, "one float4 halo lane per side carries at most 4 steps");
+    static_assert(NB % 3 == 0 && NB - S - 1 >= 1 && 2 * S < NB, "ring: NB-S-1 rows in flight, body of NB rows");
+    constexpr int D = NB - S - 1;
+    extern __shared__ float4 smem4[];
+    const int W = a.width, H = a.height;
+    const int lane = threadIdx.x;
+    const float c[5] = {a.fparam[0], a.fparam[1], a.fparam[2], a.fparam[3], a.fparam[4]};
+    const int base = blockIdx.x * 120;
+    const int cx = base - 4 + 4 * lane;
+    const int cxl = clampi(cx, 0, W - 4);
+    const bool writer = lane >= 1 && lane <= 30 && cx < W;
+    const bool wclamp = cx == 0, eclamp = cx + 4 >= W;
+    const float *t0 = (const float *)a.src - (size_t)a.src_row_begin * (size_t)W + cxl;
+    const float *p0 = (const float *)a.aux - (size_t)a.src_row_begin * (size_t)W + cxl;
+    float *ring = reinterpret_cast<float *>(smem4) + threadIdx.y * (NB * HS_SLOT) + 4 * lane;
+    const int nq = (ye - ys) + 2 * S;              // iterations t = ys-S .. ye-1+S
+    int rt = ys - S;                               // row of the next issue (T0 and P)
+    const float *tn = t0 + (ptrdiff_t)rt * W, *pn = p0 + (ptrdiff_t)rt * W;   // interior strips
+    auto issue = [&](float *sl) {
+        if (EDGE) {
+            const size_t o = (size_t)clampi(rt, 0, H - 1) * (size_t)W;
+            cp_async16(sl, t0 + o);
+            cp_async16(sl + 128, p0 + o);
+            ++rt;
+        } else {
+            cp_async16(sl, tn);
+            cp_async16(sl + 128, pn);
+            tn += W;
+            pn += W;
+        }
+    };
+#pragma unroll
+    for (int q = 0; q < D; ++q) {
+        if (q < nq) issue(ring + q * HS_SLOT);
+        cp_async_commit();
+    }
+    float4 X[S][3];
+#pragma unroll
+    for (int s = 0; s < S; ++s) X[s][0] = X[s][1] = X[s][2] = make_float4(0.f, 0.f, 0.f, 0.f);
+    float *orow = (float *)a.dst + (size_t)cx + ((size_t)ys - (size_t)a.dst_row_begin) * (size_t)W;
+    int t = ys - S;                                // T0 row arriving this iteration
+    // iteration q, kq = q % NB (a constant inside the unrolled body), steps 1 .. smin
+    auto row = [&](int q, int kq, int smin) {
+        if (q + D < nq) issue(ring + ((kq + D) % NB) * HS_SLOT);
+        cp_async_commit();
+        cp_async_wait<D>();
+        X[0][0] = X[0][1];
+        X[0][1] = X[0][2];
+        X[0][2] = *reinterpret_cast<const float4 *>(ring + kq * HS_SLOT);            // T0(t)
+#pragma unroll
+        for (int s = 1; s <= S; ++s) {
+            if (s > smin) continue;
+            float4 Nv = X[s - 1][0], Tv = X[s - 1][1], Sv = X[s - 1][2];             // rows t-s-1 .. t-s+1
+            if (EDGE) {
+                const int r = t - s;
+                if (r == 0) Nv = Tv;
+                if (r == H - 1) Sv = Tv;
+            }
+            float Wv = __shfl_up_sync(0xffffffffu, Tv.w, 1);
+            float Ev = __shfl_down_sync(0xffffffffu, Tv.x, 1);
+            if (CEDGE) {
+                if (wclamp) Wv = Tv.x;
+                if (eclamp) Ev = Tv.w;
+            }
+            const float4 Pv = *reinterpret_cast<const float4 *>(ring + ((kq - s + NB) % NB) * HS_SLOT + 128);
+            const float4 o = hs_cell4(Tv, Nv, Sv, Ev, Wv, Pv, c);                   // T_s(t-s)
+            if (s < S) {
+                X[s][0] = X[s][1];
+                X[s][1] = X[s][2];
+                X[s][2] = o;
+            } else {                                                                   // row t-S >= ys
+                if (writer) *reinterpret_cast<float4 *>(orow) = o;
+                orow += W;
+            }
+        }
+        ++t;
+    };
+    // nq >= 2S + 1 always (a strip has >= 1 row)
+#pragma unroll
+    for (int q = 0; q < 2 * S; ++q) row(q, q, q / 2);
+    int q = 2 * S;
+#pragma unroll
+    for (int k = 2 * S; k < NB; ++k, ++q)          // up to the first multiple of NB
+        if (q < nq) row(q, k, S);
+#pragma unroll 1
+    for (; q + NB <= nq; q += NB) {
+#pragma unroll
+        for (int k = 0; k < NB; ++k) row(q + k, k, S);
+    }
+#pragma unroll 1
+    for (; q < nq; ++q) row(q, q % NB, S);
+    cp_async_wait<0>();
+}
+
+template <int S, int RY, int NB>
+__device__ __forceinline__ void hotspotS_body(const orion_kargs &a)
+{
+    const int ys = a.row_begin + (blockIdx.y * 8 + threadIdx.y) * RY;
+    if (ys >= a.row_end) return;
+    const int ye = min(ys + RY, a.row_end);
+    const bool redge = ys - S < 0 || ye - 1 + S > a.height - 1;
+    const bool cedge = blockIdx.x == 0 || (int)blockIdx.x * 120 + 124 >= a.width;
+    if (!redge && !cedge)
+        hotspotS_strip<S, NB, false, false>(a, ys, ye);
+    else
+        hotspotS_strip<S, NB, true, true>(a, ys, ye);
+}
+
+// T = 256 threads (32 x 8 warps): 120 output columns x 8 strips of HS_ROWS rows per CTA; 4 steps
+// per launch, 9-slot ring (4 rows in flight) per warp.
+extern "C" __global__ void __launch_bounds__(256) orion_hotspot4h_f32_256(orion_kargs a)
+{
+    ORION_PROBE(a);
+    hotspotS_body<4, HS_ROWS, 9>(a);
+}

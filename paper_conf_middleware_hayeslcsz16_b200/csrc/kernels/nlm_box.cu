@@ -309,16 +309,19 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
     const int lane = tid & 31, warp = tid >> 5;
     const int x0 = blockIdx.x * TW;
     const int y0 = a.row_begin + blockIdx.y * TH;
-    {   // stage the planar tile (coalesced float4 loads, clamp-to-edge in global coords)
+    {   // stage the planar tile (clamp-to-edge in global coords): per pixel one 8-byte (r, g)
+        // and one 4-byte b cp.async, all of the thread's copies in flight at once
         const float4 *src = (const float4 *)a.src;
+#pragma unroll 4
         for (int idx = tid; idx < PC * PR; idx += NT) {
             const int ty = idx / PC, tx = idx - ty * PC;
             const int gx = clampi(x0 - 9 + tx, 0, a.width - 1);
             const int gy = clampi(y0 - 6 + ty, 0, a.height - 1);
-            const float4 v = __ldg(src + (size_t)(gy - a.src_row_begin) * (size_t)a.width + gx);
-            prg[ty * PW + tx] = make_float2(v.x, v.y);
-            pb[ty * PW + tx] = v.z;
+            const float *g = (const float *)(src + (size_t)(gy - a.src_row_begin) * (size_t)a.width + gx);
+            cpa8(prg + ty * PW + tx, g);
+            cpa4(pb + ty * PW + tx, g + 2);
         }
+        cp_async_wait_all();
     }
     __syncthreads();
 

@@ -143,15 +143,17 @@ extern "C" __global__ void __launch_bounds__(256) orion_nlm_box256_f4_256(orion_
     const int y0 = a.row_begin + blockIdx.y * TH;
     {
         const float4 *src = (const float4 *)a.src;
+#pragma unroll 4
         for (int idx = tid; idx < PC * PR; idx += NT) {
             const int ty = idx / PC, tx = idx - ty * PC;
             const int gx = clampi(x0 - 9 + tx, 0, a.width - 1);
             const int gy = clampi(y0 - 6 + ty, 0, a.height - 1);
-            const float4 v = __ldg(src + (size_t)(gy - a.src_row_begin) * (size_t)a.width + gx);
-            pr[ty * PW + tx] = v.x;
-            pg[ty * PW + tx] = v.y;
-            pb[ty * PW + tx] = v.z;
+            const float *g = (const float *)(src + (size_t)(gy - a.src_row_begin) * (size_t)a.width + gx);
+            cpa4(pr + ty * PW + tx, g);        // cp.async: all copies in flight at once
+            cpa4(pg + ty * PW + tx, g + 1);
+            cpa4(pb + ty * PW + tx, g + 2);
         }
+        cp_async_wait_all();
     }
     __syncthreads();
 

@@ -137,7 +137,7 @@ def test_replay_random_tables_match_oracle(shape, seed, mode, switch, expected, 
     assert fit == (tr.final_iteration if tr.final_iteration is not None else -1)
 
 
-@pytest.mark.parametrize("kernel", ["knn_f4", "nlm_f4", "nlm_f4_regheavy", "hotspot_f32", "hotspot2h_f32", "srad_f32"])
+@pytest.mark.parametrize("kernel", ["knn_f4", "nlm_f4", "nlm_f4_regheavy", "hotspot_f32", "hotspot2h_f32", "hotspot4h_f32", "srad_f32"])
 def test_embedded_ptxas_honours_register_caps(kernel):
     res = O.kernel_probe(kernel)
     assert res.regs_per_thread > 0 and res.block_threads in (64, 128, 256)

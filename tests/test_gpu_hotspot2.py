@@ -1,5 +1,6 @@
 """hotspot2_f32 / hotspot2h_f32 (two explicit steps per launch, the intermediate step kept in
-registers; edge lanes vs whole halo lanes):
+registers; edge lanes vs whole halo lanes) and hotspot4h_f32 (four steps per launch, a 4-stage
+register pipeline on the halo-lane warps):
 bit-identical to two launches of the one-step kernel and to the oracle's fp32 form, at every
 occupancy level, on ragged heights and at the image borders."""
 import numpy as np
@@ -14,11 +15,13 @@ pytestmark = pytest.mark.gpu
 from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
 
 
-@pytest.fixture(scope="module", params=["hotspot2_f32", "hotspot2h_f32"])
+@pytest.fixture(scope="module", params=["hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32"])
 def v2(request):
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
-    return O.build_all_levels(0, request.param, mode=O.REALISE_MIN_CARVEOUT)[0]
+    v = O.build_all_levels(0, request.param, mode=O.REALISE_MIN_CARVEOUT)[0]
+    v.spl = O.STEPS_PER_LAUNCH[request.param]
+    return v
 
 
 def run(v, level, t0, pw, launches):
@@ -39,7 +42,7 @@ def run(v, level, t0, pw, launches):
 def test_two_steps_bit_exact_vs_oracle_fp32(v2, shape):
     W, H = shape
     t0, pw = synth.thermal_inputs(W, H, seed=5)
-    ref = oracle.hotspot(t0, pw, 10, precision="f32")
+    ref = oracle.hotspot(t0, pw, 5 * v2.spl, precision="f32")
     for lvl in (0, len(v2) - 1):
         assert np.array_equal(run(v2, lvl, t0, pw, 5), ref), (shape, lvl)
 
@@ -49,7 +52,7 @@ def test_all_levels_identical(v2):
     outs = [run(v2, i, t0, pw, 3) for i in range(len(v2))]
     for o in outs[1:]:
         assert np.array_equal(o, outs[0])
-    assert np.array_equal(outs[0], oracle.hotspot(t0, pw, 6, precision="f32"))
+    assert np.array_equal(outs[0], oracle.hotspot(t0, pw, 3 * v2.spl, precision="f32"))
 
 
 def test_unaligned_width_rejected(v2):

@@ -84,7 +84,7 @@ def test_query_limits_match_b200(dev):
                                             ("nlm_f4_g1", 128), ("nlm_f4_direct", 128), ("nlm_f4_regheavy", 128),
                                             ("hotspot_f32", 256),
                                             ("hotspot_f32", 128), ("hotspot2_f32", 256), ("hotspot2h_f32", 256),
-                                            ("srad_f32", 256)])
+                                            ("hotspot4h_f32", 256), ("srad_f32", 256)])
 def test_every_level_realised_and_verified(dev, kernel, threads):
     v, res = variants(kernel, threads)
     planned = O.levels(O.b200_limits(), res)
@@ -247,7 +247,7 @@ def test_hotspot_full_size_crops(dev):
         assert np.array_equal(g[y0:y1, x0:x1], ref[y0 - cy0:y1 - cy0, x0 - cx0:x1 - cx0])
 
 
-@pytest.mark.parametrize("kernel", ["hotspot2_f32", "hotspot2h_f32"])
+@pytest.mark.parametrize("kernel", ["hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32"])
 def test_hotspot2_full_size_crops(dev, kernel):
     # C3 size, one two-step launch at the level bench.py settles on and at max occupancy,
     # checked on crops whose 2-cell margin makes the interior exact (every column block border
@@ -263,10 +263,11 @@ def test_hotspot2_full_size_crops(dev, kernel):
         v.launch(lvl, O.hotspot_args(t.data_ptr(), o.data_ptr(), p.data_ptr(), W, H), stream())
         torch.cuda.synchronize()
         g = o.cpu().numpy()
+        n = O.STEPS_PER_LAUNCH[kernel]
         for (y0, y1, x0, x1) in ((0, 40, 0, 40), (H - 40, H, W - 40, W), (4000, 4040, 110, 140),
                                  (255, 290, 230, 262), (0, 30, 8100, W), (8150, H, 3830, 3850)):
-            cy0, cy1, cx0, cx1 = max(0, y0 - 2), min(H, y1 + 2), max(0, x0 - 2), min(W, x1 + 2)
-            ref = oracle.hotspot(t0[cy0:cy1, cx0:cx1], pw[cy0:cy1, cx0:cx1], 2, precision="f32")
+            cy0, cy1, cx0, cx1 = max(0, y0 - n), min(H, y1 + n), max(0, x0 - n), min(W, x1 + n)
+            ref = oracle.hotspot(t0[cy0:cy1, cx0:cx1], pw[cy0:cy1, cx0:cx1], n, precision="f32")
             assert np.array_equal(g[y0:y1, x0:x1], ref[y0 - cy0:y1 - cy0, x0 - cx0:x1 - cx0]), (lvl, y0, x0)
 
 
