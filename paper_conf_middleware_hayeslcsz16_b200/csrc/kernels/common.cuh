@@ -78,6 +78,11 @@ ORION_DEVICE void cpa4(void *sdst, const void *gsrc)
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
                  "l"(gsrc) : "memory");
 }
+ORION_DEVICE void cpa16(void *sdst, const void *gsrc)
+{
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+                 "l"(gsrc) : "memory");
+}
 ORION_DEVICE void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
 // Output pixel (x, y) (global row y) into dst (rows from dst_row_begin).

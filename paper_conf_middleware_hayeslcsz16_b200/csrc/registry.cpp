@@ -27,6 +27,7 @@ extern "C" const char liborion_ptx_hotspot[];
 extern "C" const char liborion_ptx_gen[];
 extern "C" const char liborion_ptx_srad[];
 extern "C" const char liborion_ptx_nlm_box256[];
+extern "C" const char liborion_ptx_nlm_box4[];
 
 namespace orion {
 
@@ -40,6 +41,7 @@ static const char *module_ptx(const char *module)
     if (!std::strcmp(module, "gen")) return liborion_ptx_gen;
     if (!std::strcmp(module, "srad")) return liborion_ptx_srad;
     if (!std::strcmp(module, "nlm_box256")) return liborion_ptx_nlm_box256;
+    if (!std::strcmp(module, "nlm_box4")) return liborion_ptx_nlm_box4;
     return nullptr;
 }
 
@@ -56,6 +58,9 @@ static const KernelDef kKernels[] = {
     // up to 3 offset pairs per pass: 3 H_o buffers (2 CTAs/SM) -- the C2 / C5 default
     {"nlm_f4", 128, "orion_nlm_box3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
      3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},
+    // (r, g, b, 1) float4 tile plane (pitch 141) + 2 H_o buffers, two pairs per pass (2 CTAs/SM)
+    {"nlm_f4_q", 128, "orion_nlm_box4_f4_128", "nlm_box4", 128, 1, 122, 23, 6, K_NLM, 0,
+     35 * 141 * 16 + 2 * 32 * 129 * 4, 1, 1, 1},
     // same, integer (fixed-point, exact) box sums
     {"nlm_f4_i", 128, "orion_nlm_boxi3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
      3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},
