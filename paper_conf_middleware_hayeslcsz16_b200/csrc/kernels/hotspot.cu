@@ -481,7 +481,11 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2h_f32_256(orion_
 // power rows in registers 0.1599 ms per launch, from the ring 0.1559; a 12-row body 0.176
 // (instruction-cache bound); 32-row strips 0.1623 (more halo recompute); odd warps walking
 // upwards (halo rows read by both neighbours at the same time: 549 instead of 604 MB of DRAM
-// reads) 0.1600 -- the kernel is bound by issue and latency at 4 warps per scheduler, not DRAM.
+// reads) 0.1600; a 12-slot ring (7 rows in flight, 12-row body) 0.178; a 3-row body carrying
+// the slot index 0.161; a persistent grid (one wave, each warp one ~240-row strip: 560 instead
+// of 604 MB of DRAM reads, no partial wave) 0.1665 vs 0.1550 -- fewer DRAM bytes alone do not
+// make this kernel faster; at 4 warps per scheduler it is bound by issue and latency as much as
+// by DRAM (long-scoreboard 1.9 stalls per issue on the ring waits, FMA pipe 56 % busy).
 #ifndef HS_ROWS
 #define HS_ROWS 64
 #endif
