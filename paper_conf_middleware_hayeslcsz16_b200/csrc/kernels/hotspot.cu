@@ -158,16 +158,16 @@ constexpr int H2_SLOT = 136 + 136;          // floats: T0 segment [base-4, base+
 __device__ __forceinline__ void cp_async16(float *sdst, const float *gsrc)
 {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
-                 "l"(gsrc));
+                 "l"(gsrc) : "memory");
 }
 __device__ __forceinline__ void cp_async4(float *sdst, const float *gsrc)
 {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
-                 "l"(gsrc));
+                 "l"(gsrc) : "memory");
 }
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
 
 // Edge handling without per-row selects on the block position: the edge lanes' outer columns
 // are clamped in global coordinates, and at the west edge lane 0's outer T1 cell is made to be

@@ -231,16 +231,16 @@ constexpr int SRAD_SLOT = 132;  // floats per slot: 32 lanes x up to 4 columns +
 __device__ __forceinline__ void srad_cp16(float *sdst, const float *gsrc)
 {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
-                 "l"(gsrc));
+                 "l"(gsrc) : "memory");
 }
 __device__ __forceinline__ void srad_cp4(float *sdst, const float *gsrc)
 {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
-                 "l"(gsrc));
+                 "l"(gsrc) : "memory");
 }
-__device__ __forceinline__ void srad_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+__device__ __forceinline__ void srad_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 template <int N>
-__device__ __forceinline__ void srad_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+__device__ __forceinline__ void srad_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
 
 namespace {
 template <int V>
