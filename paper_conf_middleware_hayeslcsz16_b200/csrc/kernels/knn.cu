@@ -81,3 +81,56 @@ extern "C" __global__ void __launch_bounds__(64) orion_knn_f4_64(orion_kargs a) 
 // 64 x 64 = 32 CTAs instead of 8).  Same per-pixel tap order, so the same bits.
 extern "C" __global__ void __launch_bounds__(128) orion_knn1_f4_128(orion_kargs a) { ORION_PROBE(a); knn_body<32, 4, 1>(a); }
 extern "C" __global__ void __launch_bounds__(64) orion_knn1_f4_64(orion_kargs a) { ORION_PROBE(a); knn_body<8, 8, 1>(a); }
+
+// ---- tap-split form (knn_f4_t8): 8 threads per pixel ------------------------------------------
+// Small frames (C1: 64 x 64 = 4096 pixels) are latency-bound: one pixel per thread still walks
+// a serial chain of 49 taps on 32 of 148 SMs.  Here the 49 taps of a pixel are split over the 8
+// lanes of a lane group (lane g takes taps k = g, g+8, ..., k -> (i, j) = (k/7 - 3, k%7 - 3)),
+// read straight from global memory (clamp-to-edge in global coordinates; the frame is L1 / L2
+// resident), and the 8 partial sums are combined by a fixed xor-shuffle tree (offsets 4, 2, 1)
+// whose result lane 0 of the group writes.  Every weight is computed exactly as in knn_body
+// (same tap arithmetic), so the counts -- hence the lerp branch -- are the same; only the order
+// of the weighted sums differs (within the 1e-5 tolerance; bit-identical across occupancy
+// levels, which share this code).  CTA = 128 threads = 16 pixels of one row.
+__device__ __forceinline__ void knn_t8_body(const orion_kargs &a)
+{
+    const int g = threadIdx.x & 7;
+    const int x = blockIdx.x * 16 + (threadIdx.x >> 3);
+    const int y = a.row_begin + blockIdx.y;
+    const int W = a.width, H = a.height;
+    const int xc = min(x, W - 1);
+    const float4 *src = (const float4 *)a.src - (size_t)a.src_row_begin * (size_t)W;
+    const float nl2 = a.fparam[0];
+    const float wthr = a.fparam[2];
+    const float4 c00 = __ldg(src + (size_t)y * (size_t)W + xc);
+    float ax = 0.0f, ay = 0.0f, az = 0.0f, sw = 0.0f;
+    int cnt = 0;
+#pragma unroll
+    for (int s = 0; s < 7; ++s) {
+        const int k = g + 8 * s;
+        if (k >= KNN_A) break;                     // only lane 0 of a group has a 7th tap (k = 48)
+        const int i = k / 7 - KNN_R, j = k % 7 - KNN_R;
+        const int gy = clampi(y + i, 0, H - 1), gx = clampi(xc + j, 0, W - 1);
+        const float4 c = __ldg(src + (size_t)gy * (size_t)W + gx);
+        const float d = dist2(c, c00);
+        const float w = ex2(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
+        ax = __fmaf_rn(w, c.x, ax);
+        ay = __fmaf_rn(w, c.y, ay);
+        az = __fmaf_rn(w, c.z, az);
+        sw = __fadd_rn(sw, w);
+        cnt += (w > wthr);
+    }
+#pragma unroll
+    for (int o = 4; o > 0; o >>= 1) {
+        ax = __fadd_rn(ax, __shfl_xor_sync(0xffffffffu, ax, o));
+        ay = __fadd_rn(ay, __shfl_xor_sync(0xffffffffu, ay, o));
+        az = __fadd_rn(az, __shfl_xor_sync(0xffffffffu, az, o));
+        sw = __fadd_rn(sw, __shfl_xor_sync(0xffffffffu, sw, o));
+        cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+    }
+    if (g == 0 && x < W) {
+        store_out(a, x, y, lerp_out(c00, ax, ay, az, sw, cnt, a));
+        fanout_column(a, x, y, y + 1);
+    }
+}
+extern "C" __global__ void __launch_bounds__(128) orion_knn8_f4_128(orion_kargs a) { ORION_PROBE(a); knn_t8_body(a); }
