@@ -169,7 +169,8 @@ extern "C" __global__ void __launch_bounds__(256) orion_srad_f32_256(orion_kargs
 }
 
 // ROI statistics: one CTA of 1024 threads; thread t sums elements t, t+1024, ... of the
-// row-major ROI in double (4 loads in flight), then a fixed-shape shuffle tree per warp and
+// row-major ROI in double (16 loads in flight: the default 128 x 128 ROI is one batch, one
+// memory latency), then a fixed-shape shuffle tree per warp and
 // across the 32 warp sums -- deterministic, so every occupancy variant of the update kernel
 // sees the same q0sqr.
 extern "C" __global__ void __launch_bounds__(1024) orion_srad_stats(const float *J, int W, int r1, int r2, int c1,
@@ -179,7 +180,7 @@ extern "C" __global__ void __launch_bounds__(1024) orion_srad_stats(const float 
     const int t = threadIdx.x;
     const int rw = c2 - c1 + 1, n = (r2 - r1 + 1) * rw;
     double a = 0.0, b = 0.0;
-#pragma unroll 4
+#pragma unroll 16
     for (int e = t; e < n; e += 1024) {
         const int i = r1 + e / rw, j = c1 + e % rw;
         const double v = __ldg(J + (size_t)i * (size_t)W + j);
