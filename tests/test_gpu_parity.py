@@ -184,7 +184,7 @@ def _sample_points(W, H, n, seed):
     return np.array(xs), np.array(ys)
 
 
-@pytest.mark.parametrize("kernel,size", [("nlm_f4", 2048), ("nlm_f4_q", 2048), ("nlm_f4_i", 2048), ("knn_f4", 2048),
+@pytest.mark.parametrize("kernel,size", [("nlm_f4", 2048), ("nlm_f4_q", 2048), ("nlm_f4_i", 2048), ("knn_f4", 2048), ("knn_f4_t8", 2048),
                                          ("nlm_f4_regheavy", 4096)])
 def test_full_size_sampled(dev, kernel, size):
     # C2 / C4 sizes, launched as bench.py launches them (max-occupancy and original levels)
