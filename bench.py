@@ -40,7 +40,7 @@ WORKLOADS = {
                insts=49 * 12 + 10, bytes=32),
     # NLM box-sum + symmetric pairs, per pixel and offset pair: 1 difference (6), 1 horizontal
     # and 2 vertical blocked 7-sums (4 each), 2 x (1 FFMA exponent + 3 FFMA + 1 FADD + 1 compare)
-    "c2": dict(kernel="nlm_f4", W=2048, H=2048, sigma=0.13, unit="Mpix/s", name="imageDenoising NLM 2048x2048 RGBA",
+    "c2": dict(kernel="nlm_f4_w", W=2048, H=2048, sigma=0.13, unit="Mpix/s", name="imageDenoising NLM 2048x2048 RGBA",
                insts=24 * 30 + 10, bytes=32),
     # register-heavy direct NLM: 2401 patch terms x 6 + 49 x 6 per-offset terms + blend
     "c4": dict(kernel="nlm_f4_regheavy", W=4096, H=4096, sigma=0.13, unit="Mpix/s",
@@ -636,15 +636,16 @@ def run_c5(args):
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream
     wl = WORKLOADS["c5"]
+    kernel = args.kernel or wl["kernel"]
     W = H = args.size or wl["W"]
     b = shard.band(rank, world, H, 6)
     src = torch.empty((b.src_rows, W, 4), device=dev)
     O.generate_rgba(local, src.data_ptr(), W, H, b.src_begin, b.src_end, seed=1, sigma=wl["sigma"], stream=sp)
     out = torch.empty((b.rows_per_rank, W, 4), device=dev)
     full = torch.empty((world * b.rows_per_rank, W, 4), device=dev) if world > 1 else out
-    variants, res = O.build_all_levels(local, "nlm_f4")
+    variants, res = O.build_all_levels(local, kernel)
     nlev = len(variants)
-    a = O.denoise_args("nlm_f4", src.data_ptr(), out.data_ptr(), W, H, b.row_begin, b.row_end, b.src_begin,
+    a = O.denoise_args(kernel, src.data_ptr(), out.data_ptr(), W, H, b.row_begin, b.row_end, b.src_begin,
                        b.src_end, b.row_begin)
     ms = variants.sweep(a, sp, rounds=max(3, args.rounds // 3))
     tuner = O.Tuner(variants)
@@ -719,7 +720,7 @@ def run_c5(args):
                     r0, r1 = min(b.rows, c * per), min(b.rows, (c + 1) * per)
                     if r0 >= r1:
                         continue
-                    ca = O.denoise_args("nlm_f4", src.data_ptr(), out.data_ptr(), W, H, b.row_begin + r0,
+                    ca = O.denoise_args(kernel, src.data_ptr(), out.data_ptr(), W, H, b.row_begin + r0,
                                         b.row_begin + r1, b.src_begin, b.src_end, b.row_begin)
                     cev[s_][c][0].record(stream)
                     tuner.step(ca, sp)
@@ -755,7 +756,7 @@ def run_c5(args):
             "metric": METRIC, "value": H * W * args.steps / (tot * 1e-3) / 1e6, "unit": "Mpix/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": wl["name"], "kernel": "nlm_f4", "width": W, "height": H,
+            "config": {"workload": wl["name"], "kernel": kernel, "width": W, "height": H,
                        "rows_per_rank": b.rows_per_rank, "halo_rows": 6,
                        "collective": ("kernel fan-out stores into every rank's symmetric-memory image over NVLink "
                                       "+ device barrier" if mode == "fanout" else
@@ -767,7 +768,7 @@ def run_c5(args):
                              "ms_per_step": comp / args.steps},
             "allgather_ms_per_step": gat / args.steps,
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tinst/s (FP32 pipe lane-ops)",
-                         "frac": achieved / peak, "kernel": "nlm_f4", "peak_kind": peak_kind},
+                         "frac": achieved / peak, "kernel": kernel, "peak_kind": peak_kind},
             "per_rank": [{"rank": r, "final_k": c[0], "iterations_to_final": c[1], "sweep_best_k": c[2]}
                          for r, c in enumerate(allc)],
             "sweep_rank0": [{"k": variants.level(i).ctas_per_sm, "ms": round(ms[i], 4)} for i in range(nlev)],

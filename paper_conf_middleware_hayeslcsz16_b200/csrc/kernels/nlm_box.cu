@@ -40,15 +40,24 @@
 
 namespace {
 
-constexpr int TW = 122, TH = 23, NT = 128;
+// NLMB_WIDE (nlm_boxw.cu): TW = 128 output columns, every phase-B thread busy, phase-A warps of
+// 34 H columns (136 >= TW + 6), the tile two columns wider on the right; 115 188 B of shared
+// memory, still 2 CTAs/SM.  A 2048-wide frame is then 16 tile columns instead of 17.
+#ifdef NLMB_WIDE
+constexpr int TW = 128, HWARP = 34;
+#else
+constexpr int TW = 122, HWARP = 32;
+#endif
+constexpr int TH = 23, NT = 128;
+constexpr int ND = HWARP + 6;               // differences a phase-A lane slides over
 constexpr int AR = TH + 9;                  // phase-A rows (H rows): y0-6 .. y0+TH+3
-constexpr int HC = TW + 6;                  // H columns: x0-3 .. x0+TW+3
+constexpr int HC = 4 * HWARP;               // H columns: x0-3 .. (>= x0+TW+3)
 constexpr int HP = HC + 1;                  // odd H pitch
-constexpr int PC = TW + 18;                 // image tile columns: x0-9 .. x0+TW+9
+constexpr int PC = HC + 12;                 // image tile columns: x0-9 .. (>= x0+TW+9)
 constexpr int PR = TH + 12;                 // image tile rows:    y0-6 .. y0+TH+6
 constexpr int PW = PC + 1;                  // odd plane pitch
 constexpr int HBUF = AR * HP;               // floats per H buffer
-static_assert(AR == 32 && HC == 4 * 32 && NT == 128, "phase A: one lane per row, one warp per 32 H columns");
+static_assert(AR == 32 && HC >= TW + 6 && NT == 128, "phase A: one lane per row, 4 warps of HWARP H columns");
 static_assert(TW <= NT, "phase B: one thread per output column");
 
 // Packed fp32x2 arithmetic (sm_100 FADD2 / FMUL2 / FFMA2): two independent IEEE
@@ -91,7 +100,7 @@ template <int G>
 ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lane, int warp, int i,
                           int j1)
 {
-    const int cb = 3 + 32 * warp;               // tile column of u for the first difference
+    const int cb = 3 + HWARP * warp;            // tile column of u for the first difference
     const int rowc = lane * PW + cb;            // centre p(u, v)
     const int rows = rowc + i * PW + j1;        // shifted p(u+j1, v+i)
     // the shifted window holds columns q + j1 .. q + j1 + G - 1 at step q
@@ -104,10 +113,10 @@ ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lan
     }
     constexpr int GP = G / 2;                   // packed offset pairs (0 or 1)
     constexpr int GS = G - 2 * GP;              // scalar offsets left (0 or 1)
-    float2 dp[GP > 0 ? 38 : 1];
-    float ds[GS > 0 ? 38 : 1];
+    float2 dp[GP > 0 ? ND : 1];
+    float ds[GS > 0 ? ND : 1];
 #pragma unroll
-    for (int q = 0; q < 38; ++q) {
+    for (int q = 0; q < ND; ++q) {
 #pragma unroll
         for (int g = 0; g < G - 1; ++g) {
             wrg[g] = wrg[g + 1];
@@ -123,22 +132,22 @@ ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lan
         if (GS > 0) ds[GS > 0 ? q : 0] = diff2rg(wrg[G - 1], wb[G - 1], ncrg, cbv);
     }
     if (GP > 0) {
-        float2 h[32];
-        window7<32>(*reinterpret_cast<float2(*)[38]>(&dp), h);
-        float *h0 = hs + lane * HP + 32 * warp;
+        float2 h[HWARP];
+        window7<HWARP>(*reinterpret_cast<float2(*)[ND]>(&dp), h);
+        float *h0 = hs + lane * HP + HWARP * warp;
         float *h1 = h0 + HBUF;
 #pragma unroll
-        for (int q = 0; q < 32; ++q) {
+        for (int q = 0; q < HWARP; ++q) {
             h0[q] = h[q].x;
             h1[q] = h[q].y;
         }
     }
     if (GS > 0) {
-        float h[32];
-        window7<32>(*reinterpret_cast<float(*)[38]>(&ds), h);
-        float *h2 = hs + (G - 1) * HBUF + lane * HP + 32 * warp;
+        float h[HWARP];
+        window7<HWARP>(*reinterpret_cast<float(*)[ND]>(&ds), h);
+        float *h2 = hs + (G - 1) * HBUF + lane * HP + HWARP * warp;
 #pragma unroll
-        for (int q = 0; q < 32; ++q) h2[q] = h[q];
+        for (int q = 0; q < HWARP; ++q) h2[q] = h[q];
     }
 }
 
@@ -226,7 +235,7 @@ template <int G>
 ORION_DEVICE void phase_a_int(const float2 *prg, const float *pb, unsigned *hs, int lane, int warp,
                               int i, int j1)
 {
-    const int cb = 3 + 32 * warp;
+    const int cb = 3 + HWARP * warp;
     const int rowc = lane * PW + cb;
     const int rows = rowc + i * PW + j1;
     float2 wrg[G];
@@ -236,9 +245,9 @@ ORION_DEVICE void phase_a_int(const float2 *prg, const float *pb, unsigned *hs, 
         wrg[g + 1] = prg[rows + g];
         wb[g + 1] = pb[rows + g];
     }
-    unsigned q[G][38];
+    unsigned q[G][ND];
 #pragma unroll
-    for (int c = 0; c < 38; ++c) {
+    for (int c = 0; c < ND; ++c) {
 #pragma unroll
         for (int g = 0; g < G - 1; ++g) {
             wrg[g] = wrg[g + 1];
@@ -253,11 +262,11 @@ ORION_DEVICE void phase_a_int(const float2 *prg, const float *pb, unsigned *hs, 
     }
 #pragma unroll
     for (int g = 0; g < G; ++g) {
-        unsigned h[32];
-        window7_q<32>(q[g], h);
-        unsigned *hrow = hs + g * HBUF + lane * HP + 32 * warp;
+        unsigned h[HWARP];
+        window7_q<HWARP>(q[g], h);
+        unsigned *hrow = hs + g * HBUF + lane * HP + HWARP * warp;
 #pragma unroll
-        for (int c = 0; c < 32; ++c) hrow[c] = h[c];
+        for (int c = 0; c < HWARP; ++c) hrow[c] = h[c];
     }
 }
 
@@ -391,9 +400,14 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 
 }  // namespace
 
+#ifndef NLMB_WIDE
 // One pair per pass: 3 planar planes + 1 H buffer = 75 732 B of shared memory.
 extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<1, false>(a); }
 // Up to three pairs per pass: 3 planar planes + 3 H buffers = 108 756 B of shared memory.
 extern "C" __global__ void __launch_bounds__(128) orion_nlm_box3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<3, false>(a); }
 // Integer (fixed-point, exact) box sums, up to three pairs per pass.
 extern "C" __global__ void __launch_bounds__(128) orion_nlm_boxi3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<3, true>(a); }
+#else
+// 128-column tiles, up to three pairs per pass: 115 188 B of shared memory.
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_boxw3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<3, false>(a); }
+#endif

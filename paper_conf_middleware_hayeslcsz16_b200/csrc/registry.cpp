@@ -28,6 +28,7 @@ extern "C" const char liborion_ptx_gen[];
 extern "C" const char liborion_ptx_srad[];
 extern "C" const char liborion_ptx_nlm_box256[];
 extern "C" const char liborion_ptx_nlm_box4[];
+extern "C" const char liborion_ptx_nlm_boxw[];
 
 namespace orion {
 
@@ -42,6 +43,7 @@ static const char *module_ptx(const char *module)
     if (!std::strcmp(module, "srad")) return liborion_ptx_srad;
     if (!std::strcmp(module, "nlm_box256")) return liborion_ptx_nlm_box256;
     if (!std::strcmp(module, "nlm_box4")) return liborion_ptx_nlm_box4;
+    if (!std::strcmp(module, "nlm_boxw")) return liborion_ptx_nlm_boxw;
     return nullptr;
 }
 
@@ -63,6 +65,9 @@ static const KernelDef kKernels[] = {
     // (r, g, b, 1) float4 tile plane (pitch 141) + 2 H_o buffers, two pairs per pass (2 CTAs/SM)
     {"nlm_f4_q", 128, "orion_nlm_box4_f4_128", "nlm_box4", 128, 1, 122, 23, 6, K_NLM, 0,
      35 * 141 * 16 + 2 * 32 * 129 * 4, 1, 1, 1},
+    // 128-column tiles: planes (128+20) x 35 (pitch 149) + 3 H buffers of 32 x 137 floats
+    {"nlm_f4_w", 128, "orion_nlm_boxw3_f4_128", "nlm_boxw", 128, 1, 128, 23, 6, K_NLM, 0,
+     3 * 35 * 149 * 4 + 3 * 32 * 137 * 4, 1, 1, 1},
     // same, integer (fixed-point, exact) box sums
     {"nlm_f4_i", 128, "orion_nlm_boxi3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
      3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},

@@ -82,7 +82,7 @@ def test_query_limits_match_b200(dev):
 @pytest.mark.parametrize("kernel,threads", [("knn_f4", 128), ("knn_f4", 64), ("knn_f4", 256), ("knn_f4_p1", 128),
                                             ("knn_f4_t8", 128),
                                             ("nlm_f4", 128),
-                                            ("nlm_f4_q", 128), ("nlm_f4_g1", 128), ("nlm_f4_direct", 128), ("nlm_f4_regheavy", 128),
+                                            ("nlm_f4_q", 128), ("nlm_f4_w", 128), ("nlm_f4_g1", 128), ("nlm_f4_direct", 128), ("nlm_f4_regheavy", 128),
                                             ("hotspot_f32", 256),
                                             ("hotspot_f32", 128), ("hotspot2_f32", 256), ("hotspot2h_f32", 256),
                                             ("hotspot4h_f32", 256), ("srad_f32", 256)])
@@ -146,7 +146,7 @@ def test_knn_ragged_and_degenerate(dev, shape):
     check_vs_oracle(outs[0], out, alt, amb)
 
 
-@pytest.mark.parametrize("kernel", ["nlm_f4", "nlm_f4_q", "nlm_f4_g1", "nlm_f4_i", "nlm_f4_w8"])
+@pytest.mark.parametrize("kernel", ["nlm_f4", "nlm_f4_w", "nlm_f4_q", "nlm_f4_g1", "nlm_f4_i", "nlm_f4_w8"])
 @pytest.mark.parametrize("sigma", [0.05, 0.13, 0.2])
 def test_nlm_box_all_levels(dev, sigma, kernel):
     img = synth.noisy_rgba(250, 131, seed=2, sigma=sigma)
@@ -184,7 +184,7 @@ def _sample_points(W, H, n, seed):
     return np.array(xs), np.array(ys)
 
 
-@pytest.mark.parametrize("kernel,size", [("nlm_f4", 2048), ("nlm_f4_q", 2048), ("nlm_f4_i", 2048), ("knn_f4", 2048), ("knn_f4_t8", 2048),
+@pytest.mark.parametrize("kernel,size", [("nlm_f4", 2048), ("nlm_f4_w", 2048), ("nlm_f4_q", 2048), ("nlm_f4_i", 2048), ("knn_f4", 2048), ("knn_f4_t8", 2048),
                                          ("nlm_f4_regheavy", 4096)])
 def test_full_size_sampled(dev, kernel, size):
     # C2 / C4 sizes, launched as bench.py launches them (max-occupancy and original levels)
