@@ -1,12 +1,20 @@
+#!/bin/bash
+# A/B timing of two liborion builds on ONE box (gpurun): the same bench.py workload run
+# alternately with ORION_LIB=A and ORION_LIB=B, N pairs, ms_per_step of each run appended to
+# gpurun_out/ab.txt.  Build A first (e.g. git stash; build; cp liborion.so build/liborion_old.so;
+# git stash pop; build), then:
+#   gpurun -- 'bash tools/ab_run.sh c2 build/liborion_old.so paper_conf_middleware_hayeslcsz16_b200/liborion.so 2'
+# Extra bench.py flags may follow the pair count.
+WL=${1:-c2}
+A=${2:-build/liborion_old.so}
+B=${3:-paper_conf_middleware_hayeslcsz16_b200/liborion.so}
+N=${4:-2}
+shift 4 2>/dev/null
 OUT=gpurun_out
-rm -f $OUT/ab.txt
-python -m pytest tests/test_gpu_parity.py tests/test_gpu_fanout.py -q -x -k "nlm" > $OUT/t1.log 2>&1
-echo "tests rc=$?" >> $OUT/t1.log
-for i in 1 2; do
-for k in nlm_f4 nlm_f4_w; do
-python bench.py --kernel $k --steps 100 --warmup 10 --rounds 5 --no-cpu-baseline --no-carveout-axis > $OUT/x.log 2>&1
-echo "c2 $k $(grep -o '"ms_per_step": [0-9.]*' $OUT/x.log)" >> $OUT/ab.txt
-done; done
-python tools/wave_probe.py nlm_f4_w -1 2048 2048 2001 1840 1817 > $OUT/wave.log 2>&1
-python bench.py --workload c5 --kernel nlm_f4_w --steps 5 --warmup 3 > $OUT/c5w.log 2>&1
-echo "c5 nlm_f4_w $(grep -o '"ms_per_step": [0-9.]*' $OUT/c5w.log)" >> $OUT/ab.txt
+mkdir -p $OUT
+for i in $(seq 1 $N); do
+  for lib in $A $B; do
+    ORION_LIB=$lib python bench.py --workload $WL --rounds 3 --no-cpu-baseline --no-carveout-axis "$@" > $OUT/ab_last.log 2>&1
+    echo "$WL $lib $(grep -o '"ms_per_step": [0-9.]*' $OUT/ab_last.log)" >> $OUT/ab.txt
+  done
+done
