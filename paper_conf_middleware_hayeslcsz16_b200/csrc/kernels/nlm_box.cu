@@ -96,7 +96,9 @@ ORION_DEVICE float diff2rg(float2 arg, float ab, float2 ncrg, float cb)
 // Phase A for G offsets (i, j1 .. j1+G-1): lane = row r, warp's 32 H columns.  Differences
 // are channel-packed (diff2rg); the window sums of offsets g = 0, 1 run packed (fp32x2),
 // offset g = 2 scalar.
-template <int G>
+// VERT: the G offsets (i .. i+G-1, j1) -- one column offset on G rows -- with G shifted loads per
+// column instead of one (the j = 3 offsets of rows 1..3 in one pass instead of three).
+template <int G, bool VERT = false>
 ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lane, int warp, int i,
                           int j1)
 {
@@ -108,6 +110,7 @@ ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lan
     float wb[G];
 #pragma unroll
     for (int g = 0; g < G - 1; ++g) {
+        if (VERT) break;
         wrg[g + 1] = prg[rows + g];
         wb[g + 1] = pb[rows + g];
     }
@@ -117,13 +120,21 @@ ORION_DEVICE void phase_a(const float2 *prg, const float *pb, float *hs, int lan
     float ds[GS > 0 ? ND : 1];
 #pragma unroll
     for (int q = 0; q < ND; ++q) {
+        if (VERT) {
 #pragma unroll
-        for (int g = 0; g < G - 1; ++g) {
-            wrg[g] = wrg[g + 1];
-            wb[g] = wb[g + 1];
+            for (int g = 0; g < G; ++g) {
+                wrg[g] = prg[rows + g * PW + q];
+                wb[g] = pb[rows + g * PW + q];
+            }
+        } else {
+#pragma unroll
+            for (int g = 0; g < G - 1; ++g) {
+                wrg[g] = wrg[g + 1];
+                wb[g] = wb[g + 1];
+            }
+            wrg[G - 1] = prg[rows + q + G - 1];
+            wb[G - 1] = pb[rows + q + G - 1];
         }
-        wrg[G - 1] = prg[rows + q + G - 1];
-        wb[G - 1] = pb[rows + q + G - 1];
         const float2 ncrg = neg2(prg[rowc + q]);
         const float cbv = pb[rowc + q];
         if (GP > 0)
@@ -305,6 +316,10 @@ __constant__ int kPass1[24][3] = {
     {3, -3, 1}, {3, -2, 1}, {3, -1, 1}, {3, 0, 1}, {3, 1, 1}, {3, 2, 1}, {3, 3, 1}};
 __constant__ int kPass3[10][3] = {
     {0, 1, 3}, {1, -3, 3}, {1, 0, 2}, {1, 2, 2}, {2, -3, 3}, {2, 0, 2}, {2, 2, 2}, {3, -3, 3}, {3, 0, 2}, {3, 2, 2}};
+// Float path, three offsets per pass in 8 passes: (i, j1, vert) -- seven sliding passes
+// (i, j1 .. j1+2) and one vertical pass (1 .. 3, 3).
+__constant__ int kPass8[8][3] = {
+    {0, 1, 0}, {1, -3, 0}, {1, 0, 0}, {2, -3, 0}, {2, 0, 0}, {3, -3, 0}, {3, 0, 0}, {1, 3, 1}};
 
 template <int GMAX, bool INT>
 __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
@@ -350,12 +365,14 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
         for (int q = 0; q < (TH + 3) / 4; ++q) A.cnt[q] = c1 * 0x01010101u;
     }
 
-    constexpr int NPASS = GMAX == 1 ? 24 : 10;
+    constexpr bool P8 = GMAX == 3 && !INT;        // the 8-pass float schedule
+    constexpr int NPASS = GMAX == 1 ? 24 : (P8 ? 8 : 10);
 #pragma unroll 1
     for (int ps = 0; ps < NPASS; ++ps) {
-        const int i = GMAX == 1 ? kPass1[ps][0] : kPass3[ps][0];
-        const int j1 = GMAX == 1 ? kPass1[ps][1] : kPass3[ps][1];
-        const int G = GMAX == 1 ? 1 : kPass3[ps][2];
+        const int i = GMAX == 1 ? kPass1[ps][0] : (P8 ? kPass8[ps][0] : kPass3[ps][0]);
+        const int j1 = GMAX == 1 ? kPass1[ps][1] : (P8 ? kPass8[ps][1] : kPass3[ps][1]);
+        const int G = GMAX == 1 ? 1 : (P8 ? 3 : kPass3[ps][2]);
+        const int vert = P8 ? kPass8[ps][2] : 0;
         unsigned *hi = reinterpret_cast<unsigned *>(hs);
         if (INT) {
             if (GMAX == 1 || G == 1)
@@ -364,6 +381,11 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
                 phase_a_int<2>(prg, pb, hi, lane, warp, i, j1);
             else
                 phase_a_int<(GMAX >= 3 ? 3 : 1)>(prg, pb, hi, lane, warp, i, j1);
+        } else if (P8) {
+            if (vert)
+                phase_a<3, true>(prg, pb, hs, lane, warp, i, j1);
+            else
+                phase_a<3>(prg, pb, hs, lane, warp, i, j1);
         } else {
             if (GMAX == 1 || G == 1)
                 phase_a<1>(prg, pb, hs, lane, warp, i, j1);
@@ -376,10 +398,11 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
         if (t < TW) {
 #pragma unroll 1
             for (int g = 0; g < G; ++g) {
+                const int ig = vert ? i + g : i, jg = vert ? j1 : j1 + g;
                 if (INT)
-                    phase_b_int(prg, pb, hi + g * HBUF, t, i, j1 + g, nl2 * (1.0f / kQScale), wthr, A);
+                    phase_b_int(prg, pb, hi + g * HBUF, t, ig, jg, nl2 * (1.0f / kQScale), wthr, A);
                 else
-                    phase_b(prg, pb, hs + g * HBUF, t, i, j1 + g, nl2, wthr, A);
+                    phase_b(prg, pb, hs + g * HBUF, t, ig, jg, nl2, wthr, A);
             }
         }
         __syncthreads();
