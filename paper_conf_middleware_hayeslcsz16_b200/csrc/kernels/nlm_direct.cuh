@@ -23,13 +23,16 @@ __device__ __forceinline__ void nlm_direct_body(const orion_kargs &a)
     const float wthr = a.fparam[2];
     const float4 c00 = tile[ty * TW + tx];
 
+    // the centre patch, negated: each term's (r, g) difference is one FADD2 (fp32x2)
     float4 cp[REGHEAVY ? 2 * NLM_B + 1 : 1][REGHEAVY ? 2 * NLM_B + 1 : 1];
     if (REGHEAVY) {
 #pragma unroll
         for (int n = 0; n < 2 * NLM_B + 1; ++n)
 #pragma unroll
-            for (int m = 0; m < 2 * NLM_B + 1; ++m)
-                cp[REGHEAVY ? n : 0][REGHEAVY ? m : 0] = tile[(ty + n - NLM_B) * TW + tx + m - NLM_B];
+            for (int m = 0; m < 2 * NLM_B + 1; ++m) {
+                const float4 v = tile[(ty + n - NLM_B) * TW + tx + m - NLM_B];
+                cp[REGHEAVY ? n : 0][REGHEAVY ? m : 0] = make_float4(-v.x, -v.y, -v.z, 0.0f);
+            }
     }
 
     float ax = 0.f, ay = 0.f, az = 0.f, sw = 0.f;
@@ -44,9 +47,17 @@ __device__ __forceinline__ void nlm_direct_body(const orion_kargs &a)
 #pragma unroll
                 for (int m = -NLM_B; m <= NLM_B; ++m) {
                     const float4 s = tile[(ty + i + n) * TW + tx + j + m];
-                    const float4 c = REGHEAVY ? cp[REGHEAVY ? n + NLM_B : 0][REGHEAVY ? m + NLM_B : 0]
-                                              : tile[(ty + n) * TW + tx + m];
-                    d = __fadd_rn(d, dist2(s, c));
+                    float4 nc;
+                    if (REGHEAVY) {
+                        nc = cp[REGHEAVY ? n + NLM_B : 0][REGHEAVY ? m + NLM_B : 0];
+                    } else {
+                        const float4 c = tile[(ty + n) * TW + tx + m];
+                        nc = make_float4(-c.x, -c.y, -c.z, 0.0f);
+                    }
+                    // d += dr^2 + dg^2 + db^2, one FFMA per channel (a sum of non-negatives)
+                    const float2 e = __fadd2_rn(make_float2(s.x, s.y), make_float2(nc.x, nc.y));
+                    const float eb = __fadd_rn(s.z, nc.z);
+                    d = __fmaf_rn(eb, eb, __fmaf_rn(e.y, e.y, __fmaf_rn(e.x, e.x, d)));
                 }
             }
             const float w = ex2(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
