@@ -49,7 +49,7 @@ WORKLOADS = {
     "c3": dict(kernel="hotspot4h_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
                insts=12, bytes=12),
     # NEXT-4: a second Rodinia stencil (srad), 8 B/cell-iteration (read J, write J')
-    "srad": dict(kernel="srad_f32", W=8192, H=8192, unit="Mcell-steps/s", name="SRAD 8192x8192 fp32 (NEXT-4)",
+    "srad": dict(kernel="srad_f32h", W=8192, H=8192, unit="Mcell-steps/s", name="SRAD 8192x8192 fp32 (NEXT-4)",
                  insts=60, bytes=8),
     "c5": dict(kernel="nlm_f4", W=16384, H=16384, sigma=0.13, unit="Mpix/s",
                name="imageDenoising NLM 16384x16384 RGBA row-sharded with halos + NCCL all-gather",
@@ -273,7 +273,7 @@ def run_reference(args):
     for s in range(Wm + K):
         if wl["kernel"].startswith("hotspot"):
             u, dt, sample = cpu_baseline_hotspot(wl["W"], 1, per_step)
-        elif wl["kernel"] == "srad_f32":
+        elif wl["kernel"].startswith("srad_f32"):
             u, dt, sample = cpu_baseline_srad(wl["W"], 1, per_step)
         else:
             u, dt, sample = cpu_baseline_nlm("knn" if wl["kernel"].startswith("knn") else "nlm", wl["W"], wl["H"],
@@ -306,7 +306,7 @@ def run_ours(args):
     sp = stream.cuda_stream
     wl = WORKLOADS[args.workload]
     kernel, W, H = args.kernel or wl["kernel"], wl["W"], wl["H"]
-    is_srad = kernel == "srad_f32"
+    is_srad = kernel.startswith("srad_f32")
     is_stencil = kernel.startswith("hotspot") or is_srad
 
     # ---- multi-version binary: probe -> levels -> build (offline, untimed) ----------------

@@ -435,3 +435,123 @@ extern "C" __global__ void __launch_bounds__(256) orion_srad4_f32_256(orion_karg
         if (ys < a.row_end && x0 < a.width) srad_strip<1>(a, x0, ys, min(ys + 4 * SRAD_RY, a.row_end));
     }
 }
+
+// ---- halo-lane form (srad_f32h; width % 4 == 0) ------------------------------------------------
+// The float4 strip of srad_strip<4> with the warp's column halo carried by whole lanes, as in
+// hotspot2h / hotspot4h: a warp loads the 128 columns [base-4, base+124) and writes the 120
+// columns of lanes 1..30.  A cell's update needs J one column west and two east (c_E needs its
+// east neighbour) -- lane 0's last cell and lane 31's first cell and coefficient are exactly
+// that halo -- so there are no scalar outer-column loads, no lane-0 / lane-31 branches and no
+// divergent cp.async; the west / east image-edge clamps exist only in the warps that hold
+// column 0 or W-1 (CEDGE).  Every cell is srad_coeff2 / srad_update2's operation sequence with
+// the same clamp-to-edge neighbours: bit-identical to srad_f32 and srad_f32_tile.
+namespace {
+constexpr int SRADH_SLOT = 128;   // floats per ring slot: the warp's 128 columns of one J row
+}  // namespace
+
+template <bool CEDGE>
+__device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int ys, int ye)
+{
+    const int W = a.width, H = a.height;
+    const int lane = threadIdx.x;
+    const int cx = base - 4 + 4 * lane;
+    const int cxl = clampi(cx, 0, W - 4);
+    const bool wclamp = cx == 0, eclamp = cx + 4 >= W;
+    const bool writer = lane >= 1 && lane <= 30 && cx < W;
+    const SradConsts kc = srad_consts(a);
+    const float *J = (const float *)a.src - (size_t)a.src_row_begin * (size_t)W + cxl;   // row 0, own columns
+    float *Jo = (float *)a.dst + (size_t)cx - (size_t)a.dst_row_begin * (size_t)W;
+
+    auto load = [&](int y) { return __ldg(reinterpret_cast<const float4 *>(J + (size_t)y * (size_t)W)); };
+    auto coeff_row = [&](const float4 &N, const float4 &T, const float4 &S) {
+        float Wv = __shfl_up_sync(0xffffffffu, T.w, 1);
+        float Ev = __shfl_down_sync(0xffffffffu, T.x, 1);
+        if (CEDGE) {
+            if (wclamp) Wv = T.x;
+            if (eclamp) Ev = T.w;
+        }
+        CRow<4> c;
+        c.p[0] = srad_coeff2(make_float2(T.x, T.y), make_float2(N.x, N.y), make_float2(S.x, S.y),
+                             make_float2(__fsub_rn(Wv, T.x), __fsub_rn(T.x, T.y)),
+                             make_float2(__fsub_rn(T.y, T.x), __fsub_rn(T.z, T.y)), kc.iqden, kc.nq);
+        c.p[1] = srad_coeff2(make_float2(T.z, T.w), make_float2(N.z, N.w), make_float2(S.z, S.w),
+                             make_float2(__fsub_rn(T.y, T.z), __fsub_rn(T.z, T.w)),
+                             make_float2(__fsub_rn(T.w, T.z), __fsub_rn(Ev, T.w)), kc.iqden, kc.nq);
+        return c;
+    };
+    auto update_row = [&](int y, const float4 &T, const CRow<4> &c0, const CRow<4> &c1) {
+        float cE = __shfl_down_sync(0xffffffffu, c0.p[0].c.x, 1);
+        if (CEDGE && eclamp) cE = c0.p[1].c.y;
+        const float2 lo = srad_update2(make_float2(T.x, T.y), c0.p[0], c1.p[0].c,
+                                       make_float2(c0.p[0].c.y, c0.p[1].c.x), kc.lam4);
+        const float2 hi = srad_update2(make_float2(T.z, T.w), c0.p[1], c1.p[1].c, make_float2(c0.p[1].c.y, cE),
+                                       kc.lam4);
+        if (writer) *reinterpret_cast<float4 *>(Jo + (size_t)y * (size_t)W) = make_float4(lo.x, lo.y, hi.x, hi.y);
+    };
+
+    // rows y+2, y+3, ... stream through the warp's ring (slot q holds J(clamp(ys+2+q)))
+    extern __shared__ float4 srad_ring4[];
+    float *ring = reinterpret_cast<float *>(srad_ring4) + threadIdx.y * (SRAD_NB * SRADH_SLOT) + 4 * lane;
+    const float *pn = J + (size_t)min(ys + 2, H - 1) * (size_t)W;
+    int rn = ys + 2;
+    auto issue = [&](float *sl) {
+        srad_cp16(sl, pn);
+        if (rn < H - 1) pn += W;
+        ++rn;
+    };
+    const int yb = min(ye, H - 1);
+    const int nq = yb - ys;
+#pragma unroll
+    for (int q = 0; q < SRAD_NB - 1; ++q) {
+        if (q < nq) issue(ring + q * SRADH_SLOT);
+        srad_commit();
+    }
+    float4 j0 = load(ys), j1 = load(min(ys + 1, H - 1)), j2;
+    CRow<4> c0 = coeff_row(load(max(ys - 1, 0)), j0, j1), c1;
+    auto row = [&](int q, float *sl_read, float *sl_issue, const float4 &N, const float4 &T, float4 &S,
+                   const CRow<4> &cT, CRow<4> &cS) {
+        if (q + SRAD_NB - 1 < nq) issue(sl_issue);
+        srad_commit();
+        srad_wait<SRAD_NB - 1>();
+        S = *reinterpret_cast<const float4 *>(sl_read);
+        cS = coeff_row(N, T, S);
+        update_row(ys + q, N, cT, cS);
+    };
+    int q = 0;
+#define SH_S(k) (ring + (k) * SRADH_SLOT)
+#define SH_I(k) SH_S(((k) + SRAD_NB - 1) % SRAD_NB)
+#pragma unroll 1
+    for (; q + 6 <= nq; q += 6) {                               // slot of row q + k is k
+        row(q, SH_S(0), SH_I(0), j0, j1, j2, c0, c1);
+        row(q + 1, SH_S(1), SH_I(1), j1, j2, j0, c1, c0);
+        row(q + 2, SH_S(2), SH_I(2), j2, j0, j1, c0, c1);
+        row(q + 3, SH_S(3), SH_I(3), j0, j1, j2, c1, c0);
+        row(q + 4, SH_S(4), SH_I(4), j1, j2, j0, c0, c1);
+        row(q + 5, SH_S(5), SH_I(5), j2, j0, j1, c1, c0);
+    }
+#pragma unroll 1
+    for (; q < nq; ++q) {
+        row(q, SH_S(q % SRAD_NB), SH_I(q % SRAD_NB), j0, j1, j2, c0, c1);
+        j0 = j1;
+        j1 = j2;
+        c0 = c1;
+    }
+#undef SH_S
+#undef SH_I
+    srad_wait<0>();
+    if (ye == H) update_row(H - 1, j0, c0, c0);               // last image row: c_S = own c
+}
+
+// T = 256 threads (32 x 8 warps), output tile 120 x (8 * SRAD_RY); width % 4 == 0.
+extern "C" __global__ void __launch_bounds__(256) orion_srad4h_f32_256(orion_kargs a)
+{
+    ORION_PROBE(a);
+    const int ys = a.row_begin + blockIdx.y * (8 * SRAD_RY) + threadIdx.y * SRAD_RY;
+    if (ys >= a.row_end) return;
+    const int base = blockIdx.x * 120;
+    const bool cedge = base == 0 || base + 124 >= a.width;
+    if (cedge)
+        srad_strip_h<true>(a, base, ys, min(ys + SRAD_RY, a.row_end));
+    else
+        srad_strip_h<false>(a, base, ys, min(ys + SRAD_RY, a.row_end));
+}

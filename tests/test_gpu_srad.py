@@ -15,11 +15,22 @@ from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
 ROI = (0, 127, 0, 127)
 
 
-@pytest.fixture(scope="module")
-def srad():
+class Built(tuple):
+    """(variants, resources) plus the kernel id."""
+
+
+@pytest.fixture(scope="module", params=["srad_f32", "srad_f32h"])
+def srad(request):
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
-    return O.build_all_levels(0, "srad_f32", mode=O.REALISE_MIN_CARVEOUT)
+    b = Built(O.build_all_levels(0, request.param, mode=O.REALISE_MIN_CARVEOUT))
+    b.kernel = request.param
+    return b
+
+
+def aligned(srad, W):
+    """srad_f32h needs width % 4 == 0 (float4 lanes only)."""
+    return W + (-W % 4) if srad.kernel == "srad_f32h" else W
 
 
 def run(v, level, j0, iters, lam=0.5, roi=ROI):
@@ -67,7 +78,7 @@ def test_bit_exact_across_levels_and_vs_oracle(srad):
 
 def test_tile_and_sliding_kernels_identical(srad):
     vt, _ = O.build_all_levels(0, "srad_f32_tile", mode=O.REALISE_MIN_CARVEOUT)
-    t0, _ = synth.thermal_inputs(257, 190, seed=8)
+    t0, _ = synth.thermal_inputs(aligned(srad, 257), 190, seed=8)
     a, _ = run(srad[0], len(srad[0]) - 1, t0, 6)
     b, _ = run(vt, 0, t0, 6)
     assert np.array_equal(a, b)
@@ -82,7 +93,7 @@ def test_roi_statistics(srad):
 
 @pytest.mark.parametrize("shape", [(33, 17), (129, 130), (1, 64)])
 def test_ragged_shapes(srad, shape):
-    W, H = shape
+    W, H = aligned(srad, shape[0]), shape[1]
     t0, _ = synth.thermal_inputs(W, H, seed=3)
     roi = (0, H - 1, 0, W - 1)
     g, _ = run(srad[0], len(srad[0]) - 1, t0, 3, roi=roi)

@@ -32,9 +32,9 @@ pw = torch.empty_like(t0)
 t1 = torch.empty_like(t0)
 O.generate_thermal(0, t0.data_ptr(), pw.data_ptr(), WT, HT, stream=sp)
 q0 = torch.empty(1, device="cuda")
-for k in ("hotspot_f32", "hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32", "srad_f32", "srad_f32_tile"):
+for k in ("hotspot_f32", "hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32", "srad_f32", "srad_f32h", "srad_f32_tile"):
     v, _ = O.build_all_levels(0, k)
-    for w in ((WT, WT - 3) if k.startswith("srad") else (WT,)):
+    for w in ((WT, WT - 3) if k in ("srad_f32", "srad_f32_tile") else (WT,)):
         for i in (0, len(v) - 1):
             if k.startswith("srad"):
                 O.srad_roi_stats(0, t0.data_ptr(), w, HT, (0, 20, 0, 20), q0.data_ptr(), sp)
