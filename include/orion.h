@@ -120,14 +120,17 @@ orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int bloc
 
 /* ---- code generation (question 1; host-only, no GPU needed) ------------------------------ */
 
-/* Kernel ids: "knn_f4" (T = 128 / 256 / 64), "nlm_f4" (box sums, 3 offset pairs per pass),
+/* Kernel ids: "knn_f4" (T = 128 / 256 / 64), "knn_f4_p1" (one pixel per thread), "knn_f4_t8" (the 49
+ * taps of a pixel split over 8 lanes), "nlm_f4" (box sums, 3 offset pairs per pass), "nlm_f4_w" (same,
+ * 128-column tiles), "nlm_f4_q" (float4 tile plane, 2 pairs per pass),
  * "nlm_f4_i" (same, exact fixed-point integer windows), "nlm_f4_w8" (same tile, 256 threads),
  * "nlm_f4_g1" (1 pair per pass), "nlm_f4_direct", "nlm_f4_regheavy" (T = 128 / 64),
  * "hotspot_f32" (T = 256 / 128), "hotspot2_f32" (two stencil steps per launch, edge lanes fetch
  * the outer columns; width % 4 == 0), "hotspot2h_f32" (two steps per launch, whole halo lanes:
  * 120 output columns per warp; width % 4 == 0), "hotspot4h_f32" (four steps per launch, the same
  * halo-lane warps as a 4-stage register pipeline; width % 4 == 0; the C3 default),
- * "srad_f32" (register-sliding, any width), "srad_f32_tile" (shared-memory form, same bits).
+ * "srad_f32" (register-sliding, any width), "srad_f32h" (same with whole halo lanes; width % 4 == 0),
+ * "srad_f32_tile" (shared-memory form, same bits).
  * block_threads = 0 selects the kernel's default CTA size.  Fills the natural resources
  * (compiles the kernel's PTX once, uncapped, with the embedded ptxas). */
 orion_status orion_kernel_probe(const char *kernel_id, int block_threads, orion_kernel_resources *out);
@@ -277,7 +280,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
 /* A whole iterative stencil run end to end from HOST buffers -- the Rodinia driver shape
  * (copy the grid in, iterate, copy it out), the iterations being the ones
  * Fig. 9 tunes across (P:L651-P:L653).  Kernels of kind hotspot ("hotspot_f32",
- * "hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32") and srad ("srad_f32", "srad_f32_tile") only, whole grids only
+ * "hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32") and srad ("srad_f32", "srad_f32h", "srad_f32_tile") only, whole grids only
  * (a->row_begin = a->src_row_begin = a->dst_row_begin = 0, a->row_end = a->src_row_end =
  * a->height).
  *   a->src  host initial grid (fp32, width x height, row-major; pinned for async copies)
