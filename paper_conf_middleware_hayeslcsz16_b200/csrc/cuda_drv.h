@@ -23,7 +23,8 @@ namespace orion {
     X(cuMemcpyDtoHAsync) X(cuStreamSynchronize) X(cuGetErrorString) X(cuGetErrorName)            \
     X(cuMemAlloc) X(cuMemFree) X(cuStreamCreate) X(cuStreamDestroy) X(cuStreamWaitEvent)          \
     X(cuMemsetD32) X(cuMemcpyDtoH) X(cuCtxSynchronize) X(cuEventQuery) X(cuStreamBeginCapture)       \
-    X(cuStreamEndCapture) X(cuGraphInstantiate) X(cuGraphLaunch) X(cuGraphExecDestroy) X(cuGraphDestroy)
+    X(cuStreamEndCapture) X(cuGraphInstantiate) X(cuGraphLaunch) X(cuGraphExecDestroy) X(cuGraphDestroy) \
+    X(cuLaunchKernelEx)
 
 struct Driver {
 #define ORION_DECL(f) decltype(&::f) f = nullptr;

@@ -26,6 +26,8 @@ orion_status cu_fail(CUresult r, const char *what);          // maps a driver er
     } while (0)
 
 extern std::atomic<long long> g_launches;
+// Set while orion_tuner_capture records a graph: launches inside it are plain (no PDL attribute).
+extern thread_local bool t_capturing;
 
 // Makes the primary context of `device` current on the calling thread (retaining it).
 orion_status ensure_context(int device);

@@ -12,6 +12,7 @@
 //   verification   -> cuOccupancyMaxActiveBlocksPerMultiprocessor must report exactly k.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -74,6 +75,18 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
     return ORION_OK;
 }
 
+// Launches use programmatic stream serialization (PDL) unless ORION_PDL=0, and never while a
+// graph is being captured.  Measured A/B on one box (same library, ORION_PDL=0 vs 1): C2
+// 0.2217 -> 0.2197 ms, SRAD 0.1044 -> 0.1029 ms, C3 0.1571 -> 0.1564 ms per launch.
+static bool pdl_enabled()
+{
+    static const bool on = [] {
+        const char *e = std::getenv("ORION_PDL");
+        return !(e && e[0] == '0');
+    }();
+    return on && !t_capturing;
+}
+
 orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const orion_kargs &k, CUstream s)
 {
     const int rows = k.row_end - k.row_begin;
@@ -81,8 +94,31 @@ orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const
     const unsigned gx = (unsigned)((k.width + def.tile_w - 1) / def.tile_w);
     const unsigned gy = (unsigned)((rows + def.tile_h - 1) / def.tile_h);
     void *params[] = {const_cast<orion_kargs *>(&k)};
-    ORION_CU(drv().cuLaunchKernel(fn, gx, gy, 1, (unsigned)def.bx, (unsigned)def.by, 1, (unsigned)dyn_bytes, s,
-                                  params, nullptr));
+    if (pdl_enabled()) {
+        // programmatic dependent launch: this grid may be scheduled while the previous kernel
+        // of the stream drains; every kernel waits (griddepcontrol.wait, kernels/common.cuh)
+        // for its predecessor's completion before touching memory, so results are unchanged
+        CUlaunchAttribute attr;
+        std::memset(&attr, 0, sizeof attr);
+        attr.id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+        attr.value.programmaticStreamSerializationAllowed = 1;
+        CUlaunchConfig cfg;
+        std::memset(&cfg, 0, sizeof cfg);
+        cfg.gridDimX = gx;
+        cfg.gridDimY = gy;
+        cfg.gridDimZ = 1;
+        cfg.blockDimX = (unsigned)def.bx;
+        cfg.blockDimY = (unsigned)def.by;
+        cfg.blockDimZ = 1;
+        cfg.sharedMemBytes = (unsigned)dyn_bytes;
+        cfg.hStream = s;
+        cfg.attrs = &attr;
+        cfg.numAttrs = 1;
+        ORION_CU(drv().cuLaunchKernelEx(&cfg, fn, params, nullptr));
+    } else {
+        ORION_CU(drv().cuLaunchKernel(fn, gx, gy, 1, (unsigned)def.bx, (unsigned)def.by, 1, (unsigned)dyn_bytes, s,
+                                      params, nullptr));
+    }
     g_launches.fetch_add(1);
     return ORION_OK;
 }
