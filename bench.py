@@ -818,6 +818,11 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
+    if args.workload == "c1" and args.graph != "off":
+        # the settled C1 iterations replay as a CUDA graph, whose kernel nodes are plain
+        # launches; the sweep and the exploration must time the levels the same way, so this
+        # process launches without programmatic dependent launch (liborion reads ORION_PDL once)
+        os.environ.setdefault("ORION_PDL", "0")
     if args.impl == "reference":
         run_reference(args)
     elif args.workload == "c5":

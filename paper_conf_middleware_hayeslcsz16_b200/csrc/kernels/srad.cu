@@ -177,6 +177,8 @@ extern "C" __global__ void __launch_bounds__(1024) orion_srad_stats(const float 
                                                                      int c2, float *q0)
 {
     __shared__ double s1[32], s2[32];
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");   // PDL (see orion_probe)
+    asm volatile("griddepcontrol.wait;" ::: "memory");
     const int t = threadIdx.x;
     const int rw = c2 - c1 + 1, n = (r2 - r1 + 1) * rw;
     double a = 0.0, b = 0.0;

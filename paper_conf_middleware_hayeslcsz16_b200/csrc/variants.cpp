@@ -87,6 +87,38 @@ static bool pdl_enabled()
     return on && !t_capturing;
 }
 
+// Programmatic dependent launch when enabled: this grid may be scheduled while the previous
+// kernel of the stream drains; every kernel waits (griddepcontrol.wait, kernels/common.cuh and
+// orion_srad_stats) for its predecessor's completion before touching memory, so results are
+// unchanged.
+static orion_status launch_maybe_pdl(CUfunction fn, unsigned gx, unsigned gy, unsigned bx, unsigned by,
+                                     unsigned smem, CUstream s, void **params)
+{
+    if (!pdl_enabled()) {
+        ORION_CU(drv().cuLaunchKernel(fn, gx, gy, 1, bx, by, 1, smem, s, params, nullptr));
+        return ORION_OK;
+    }
+    CUlaunchAttribute attr;
+    std::memset(&attr, 0, sizeof attr);
+    attr.id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+    attr.value.programmaticStreamSerializationAllowed = 1;
+    CUlaunchConfig cfg;
+    std::memset(&cfg, 0, sizeof cfg);
+    cfg.gridDimX = gx;
+    cfg.gridDimY = gy;
+    cfg.gridDimZ = 1;
+    cfg.blockDimX = bx;
+    cfg.blockDimY = by;
+    cfg.blockDimZ = 1;
+    cfg.sharedMemBytes = smem;
+    cfg.hStream = s;
+    cfg.attrs = &attr;
+    cfg.numAttrs = 1;
+    ORION_CU(drv().cuLaunchKernelEx(&cfg, fn, params, nullptr));
+    return ORION_OK;
+}
+
+
 orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const orion_kargs &k, CUstream s)
 {
     const int rows = k.row_end - k.row_begin;
@@ -94,31 +126,7 @@ orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const
     const unsigned gx = (unsigned)((k.width + def.tile_w - 1) / def.tile_w);
     const unsigned gy = (unsigned)((rows + def.tile_h - 1) / def.tile_h);
     void *params[] = {const_cast<orion_kargs *>(&k)};
-    if (pdl_enabled()) {
-        // programmatic dependent launch: this grid may be scheduled while the previous kernel
-        // of the stream drains; every kernel waits (griddepcontrol.wait, kernels/common.cuh)
-        // for its predecessor's completion before touching memory, so results are unchanged
-        CUlaunchAttribute attr;
-        std::memset(&attr, 0, sizeof attr);
-        attr.id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
-        attr.value.programmaticStreamSerializationAllowed = 1;
-        CUlaunchConfig cfg;
-        std::memset(&cfg, 0, sizeof cfg);
-        cfg.gridDimX = gx;
-        cfg.gridDimY = gy;
-        cfg.gridDimZ = 1;
-        cfg.blockDimX = (unsigned)def.bx;
-        cfg.blockDimY = (unsigned)def.by;
-        cfg.blockDimZ = 1;
-        cfg.sharedMemBytes = (unsigned)dyn_bytes;
-        cfg.hStream = s;
-        cfg.attrs = &attr;
-        cfg.numAttrs = 1;
-        ORION_CU(drv().cuLaunchKernelEx(&cfg, fn, params, nullptr));
-    } else {
-        ORION_CU(drv().cuLaunchKernel(fn, gx, gy, 1, (unsigned)def.bx, (unsigned)def.by, 1, (unsigned)dyn_bytes, s,
-                                      params, nullptr));
-    }
+    ORION_TRY(launch_maybe_pdl(fn, gx, gy, (unsigned)def.bx, (unsigned)def.by, (unsigned)dyn_bytes, s, params));
     g_launches.fetch_add(1);
     return ORION_OK;
 }
@@ -469,7 +477,7 @@ extern "C" orion_status orion_srad_roi_stats(int device, const void *J, int widt
     CUfunction f;
     ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_srad_stats"));
     void *params[] = {&J, &width, &r1, &r2, &c1, &c2, &q0};
-    ORION_CU(drv().cuLaunchKernel(f, 1, 1, 1, 1024, 1, 1, 0, (CUstream)stream, params, nullptr));
+    ORION_TRY(launch_maybe_pdl(f, 1, 1, 1024, 1, 0, (CUstream)stream, params));
     g_launches.fetch_add(1);
     return ORION_OK;
 }
