@@ -397,18 +397,29 @@ def run_ours(args):
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     n_launch0 = O.launch_count()
+    # launch-bound frames (C1 by default): the K settled iterations replay as one CUDA graph.
+    # --graph native issues them in one library call instead (orion_tune_steps, under
+    # programmatic dependent launch): measured 3.6-3.7 us per C1 frame against 3.4-3.5 us for the
+    # graph (each frame is a DRAM-cold 64 KiB read either way).
     use_graph = (args.graph == "on" or (args.graph == "auto" and args.workload == "c1")) and not is_stencil \
         and tuner.final()[0] >= 0
+    native = not use_graph and args.graph == "native"
     graph = None
-    if use_graph:   # launch-bound frames: the K settled iterations replay as one CUDA graph
+    native_args = None
+    if use_graph:   # the K settled iterations replay as one CUDA graph
         graph = tuner.capture([step_args(step + k) for k in range(args.steps)])
         step += args.steps
         torch.cuda.synchronize()
+    elif native:
+        native_args = [step_args(step + k) for k in range(args.steps)]
+        step += args.steps
     torch.cuda.nvtx.range_push("timed")   # the launch list (ncu --nvtx-include "timed/") covers only this
     with ClockSampler(local) as clk:
         e0.record(stream)
         if graph is not None:
             graph.launch(sp)
+        elif native_args is not None:
+            tuner.steps(native_args, sp)
         else:
             for _ in range(args.steps):
                 tuner.step(step_args(step), sp)
@@ -579,7 +590,9 @@ def run_ours(args):
                    "l2": "inputs larger than L2: rotating pool of frames" if not is_stencil else
                          "grid 768 MiB > L2 (126 MB)",
                    "parallelism": f"dp{world} (independent frames per GPU)",
-                   "cuda_graph": graph is not None},
+                   "cuda_graph": graph is not None,
+                   "issue": "graph" if graph is not None else ("orion_tune_steps" if native_args is not None
+                                                               else "orion_tune_step per step")},
         "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
         "energy": clk.energy(args.steps),
         "select_mode": args.select,
@@ -801,9 +814,10 @@ def main():
     ap.add_argument("--c5-chunks", type=int, default=4, help="C5: row chunks per band whose all-gathers overlap compute")
     ap.add_argument("--c5-mode", default="auto", choices=("auto", "fanout", "gather"),
                     help="C5 exchange: kernel fan-out into symmetric memory (auto: when available) or all-gather")
-    ap.add_argument("--graph", default="auto", choices=("auto", "on", "off"),
-                    help="replay the K settled iterations as one CUDA graph (orion_tuner_capture); "
-                         "auto = on for the launch-bound C1 frames")
+    ap.add_argument("--graph", default="auto", choices=("auto", "on", "native", "off"),
+                    help="on: replay the K timed iterations as one CUDA graph (orion_tuner_capture); native: "
+                         "issue them in one library call (orion_tune_steps); off: one Python call per "
+                         "iteration; auto = on for the launch-bound C1 frames, off otherwise")
     ap.add_argument("--async-timing", type=int, default=0, choices=(0, 1),
                     help="1: the tuner reads its event pairs without host synchronisation "
                          "(orion_tuner_cfg.async_timing; exploration then spans as many iterations as the host "
@@ -818,10 +832,9 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
-    if args.workload == "c1" and args.graph != "off":
-        # the settled C1 iterations replay as a CUDA graph, whose kernel nodes are plain
-        # launches; the sweep and the exploration must time the levels the same way, so this
-        # process launches without programmatic dependent launch (liborion reads ORION_PDL once)
+    if args.graph == "on" or (args.graph == "auto" and args.workload == "c1"):
+        # graph kernel nodes are plain launches; the sweep must time the levels the same way, so
+        # this process launches without programmatic dependent launch (liborion reads it once)
         os.environ.setdefault("ORION_PDL", "0")
     if args.impl == "reference":
         run_reference(args)

@@ -259,6 +259,13 @@ orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, 
 /* The measured time of an exploring iteration is work-normalised (ns per output element,
  * P:L975) before Fig. 9 compares it, so iterations of different sizes compare fairly. */
 
+/* n consecutive iterations, exactly n calls of orion_tune_step on args[0..n-1] (host array of n
+ * orion_args, caller-owned), issued from the library in one call: launch-bound frames (C1) do not
+ * pay a foreign-function call per iteration.  *last (may be NULL) = the report of the last
+ * iteration.  Errors: ORION_E_INVALID for NULL / n < 0; otherwise the first failing
+ * orion_tune_step's status (the iterations before it have been issued). */
+orion_status orion_tune_steps(orion_tuner *t, const orion_args *args, int n, void *stream, orion_step_report *last);
+
 /* Kernel splitting ("we split one kernel invocation into multiple invocations, such
  * that every invocation of the split kernel launches a subset of the threads", [30]): the
  * output rows [row_begin, row_end) of ONE frame are processed as `bands` consecutive row

@@ -319,6 +319,17 @@ orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, 
     return report(lvl, measure ? 0 : 1);
 }
 
+orion_status orion_tune_steps(orion_tuner *t, const orion_args *args, int n, void *stream, orion_step_report *last)
+{
+    if (!t || !args || n < 0) return fail(ORION_E_INVALID, "orion_tune_steps: bad argument");
+    orion_step_report r{};
+    r.level_idx = -1;
+    r.ms = -1.0f;
+    for (int i = 0; i < n; ++i) ORION_TRY(orion_tune_step(t, &args[i], stream, &r));
+    if (last) *last = r;
+    return ORION_OK;
+}
+
 orion_status orion_tune_split(orion_tuner *t, const orion_args *a, int bands, void *stream, orion_step_report *reports)
 {
     if (!t || !a || bands < 1) return fail(ORION_E_INVALID, "orion_tune_split: bad argument");

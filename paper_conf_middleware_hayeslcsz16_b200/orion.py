@@ -140,6 +140,7 @@ def lib() -> ctypes.CDLL:
                 "orion_tuner_default_cfg": [P(TunerCfg)],
                 "orion_tuner_create": [V, P(TunerCfg), P(V)],
                 "orion_tune_step": [V, P(Args), V, P(StepReport)],
+                "orion_tune_steps": [V, P(Args), I, V, P(StepReport)],
                 "orion_tune_step_host": [V, P(Args), V, V, V, V, P(StepReport), P(ctypes.c_longlong),
                                          P(ctypes.c_longlong)],
                 "orion_tune_split": [V, P(Args), I, V, P(StepReport)],
@@ -375,6 +376,13 @@ class Tuner:
                                           "phase": "explore" if r.phase == 0 else "final",
                                           "ms": r.ms if r.ms >= 0 else None,
                                           "final_level_idx": r.final_level_idx}) + "\n")
+        return r
+
+    def steps(self, args_list: list, stream=None) -> StepReport:
+        """orion_tune_steps: len(args_list) iterations issued by the library in one call."""
+        arr = (Args * len(args_list))(*args_list)
+        r = StepReport()
+        _check(lib().orion_tune_steps(self.h, arr, len(args_list), _s(stream), ctypes.byref(r)), "orion_tune_steps")
         return r
 
     def split(self, args: Args, bands: int, stream=None) -> list[StepReport]:
