@@ -88,3 +88,33 @@ def test_trace_jsonl(knn, tmp_path):
     assert [r["iteration"] for r in recs] == list(range(12))
     assert recs[0]["phase"] == "explore" and recs[0]["ms"] is not None
     assert all(r["ctas_per_sm"] >= 1 for r in recs)
+
+
+def test_tune_steps_equals_step_loop(knn):
+    # orion_tune_steps: n iterations in one library call == n orion_tune_step calls (same Fig. 9
+    # walk, same final level, same output bits, n launches counted)
+    W = H = 64
+    n = 40
+    sp = torch.cuda.current_stream().cuda_stream
+    srcs = [torch.from_numpy(synth.noisy_rgba(W, H, seed=30 + f, sigma=0.2)).cuda() for f in range(4)]
+    outs = []
+    finals = []
+    for mode in ("loop", "steps"):
+        dsts = [torch.zeros_like(s) for s in srcs]
+        args = [O.denoise_args("knn_f4", srcs[f % 4].data_ptr(), dsts[f % 4].data_ptr(), W, H) for f in range(n)]
+        t = O.Tuner(knn)
+        t.resume(len(knn) - 1)                      # a fixed final level: both runs launch the same kernel
+        c0 = O.launch_count()
+        if mode == "loop":
+            for a in args:
+                t.step(a, sp)
+        else:
+            r = t.steps(args, sp)
+            assert r.final_level_idx == len(knn) - 1 and r.phase == 1
+        torch.cuda.synchronize()
+        assert O.launch_count() - c0 == n
+        finals.append(t.final()[0])
+        outs.append([d.cpu().numpy() for d in dsts])
+    assert finals[0] == finals[1]
+    for a, b in zip(*outs):
+        assert np.array_equal(a, b)
