@@ -485,7 +485,9 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2h_f32_256(orion_
 // the slot index 0.161; a persistent grid (one wave, each warp one ~240-row strip: 560 instead
 // of 604 MB of DRAM reads, no partial wave) 0.1665 vs 0.1550 -- fewer DRAM bytes alone do not
 // make this kernel faster; at 4 warps per scheduler it is bound by issue and latency as much as
-// by DRAM (long-scoreboard 1.9 stalls per issue on the ring waits, FMA pipe 56 % busy).
+// by DRAM (long-scoreboard 1.9 stalls per issue on the ring waits, FMA pipe 56 % busy).  64-row
+// strips also make a strip's 72 iterations exactly the 9 prologue/fill iterations + 7 bodies of 9
+// (no slow remainder loop): 61-row strips (3.96 instead of 3.73 waves) measured 0.159 vs 0.156.
 #ifndef HS_ROWS
 #define HS_ROWS 64
 #endif
