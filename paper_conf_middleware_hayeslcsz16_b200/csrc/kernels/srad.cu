@@ -544,16 +544,20 @@ __device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int
     if (ye == H) update_row(H - 1, j0, c0, c0);               // last image row: c_S = own c
 }
 
-// T = 256 threads (32 x 8 warps), output tile 120 x (8 * SRAD_RY); width % 4 == 0.
+// T = 256 threads (32 x 8 warps), output tile 120 x (8 * SRADH_RY); width % 4 == 0.  42-row
+// strips: a multiple of the 6-row loop body (no remainder iterations), 25 x 69 CTAs at 8192^2.
+#ifndef SRADH_RY
+#define SRADH_RY 42
+#endif
 extern "C" __global__ void __launch_bounds__(256) orion_srad4h_f32_256(orion_kargs a)
 {
     ORION_PROBE(a);
-    const int ys = a.row_begin + blockIdx.y * (8 * SRAD_RY) + threadIdx.y * SRAD_RY;
+    const int ys = a.row_begin + blockIdx.y * (8 * SRADH_RY) + threadIdx.y * SRADH_RY;
     if (ys >= a.row_end) return;
     const int base = blockIdx.x * 120;
     const bool cedge = base == 0 || base + 124 >= a.width;
     if (cedge)
-        srad_strip_h<true>(a, base, ys, min(ys + SRAD_RY, a.row_end));
+        srad_strip_h<true>(a, base, ys, min(ys + SRADH_RY, a.row_end));
     else
-        srad_strip_h<false>(a, base, ys, min(ys + SRAD_RY, a.row_end));
+        srad_strip_h<false>(a, base, ys, min(ys + SRADH_RY, a.row_end));
 }

@@ -96,8 +96,8 @@ static const KernelDef kKernels[] = {
     // srad, register-sliding: 124 x 128 tile; float4 lanes (width % 4 == 0) or scalar lanes;
     // rows stream through a 4-slot cp.async ring per warp (8 x 4 x 132 floats)
     {"srad_f32", 256, "orion_srad4_f32_256", "srad", 32, 8, 124, 256, 2, K_SRAD, 0, 8 * 6 * 132 * 4},
-    // srad, halo lanes: 120 x 256 tile, width % 4 == 0; 6-slot ring of 8 warps x 6 x 128 floats
-    {"srad_f32h", 256, "orion_srad4h_f32_256", "srad", 32, 8, 120, 256, 2, K_SRAD, 0, 8 * 6 * 128 * 4, 4},
+    // srad, halo lanes: 120 x 336 tile, width % 4 == 0; 6-slot ring of 8 warps x 6 x 128 floats
+    {"srad_f32h", 256, "orion_srad4h_f32_256", "srad", 32, 8, 120, 8 * 42, 2, K_SRAD, 0, 8 * 6 * 128 * 4, 4},
 };
 
 const KernelDef *find_kernel(const char *id, int threads)
