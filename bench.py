@@ -36,7 +36,7 @@ METRIC = "tuned Mpix/s vs max-occupancy build; tuner regret vs exhaustive level 
 WORKLOADS = {
     # KNN: 49 taps x (3 FSUB + FMUL + 2 FFMA distance, 1 FFMA exponent, 3 FFMA + 1 FADD
     # accumulate, 1 compare) + ~10 for the blend
-    "c1": dict(kernel="knn_f4_t8", W=64, H=64, sigma=0.2, unit="Mpix/s", name="imageDenoising KNN 64x64 RGBA r=3",
+    "c1": dict(kernel="knn_f4_t16", W=64, H=64, sigma=0.2, unit="Mpix/s", name="imageDenoising KNN 64x64 RGBA r=3",
                insts=49 * 12 + 10, bytes=32),
     # NLM box-sum + symmetric pairs, per pixel and offset pair: 1 difference (6), 1 horizontal
     # and 2 vertical blocked 7-sums (4 each), 2 x (1 FFMA exponent + 3 FFMA + 1 FADD + 1 compare)

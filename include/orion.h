@@ -120,8 +120,8 @@ orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int bloc
 
 /* ---- code generation (question 1; host-only, no GPU needed) ------------------------------ */
 
-/* Kernel ids: "knn_f4" (T = 128 / 256 / 64), "knn_f4_p1" (one pixel per thread), "knn_f4_t8" (the 49
- * taps of a pixel split over 8 lanes), "nlm_f4" (box sums, 3 offset pairs per pass), "nlm_f4_w" (same,
+/* Kernel ids: "knn_f4" (T = 128 / 256 / 64), "knn_f4_p1" (one pixel per thread), "knn_f4_t8" / "knn_f4_t16" (the
+ * 49 taps of a pixel split over 8 / 16 lanes), "nlm_f4" (box sums, 3 offset pairs per pass), "nlm_f4_w" (same,
  * 128-column tiles), "nlm_f4_q" (float4 tile plane, 2 pairs per pass),
  * "nlm_f4_i" (same, exact fixed-point integer windows), "nlm_f4_w8" (same tile, 256 threads),
  * "nlm_f4_g1" (1 pair per pass), "nlm_f4_direct", "nlm_f4_regheavy" (T = 128 / 64),

@@ -92,10 +92,12 @@ extern "C" __global__ void __launch_bounds__(64) orion_knn1_f4_64(orion_kargs a)
 // (same tap arithmetic), so the counts -- hence the lerp branch -- are the same; only the order
 // of the weighted sums differs (within the 1e-5 tolerance; bit-identical across occupancy
 // levels, which share this code).  CTA = 128 threads = 16 pixels of one row.
-__device__ __forceinline__ void knn_t8_body(const orion_kargs &a)
+template <int LP>
+__device__ __forceinline__ void knn_tap_split_body(const orion_kargs &a)
 {
-    const int g = threadIdx.x & 7;
-    const int x = blockIdx.x * 16 + (threadIdx.x >> 3);
+    static_assert(LP == 8 || LP == 16, "lanes per pixel");
+    const int g = threadIdx.x & (LP - 1);
+    const int x = blockIdx.x * (128 / LP) + (threadIdx.x / LP);
     const int y = a.row_begin + blockIdx.y;
     const int W = a.width, H = a.height;
     const int xc = min(x, W - 1);
@@ -106,9 +108,9 @@ __device__ __forceinline__ void knn_t8_body(const orion_kargs &a)
     float ax = 0.0f, ay = 0.0f, az = 0.0f, sw = 0.0f;
     int cnt = 0;
 #pragma unroll
-    for (int s = 0; s < 7; ++s) {
-        const int k = g + 8 * s;
-        if (k >= KNN_A) break;                     // only lane 0 of a group has a 7th tap (k = 48)
+    for (int s = 0; s < (KNN_A + LP - 1) / LP; ++s) {
+        const int k = g + LP * s;
+        if (k >= KNN_A) break;                     // only lane 0 of a group has the last tap (k = 48)
         const int i = k / 7 - KNN_R, j = k % 7 - KNN_R;
         const int gy = clampi(y + i, 0, H - 1), gx = clampi(xc + j, 0, W - 1);
         const float4 c = __ldg(src + (size_t)gy * (size_t)W + gx);
@@ -121,7 +123,7 @@ __device__ __forceinline__ void knn_t8_body(const orion_kargs &a)
         cnt += (w > wthr);
     }
 #pragma unroll
-    for (int o = 4; o > 0; o >>= 1) {
+    for (int o = LP / 2; o > 0; o >>= 1) {
         ax = __fadd_rn(ax, __shfl_xor_sync(0xffffffffu, ax, o));
         ay = __fadd_rn(ay, __shfl_xor_sync(0xffffffffu, ay, o));
         az = __fadd_rn(az, __shfl_xor_sync(0xffffffffu, az, o));
@@ -133,4 +135,6 @@ __device__ __forceinline__ void knn_t8_body(const orion_kargs &a)
         fanout_column(a, x, y, y + 1);
     }
 }
-extern "C" __global__ void __launch_bounds__(128) orion_knn8_f4_128(orion_kargs a) { ORION_PROBE(a); knn_t8_body(a); }
+extern "C" __global__ void __launch_bounds__(128) orion_knn8_f4_128(orion_kargs a) { ORION_PROBE(a); knn_tap_split_body<8>(a); }
+// 16 lanes per pixel (3-4 taps each), 8 pixels of one row per CTA.
+extern "C" __global__ void __launch_bounds__(128) orion_knn16_f4_128(orion_kargs a) { ORION_PROBE(a); knn_tap_split_body<16>(a); }

@@ -58,6 +58,8 @@ static const KernelDef kKernels[] = {
     {"knn_f4_p1", 64, "orion_knn1_f4_64", "knn", 8, 8, 8, 8, 3, K_KNN, 1, 0, 1, 1, 1},
     // 8 threads per pixel (taps split, shuffle-tree combine), 16 pixels of one row per CTA, no tile
     {"knn_f4_t8", 128, "orion_knn8_f4_128", "knn", 128, 1, 16, 1, 3, K_KNN, 0, 0, 1, 1, 1},
+    // 16 threads per pixel, 8 pixels of one row per CTA
+    {"knn_f4_t16", 128, "orion_knn16_f4_128", "knn", 128, 1, 8, 1, 3, K_KNN, 0, 0, 1, 1, 1},
     // nlm_box: 3 planar (122+18) x (23+12) fp32 planes (pitch 141) + 32 x 129 floats of H_o
     // up to 3 offset pairs per pass: 3 H_o buffers (2 CTAs/SM) -- the C2 / C5 default
     {"nlm_f4", 128, "orion_nlm_box3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,

@@ -15,13 +15,13 @@ sp = torch.cuda.current_stream().cuda_stream
 W, H = 70, 45                                     # ragged: not a multiple of any tile
 img = torch.empty((H, W, 4), device="cuda")
 O.generate_rgba(0, img.data_ptr(), W, H, sigma=0.13, stream=sp)
-for k in ("knn_f4", "knn_f4_t8", "nlm_f4", "nlm_f4_w", "nlm_f4_q", "nlm_f4_i", "nlm_f4_g1", "nlm_f4_w8", "nlm_f4_direct", "nlm_f4_regheavy"):
+for k in ("knn_f4", "knn_f4_t8", "knn_f4_t16", "nlm_f4", "nlm_f4_w", "nlm_f4_q", "nlm_f4_i", "nlm_f4_g1", "nlm_f4_w8", "nlm_f4_direct", "nlm_f4_regheavy"):
     v, _ = O.build_all_levels(0, k)
     out = torch.empty_like(img)
     full = torch.empty_like(img)
     for i in (0, len(v) - 1):
         a = O.denoise_args(k, img.data_ptr(), out.data_ptr(), W, H)
-        if k in ("knn_f4", "knn_f4_t8", "nlm_f4", "nlm_f4_w", "nlm_f4_q", "nlm_f4_i", "nlm_f4_g1", "nlm_f4_w8"):
+        if k in ("knn_f4", "knn_f4_t8", "knn_f4_t16", "nlm_f4", "nlm_f4_w", "nlm_f4_q", "nlm_f4_i", "nlm_f4_g1", "nlm_f4_w8"):
             a = O.with_fanout(a, [full.data_ptr()])
         v.launch(i, a, sp)
     torch.cuda.synchronize()
