@@ -124,6 +124,12 @@ class ClockSampler:
         if not self.ok or self.e0 is None or self.e1 is None:
             return None
         j = (self.e1 - self.e0) / 1e3
+        window = self.t1 - self.t0
+        if j <= 0 or window < 0.2:
+            # The board counter advances in coarse ticks: a short timed region reads 0 J,
+            # which is not a measurement.
+            return {"joules_per_step": None, "mean_watts": None, "source": "nvml total energy",
+                    "note": f"timed region {window * 1e3:.1f} ms is below the counter's update period"}
         return {"joules_per_step": j / steps, "mean_watts": j / (self.t1 - self.t0), "source": "nvml total energy"}
 
     def summary(self):
