@@ -125,7 +125,7 @@ class ClockSampler:
             return None
         j = (self.e1 - self.e0) / 1e3
         window = self.t1 - self.t0
-        if j <= 0 or window < 0.2:
+        if j <= 0 or window < 0.05:
             # The board counter advances in coarse ticks: a short timed region reads 0 J,
             # which is not a measurement.
             return {"joules_per_step": None, "mean_watts": None, "source": "nvml total energy",
