@@ -325,6 +325,13 @@ void orion_host_pipe_destroy(orion_host_pipe *p);
 /* Current ladder: *direction, ladder level indices (ladder[0] = original) -> out[]. */
 orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, int capacity, int *n_out);
 orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final);
+/* The runtime table Fig. 9 has seen so far (P:L605-P:L643; work-normalised per P:L975):
+ * out[i] = the value observed for level i -- ns per output element, the fastest of its
+ * samples_per_level samples -- or -1 for a level not (yet) measured.  `n` must equal the
+ * number of variants (ORION_E_INVALID otherwise).  Host-only read of tuner state; used to
+ * replay a live walk through an independent Fig. 9 (the oracle's O4) and check that the
+ * decisions are identical. */
+orion_status orion_tuner_tried(const orion_tuner *t, float *out, int n);
 /* Checkpoint / resume of the tuner's decision: a final level recorded from an
  * earlier run (orion_tuner_final, keyed by the caller on kernel id, device and shape) is set
  * directly, so a restarted application skips the Fig. 9 exploration.  ORION_E_INVALID for an

@@ -66,8 +66,12 @@ class _HsParams(ctypes.Structure):
 def _load():
     global _lib
     if _lib is None:
-        build()
-        lib = ctypes.CDLL(_LIB_PATH)
+        # ORACLE_LIB_OVERRIDE: a deliberately mutated build, used only by
+        # tests/test_oracle_mutations.py to show that the pins catch plausible mistakes
+        override = os.environ.get("ORACLE_LIB_OVERRIDE")
+        if not override:
+            build()
+        lib = ctypes.CDLL(override or _LIB_PATH)
         P = ctypes.c_void_p
         lib.oracle_denoise_rows.restype = ctypes.c_long
         lib.oracle_denoise_rows.argtypes = [P, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int,

@@ -578,6 +578,14 @@ orion_status orion_tuner_resume(orion_tuner *t, int final_level_idx)
     return ORION_OK;
 }
 
+orion_status orion_tuner_tried(const orion_tuner *t, float *out, int n)
+{
+    if (!t || !out || n != (int)t->v->vars.size()) return fail(ORION_E_INVALID, "orion_tuner_tried: bad argument");
+    for (int i = 0; i < n; ++i) out[i] = -1.0f;
+    for (auto &kv : t->f.tried) out[kv.first] = kv.second;
+    return ORION_OK;
+}
+
 orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final)
 {
     if (!t) return fail(ORION_E_INVALID, "orion_tuner_final: NULL");

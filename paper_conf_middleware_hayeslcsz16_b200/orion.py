@@ -154,6 +154,7 @@ def lib() -> ctypes.CDLL:
                 "orion_host_pipe_drain": [V],
                 "orion_tuner_ladder": [V, P(I), P(I), I, P(I)],
                 "orion_tuner_final": [V, P(I), P(I)],
+                "orion_tuner_tried": [V, P(ctypes.c_float), I],
                 "orion_tuner_replay": [P(TunerCfg), P(Level), I, I, P(ctypes.c_float), I, P(I), P(I), P(I)],
                 "orion_generate_rgba": [I, V, I, I, I, I, ctypes.c_uint, ctypes.c_float, V],
                 "orion_generate_thermal": [I, V, V, I, I, ctypes.c_uint, V],
@@ -421,6 +422,13 @@ class Tuner:
         buf = (ctypes.c_int * 64)()
         _check(lib().orion_tuner_ladder(self.h, ctypes.byref(d), buf, 64, ctypes.byref(n)), "orion_tuner_ladder")
         return d.value, [buf[i] for i in range(n.value)]
+
+    def tried(self) -> list[float]:
+        """orion_tuner_tried: the per-level table Fig. 9 observed (ns per output element; -1 = not run)."""
+        n = len(self.variants)
+        buf = (ctypes.c_float * n)()
+        _check(lib().orion_tuner_tried(self.h, buf, n), "orion_tuner_tried")
+        return [buf[i] for i in range(n)]
 
     def final(self):
         f, it = ctypes.c_int(), ctypes.c_int()

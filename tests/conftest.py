@@ -21,8 +21,11 @@ def occ_ref(tmp_path_factory):
     subprocess.check_call(["g++", "-O1", "-I/usr/local/cuda/include",
                            os.path.join(ROOT, "tests", "helpers", "occ_ref.cpp"), "-o", exe])
 
-    def run(cases):
+    def run(cases, mask=False):
+        """CTAs/SM per case; with mask=True, (CTAs/SM, limitingFactors) pairs."""
         inp = "".join(" ".join(str(x) for x in (tuple(c) + (100,))[:5]) + "\n" for c in cases)
-        out = subprocess.run([exe], input=inp, capture_output=True, text=True, check=True).stdout
-        return [int(x) for x in out.split()]
+        out = subprocess.run([exe] + (["--mask"] if mask else []), input=inp, capture_output=True,
+                             text=True, check=True).stdout
+        vals = [int(x) for x in out.split()]
+        return list(zip(vals[0::2], vals[1::2])) if mask else vals
     return run

@@ -4,10 +4,14 @@
 // prints the CTAs/SM that cudaOccMaxActiveBlocksPerMultiprocessor reports for a
 // B200 (cc 10.0) with the given carveout preference (percent; -1 = default) and the
 // dynamic-smem opt-in set.  Input lines: "T regs smem_static smem_dyn carveout_pct".
+// With the argument "--mask" each output line is "k limitingFactors" (the header's
+// OCC_LIMIT_* bits: WARPS 1, REGISTERS 2, SHARED_MEMORY 4, BLOCKS 8).
 #include <cuda_occupancy.h>
 #include <cstdio>
+#include <cstring>
 
-int main() {
+int main(int argc, char **argv) {
+    const bool mask = argc > 1 && std::strcmp(argv[1], "--mask") == 0;
     cudaOccDeviceProp prop;
     prop.computeMajor = 10;
     prop.computeMinor = 0;
@@ -35,7 +39,11 @@ int main() {
         state.cacheConfig = CACHE_PREFER_NONE;
         cudaOccResult res;
         cudaOccError e = cudaOccMaxActiveBlocksPerMultiprocessor(&res, &prop, &attr, &state, T, (size_t)sdyn);
-        std::printf("%d\n", e == CUDA_OCC_SUCCESS ? res.activeBlocksPerMultiprocessor : -1);
+        if (mask)
+            std::printf("%d %u\n", e == CUDA_OCC_SUCCESS ? res.activeBlocksPerMultiprocessor : -1,
+                        e == CUDA_OCC_SUCCESS ? res.limitingFactors : 0u);
+        else
+            std::printf("%d\n", e == CUDA_OCC_SUCCESS ? res.activeBlocksPerMultiprocessor : -1);
     }
     return 0;
 }

@@ -49,3 +49,26 @@ def test_split_more_bands_than_rows(sp):
     torch.cuda.synchronize()
     assert torch.equal(dst, ref)
     assert sum(r.iteration >= 0 for r in reps) == 5 and reps[-1].iteration == -1
+
+
+@pytest.mark.parametrize("kernel,bands", [("nlm_f4_regheavy", 16), ("nlm_f4_w", 7), ("knn_f4_t16", 5)])
+def test_split_frame_vs_oracle(sp, kernel, bands):
+    # NEXT-1 output against the oracle itself (not only the unsplit launch): every pixel of the
+    # banded frame, whatever level each band ran at
+    import numpy as np
+    import oracle
+    import synth
+    W, H = 333, 170
+    v, _ = O.build_all_levels(0, kernel)
+    img = synth.noisy_rgba(W, H, seed=6, sigma=0.2 if kernel.startswith("knn") else 0.13)
+    src = torch.from_numpy(img).cuda()
+    dst = torch.full_like(src, float("nan"))
+    t = O.Tuner(v)
+    reps = t.split(O.denoise_args(kernel, src.data_ptr(), dst.data_ptr(), W, H), bands, sp)
+    torch.cuda.synchronize()
+    assert len({r.level_idx for r in reps if r.iteration >= 0}) >= 2      # the bands ran different levels
+    g = dst.cpu().numpy()
+    out, alt, amb = oracle.denoise("knn" if kernel.startswith("knn") else "nlm", img)
+    gg = g[..., :3].astype(np.float64)
+    ok = (np.abs(gg - out) <= 1e-5).all(-1) | (amb & (np.abs(gg - alt) <= 1e-5).all(-1))
+    assert ok.all() and (g[..., 3] == 0).all()

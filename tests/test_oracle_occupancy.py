@@ -135,3 +135,46 @@ def test_min_carveout_levels_realise_k_per_nvidia_header(occ_ref, T, natural, ne
     # a kernel without shared memory keeps almost all of the array as L1 at every level
     if need == 0:
         assert max(l.carveout_kb for l in lmin) <= 100
+
+
+# cuda_occupancy.h's OCC_LIMIT_* bits -> the oracle's (orion.h's) LIM_* bits
+_HDR_TO_ORACLE = {0x01: O.LIM_WARPS, 0x02: O.LIM_REGS, 0x04: O.LIM_SMEM, 0x08: O.LIM_BLOCKS}
+
+
+def _from_header_mask(m):
+    return sum(v for b, v in _HDR_TO_ORACLE.items() if m & b)
+
+
+def test_limiter_mask_against_nvidia_limiting_factors(occ_ref):
+    # The limiter bitmask of a level is pinned to cudaOccResult.limitingFactors:
+    # every limit that equals the final CTA count, ties included (warps + registers, etc.).
+    cases = []
+    for T in (32, 64, 128, 256, 512, 1024):
+        for regs in (16, 32, 40, 48, 64, 72, 128, 168, 255):
+            for sst, sdyn in ((0, 0), (0, 6144), (0, 12800), (2048, 30000), (0, 76928), (0, 115840)):
+                for pct in (-1, 28, 100):
+                    cases.append((T, regs, sst, sdyn, pct))
+    want = occ_ref(cases, mask=True)
+    bad = []
+    for (T, r, s, d, p), (k, m) in zip(cases, want):
+        pct = None if p < 0 else p
+        if O.ctas_per_sm(O.B200, T, r, s, d, pct) != k or \
+                O.limiter_mask(O.B200, T, r, s, d, pct) != _from_header_mask(m):
+            bad.append(((T, r, s, d, p), O.limiter_mask(O.B200, T, r, s, d, pct), _from_header_mask(m)))
+    assert not bad, bad[:10]
+    # the grid exercises every limiter alone and the common ties
+    masks = {_from_header_mask(m) for _, m in want}
+    for bit in (O.LIM_REGS, O.LIM_SMEM, O.LIM_WARPS, O.LIM_BLOCKS):
+        assert bit in masks
+    assert any(m & (m - 1) for m in masks)
+
+
+def test_every_level_limiter_against_nvidia_header(occ_ref):
+    # the limiter field of each realised level equals the header's answer for that realisation
+    for T, natural, need in [(64, 39, 0), (128, 255, 0), (128, 39, 8704), (256, 96, 2048)]:
+        for mode in (O.REALISE_MAX_SMEM, O.REALISE_MIN_CARVEOUT):
+            lv = O.levels(O.B200, T, natural, 0, need, mode=mode)
+            cases = [(T, natural if l.reg_cap == 0 else l.reg_cap, 0, need + l.smem_pad_bytes,
+                      O.carveout_pct_for(O.B200, l.carveout_kb) if l.carveout_kb > 0 else -1) for l in lv]
+            got = occ_ref(cases, mask=True)
+            assert [(l.ctas_per_sm, l.limiter) for l in lv] == [(k, _from_header_mask(m)) for k, m in got]
