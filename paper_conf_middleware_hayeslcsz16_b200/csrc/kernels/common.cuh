@@ -45,6 +45,17 @@ ORION_DEVICE bool orion_probe(const orion_kargs &a)
 
 ORION_DEVICE int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
 
+// Row of the input slab a staged tile reads for global row gy: clamp-to-edge in GLOBAL
+// coordinates (the definition), then into the rows the slab holds.  The second clamp never
+// changes a row that a stored output depends on (the host guarantees the slab covers
+// [row_begin - halo, row_end + halo) after global clamping); it only keeps the tile rows past
+// row_end -- computed, never stored -- inside the slab's allocation (a band whose height is
+// not a multiple of the tile height would otherwise read up to TH - 1 rows past it).
+ORION_DEVICE int slab_row(const orion_kargs &a, int gy)
+{
+    return clampi(clampi(gy, 0, a.height - 1), a.src_row_begin, a.src_row_end - 1);
+}
+
 // Squared RGB distance, |a - b|^2 with a fixed operation order.
 ORION_DEVICE float dist2(float4 a, float4 b)
 {
@@ -59,13 +70,13 @@ template <int TW, int TH, int NT>
 ORION_DEVICE void load_tile_clamped(float4 *tile, const orion_kargs &a, int gx0, int gy0)
 {
     const float4 *src = (const float4 *)a.src;
-    const int W = a.width, H = a.height;
+    const int W = a.width;
     const int tid = threadIdx.y * blockDim.x + threadIdx.x;
     for (int idx = tid; idx < TW * TH; idx += NT) {
         int ty = idx / TW;
         int tx = idx - ty * TW;
         int gx = clampi(gx0 + tx, 0, W - 1);
-        int gy = clampi(gy0 + ty, 0, H - 1);
+        int gy = slab_row(a, gy0 + ty);
         tile[idx] = __ldg(src + (size_t)(gy - a.src_row_begin) * (size_t)W + gx);
     }
 }

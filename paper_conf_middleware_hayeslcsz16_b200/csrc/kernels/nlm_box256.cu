@@ -147,7 +147,7 @@ extern "C" __global__ void __launch_bounds__(256) orion_nlm_box256_f4_256(orion_
         for (int idx = tid; idx < PC * PR; idx += NT) {
             const int ty = idx / PC, tx = idx - ty * PC;
             const int gx = clampi(x0 - 9 + tx, 0, a.width - 1);
-            const int gy = clampi(y0 - 6 + ty, 0, a.height - 1);
+            const int gy = slab_row(a, y0 - 6 + ty);
             const float *g = (const float *)(src + (size_t)(gy - a.src_row_begin) * (size_t)a.width + gx);
             cpa4(pr + ty * PW + tx, g);        // cp.async: all copies in flight at once
             cpa4(pg + ty * PW + tx, g + 1);

@@ -162,7 +162,7 @@ __device__ __forceinline__ void nlm_box4_body(const orion_kargs &a)
         for (int idx = tid; idx < PC * PR; idx += NT) {
             const int ty = idx / PC, tx = idx - ty * PC;
             const int gx = clampi(x0 - 9 + tx, 0, a.width - 1);
-            const int gy = clampi(y0 - 6 + ty, 0, a.height - 1);
+            const int gy = slab_row(a, y0 - 6 + ty);
             cpa16(pl + ty * PW + tx, src + (size_t)(gy - a.src_row_begin) * (size_t)a.width + gx);
         }
         cp_async_wait_all();
