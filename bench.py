@@ -1,18 +1,25 @@
 #!/usr/bin/env python3
 """bench.py -- Orion occupancy-tuned hot path on B200 (BASELINE.json metric).
 
-One "step" = one application iteration of the whole hot path on one synthetic
-frame: orion_tune_step (Fig. 9 dynamic selection over the Fig. 8 ladder of the
-occupancy variants orion_build_variants produced from orion_levels) launching
-the NLM imageDenoising kernel on a 2048x2048 RGBA frame (config C2,
-BASELINE.json configs[1]).  Variants are built and every level is swept
-(orion_sweep, the exhaustive brute-force reference) before the timed region.
+One "step" = one application iteration of the whole hot path on one synthetic frame:
+orion_tune_step (Fig. 9 dynamic selection over the Fig. 8 ladder of the occupancy variants
+orion_build_variants produced from orion_levels) launching the configuration's kernel.
+Variants are built and every level is swept (orion_sweep, the exhaustive brute-force
+reference) before the timed region.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                  [--workload c1|c2|c3|c4|c5] [--no-cpu-baseline]
+                  [--workload c1|c2|c3|c4|c5|srad] [--only] [--no-cpu-baseline]
 
-Multi-GPU (torchrun, one process per GPU): weak scaling -- every rank tunes and
-runs its own C2 frames (no data-path collective); time = max over ranks.
+N = 1 (default): the headline is C2 (NLM 2048^2, BASELINE.json configs[1]); the same JSON
+line carries a sub-record per other configuration (C1, C3, C4, C5 at P = 1, SRAD) with its
+sweep, tuner walk, regret, vs max-occupancy, roofline and end-to-end figure, plus the NEXT-3
+resource-saving / energy record (Fig. 12 / 13 analogue).  --only: the headline workload alone.
+
+N > 1: the headline is C5 -- one 16384^2 NLM frame row-sharded over the N ranks (slab + 6-row
+halo generated in place, a tuner per rank, the output bands gathered into every rank's full
+image over NVLink) -- with C5 at P = 1 on rank 0 as the anchor of the curve.  Without
+torchrun, `--gpus N` re-launches itself under torch.distributed.run (one process per GPU).
+
 Prints ONE JSON line on rank 0.
 """
 from __future__ import annotations
@@ -21,7 +28,9 @@ import argparse
 import json
 import math
 import os
+import socket
 import statistics
+import subprocess
 import sys
 import threading
 import time
@@ -31,30 +40,32 @@ sys.path.insert(0, ROOT)
 
 METRIC = "tuned Mpix/s vs max-occupancy build; tuner regret vs exhaustive level sweep"
 
-# Workloads (BASELINE.json configs).  algorithmic FP32-pipe instructions per output unit
-# of the formulation each kernel implements, and HBM bytes per unit.
+# Workloads (BASELINE.json configs).  `insts`: algorithmic FP32-pipe instructions per output
+# unit of the formulation each kernel implements; `bytes`: HBM bytes per unit.
 WORKLOADS = {
     # KNN: 49 taps x (3 FSUB + FMUL + 2 FFMA distance, 1 FFMA exponent, 3 FFMA + 1 FADD
     # accumulate, 1 compare) + ~10 for the blend
     "c1": dict(kernel="knn_f4_t16", W=64, H=64, sigma=0.2, unit="Mpix/s", name="imageDenoising KNN 64x64 RGBA r=3",
-               insts=49 * 12 + 10, bytes=32),
+               insts=49 * 12 + 10, bytes=32, steps=3000, cfg_index=0),
     # NLM box-sum + symmetric pairs, per pixel and offset pair: 1 difference (6), 1 horizontal
     # and 2 vertical blocked 7-sums (4 each), 2 x (1 FFMA exponent + 3 FFMA + 1 FADD + 1 compare)
     "c2": dict(kernel="nlm_f4_w", W=2048, H=2048, sigma=0.13, unit="Mpix/s", name="imageDenoising NLM 2048x2048 RGBA",
-               insts=24 * 30 + 10, bytes=32),
-    # register-heavy direct NLM: 2401 patch terms x 6 + 49 x 6 per-offset terms + blend
-    "c4": dict(kernel="nlm_f4_regheavy", W=4096, H=4096, sigma=0.13, unit="Mpix/s",
-               name="register-heavy NLM 4096x4096 RGBA, maxrregcount caps", insts=2401 * 6 + 49 * 6 + 10, bytes=32),
+               insts=24 * 30 + 10, bytes=32, steps=300, cfg_index=1),
     # thermal stencil: four explicit steps per launch (hotspot4h_f32), 12 B per cell per launch
     "c3": dict(kernel="hotspot4h_f32", W=8192, H=8192, unit="Mcell-steps/s", name="thermal stencil 8192x8192 fp32",
-               insts=12, bytes=12),
+               insts=12, bytes=12, steps=25, cfg_index=2),
+    # register-heavy direct NLM: 2401 patch terms x 6 + 49 x 6 per-offset terms + blend
+    "c4": dict(kernel="nlm_f4_regheavy", W=4096, H=4096, sigma=0.13, unit="Mpix/s",
+               name="register-heavy NLM 4096x4096 RGBA, maxrregcount caps", insts=2401 * 6 + 49 * 6 + 10, bytes=32,
+               steps=30, cfg_index=3),
+    "c5": dict(kernel="nlm_f4_w", W=16384, H=16384, sigma=0.13, unit="Mpix/s",
+               name="imageDenoising NLM 16384x16384 RGBA row-sharded with halos + all-gather",
+               insts=24 * 30 + 10, bytes=32, steps=10, cfg_index=4),
     # NEXT-4: a second Rodinia stencil (srad), 8 B/cell-iteration (read J, write J')
     "srad": dict(kernel="srad_f32h", W=8192, H=8192, unit="Mcell-steps/s", name="SRAD 8192x8192 fp32 (NEXT-4)",
-                 insts=60, bytes=8),
-    "c5": dict(kernel="nlm_f4", W=16384, H=16384, sigma=0.13, unit="Mpix/s",
-               name="imageDenoising NLM 16384x16384 RGBA row-sharded with halos + NCCL all-gather",
-               insts=24 * 30 + 10, bytes=32),
+                 insts=60, bytes=8, steps=100, cfg_index=None),
 }
+SUB_RECORDS = ("c1", "c3", "c4", "srad", "c5")
 
 
 def load_peaks():
@@ -67,7 +78,9 @@ def load_peaks():
 
 
 class ClockSampler:
-    """nvidia-smi-equivalent sampling (NVML) of SM clock + throttle reasons during the timed region."""
+    """nvidia-smi-equivalent sampling (NVML) of SM clock + throttle reasons during the timed
+    region, and the board energy counter over it.  Call ``mark_end()`` right after the closing
+    synchronize: the window then ends with the GPU work, not after the sampler thread joins."""
 
     REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
                0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
@@ -77,6 +90,7 @@ class ClockSampler:
         self.samples, self.reasons, self.ok = [], set(), False
         self.period = period
         self.stop = threading.Event()
+        self.e1 = self.t1 = None
         try:
             import pynvml
             pynvml.nvmlInit()
@@ -88,17 +102,20 @@ class ClockSampler:
             self.err = str(e)
             self.max_mhz = None
 
+    def _sample(self):
+        try:
+            self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+            r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            for bit, name in self.REASONS.items():
+                if r & bit:
+                    self.reasons.add(name)
+        except Exception:
+            pass
+
     def _run(self):
-        while not self.stop.is_set():
-            try:
-                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
-                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
-                for bit, name in self.REASONS.items():
-                    if r & bit:
-                        self.reasons.add(name)
-            except Exception:
-                pass
-            time.sleep(self.period)
+        self._sample()
+        while not self.stop.wait(self.period):     # returns at once when stopped
+            self._sample()
 
     def _energy_mj(self):
         try:
@@ -113,11 +130,15 @@ class ClockSampler:
             self.t.start()
         return self
 
+    def mark_end(self):
+        if self.ok and self.t1 is None:
+            self.e1, self.t1 = self._energy_mj(), time.perf_counter()
+
     def __exit__(self, *a):
         if self.ok:
+            self.mark_end()
             self.stop.set()
             self.t.join()
-            self.e1, self.t1 = self._energy_mj(), time.perf_counter()
 
     def energy(self, steps: int):
         """Board energy over the timed region (NVML counter, mJ): J per step and mean W."""
@@ -130,7 +151,8 @@ class ClockSampler:
             # which is not a measurement.
             return {"joules_per_step": None, "mean_watts": None, "source": "nvml total energy",
                     "note": f"timed region {window * 1e3:.1f} ms is below the counter's update period"}
-        return {"joules_per_step": j / steps, "mean_watts": j / (self.t1 - self.t0), "source": "nvml total energy"}
+        return {"joules_per_step": j / steps, "mean_watts": j / window, "window_s": window,
+                "source": "nvml total energy"}
 
     def summary(self):
         if not self.ok:
@@ -139,13 +161,44 @@ class ClockSampler:
                 "reasons": sorted(self.reasons - {"gpu_idle"}), "samples": len(self.samples)}
 
 
+# ---- processes: one per GPU -------------------------------------------------------------------
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def free_port() -> int:
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def spawn_command(n: int, argv: list[str], port: int) -> list[str]:
+    """The torchrun re-launch of this script on n ranks (one process per GPU)."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+            "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *argv]
+
+
+def spawn(n: int, argv: list[str]) -> int:
+    """`--gpus N` without torchrun: re-launch under torch.distributed.run and pass its exit
+    code on (rank 0's JSON line is the only stdout line)."""
+    env = dict(os.environ, ORION_BENCH_SPAWNED="1")
+    return subprocess.run(spawn_command(n, argv, free_port()), env=env).returncode
+
+
+def backend_name() -> str:
+    """ORION_BENCH_BACKEND=gloo only exists to exercise the multi-rank control flow on one GPU
+    (ranks then share device local % device_count) or on CPU (--plumbing-check)."""
+    return os.environ.get("ORION_BENCH_BACKEND", "nccl")
+
+
 def init_dist(world: int, local: int) -> int:
-    """One process per GPU: bind the device and (N > 1) the NCCL process group.  The
-    ORION_BENCH_BACKEND=gloo override exists only to exercise the multi-rank control flow
-    on a single-GPU box (ranks then share device local % device_count)."""
+    """One process per GPU: bind the device and (N > 1) the process group."""
     import torch
     import torch.distributed as dist
-    backend = os.environ.get("ORION_BENCH_BACKEND", "nccl")
+    backend = backend_name()
     dev = local % max(1, torch.cuda.device_count()) if backend != "nccl" else local
     torch.cuda.set_device(dev)
     if world > 1:
@@ -156,28 +209,24 @@ def init_dist(world: int, local: int) -> int:
     return dev
 
 
-def dist_env():
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    return world, rank, local
-
-
-# ---------------------------------------------------------------------------------------------
+# ---- the CPU oracle timed on the host (a baseline, not the target) ------------------------------
 _SLAB_CACHE: dict = {}
 
 
-def cpu_baseline_nlm(kind: str, W: int, H: int, sigma: float, budget_s: float):
-    """The oracle (C, double, single thread) timed on a bounded row band of the same frame."""
-    import numpy as np
-    import oracle
+def _oracle_slab(W, H, sigma):
     import synth
-    rows_per = 2 if kind == "nlm" else 16
     y0 = H // 2
     key = (W, H, sigma)
     if key not in _SLAB_CACHE:   # the input slab is drawn once, outside any timing
         _SLAB_CACHE[key] = synth.noisy_rgba(W, H, seed=1, sigma=sigma, row_begin=y0 - 6, row_end=y0 + 6 + 1024)
-    img = _SLAB_CACHE[key]
+    return y0, _SLAB_CACHE[key]
+
+
+def cpu_baseline_nlm(kind: str, W: int, H: int, sigma: float, budget_s: float):
+    """The oracle (C, double, single thread) timed on a bounded row band of the same frame."""
+    import oracle
+    rows_per = 2 if kind == "nlm" else 16
+    y0, img = _oracle_slab(W, H, sigma)
     t0 = time.perf_counter()
     n = 0
     y = y0
@@ -188,21 +237,15 @@ def cpu_baseline_nlm(kind: str, W: int, H: int, sigma: float, budget_s: float):
         dt = time.perf_counter() - t0
         if dt >= budget_s or y >= min(H, y0 + 1024):
             break
-    return n * W, dt, f"{n} rows x {W} px of the C2 frame (rows {y0}..{y0 + n}), oracle/denoise.c, double"
+    return n * W, dt, f"{n} rows x {W} px of the {W}x{H} frame (rows {y0}..{y0 + n}), oracle/denoise.c, double"
 
 
 def cpu_baseline_nlm_threads(kind: str, W: int, H: int, sigma: float, budget_s: float, threads: int):
     """The same oracle call, unchanged, on `threads` host threads at once (ctypes releases the
     GIL inside the C function): each thread takes the next row chunk of the same slab."""
-    import threading
     import oracle
-    import synth
     rows_per = 2 if kind == "nlm" else 16
-    y0 = H // 2
-    key = (W, H, sigma)
-    if key not in _SLAB_CACHE:
-        _SLAB_CACHE[key] = synth.noisy_rgba(W, H, seed=1, sigma=sigma, row_begin=y0 - 6, row_end=y0 + 6 + 1024)
-    img = _SLAB_CACHE[key]
+    y0, img = _oracle_slab(W, H, sigma)
     span = min(H - y0, 1024)
     lock = threading.Lock()
     state = {"next": 0, "rows": 0}
@@ -225,7 +268,7 @@ def cpu_baseline_nlm_threads(kind: str, W: int, H: int, sigma: float, budget_s: 
     for t in ts:
         t.join()
     dt = time.perf_counter() - t0
-    return state["rows"] * W, dt, f"{state['rows']} rows x {W} px of the C2 frame on {threads} threads"
+    return state["rows"] * W, dt, f"{state['rows']} rows x {W} px of the {W}x{H} frame on {threads} threads"
 
 
 def host_threads() -> int:
@@ -267,15 +310,35 @@ def cpu_baseline_hotspot(W: int, steps: int, budget_s: float):
     return n * rows * W * steps, dt, f"{n} x ({rows} x {W} cells x {steps} steps), oracle/stencil.c f64"
 
 
+def cpu_baseline(kernel: str, wl: dict, seconds: float, all_cores: bool):
+    """The oracle as it stands on a bounded sample of the workload (rank 0, N = 1)."""
+    W, H = wl["W"], wl["H"]
+    if kernel.startswith("hotspot"):
+        u, dt, sample = cpu_baseline_hotspot(W, 1, seconds)
+    elif kernel.startswith("srad"):
+        u, dt, sample = cpu_baseline_srad(W, 1, seconds)
+    else:
+        u, dt, sample = cpu_baseline_nlm("knn" if kernel.startswith("knn") else "nlm", W, H, wl["sigma"], seconds)
+    cpu = {"value": u / dt / 1e6, "unit": wl["unit"], "cores": 1, "kind": "oracle", "sample": sample}
+    if all_cores and not (kernel.startswith("hotspot") or kernel.startswith("srad")) and host_threads() > 1:
+        nt = host_threads()   # SURVEY 8(d): also row-parallel on every host core
+        u2, dt2, sample2 = cpu_baseline_nlm_threads("knn" if kernel.startswith("knn") else "nlm", W, H, wl["sigma"],
+                                                    seconds, nt)
+        cpu["all_cores"] = {"value": u2 / dt2 / 1e6, "unit": wl["unit"], "cores": nt, "kind": "oracle",
+                            "sample": sample2}
+    return cpu
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle as it stands, timed on bounded samples (rank 0 only)."""
     world, rank, _ = dist_env()
     if rank != 0:
         return
-    wl = WORKLOADS[args.workload]
-    K, Wm = args.steps, args.warmup
+    wl = WORKLOADS[args.workload if world == 1 else "c5"]
+    K, Wm = args.steps or 5, args.warmup
     per_step = max(0.2, min(2.0, 150.0 / max(1, K + Wm)))
     times, units = [], []
+    sample = ""
     for s in range(Wm + K):
         if wl["kernel"].startswith("hotspot"):
             u, dt, sample = cpu_baseline_hotspot(wl["W"], 1, per_step)
@@ -297,23 +360,69 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
-# ---------------------------------------------------------------------------------------------
-def run_ours(args):
+# ---- one configuration on one GPU ---------------------------------------------------------------
+def _roofline(kernel, wl, units_per_launch, kernel_ms):
+    peaks, peak_kind = load_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    stencil = kernel.startswith("hotspot") or kernel.startswith("srad")
+    if stencil:
+        achieved = wl["bytes"] * units_per_launch / (kernel_ms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "peak_kind": peak_kind + " (copy bandwidth)"}
+    else:
+        peak = 148 * 128 * sm_max * 1e6 / 1e12
+        achieved = wl["insts"] * units_per_launch / (kernel_ms * 1e-3) / 1e12
+        roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tinst/s (FP32 pipe lane-ops)",
+                "frac": achieved / peak,
+                "peak_kind": f"derived: 148 SM x 128 FP32 lanes x {sm_max:.0f} MHz (sm_max_mhz, {peak_kind})",
+                "hbm_frac": wl["bytes"] * units_per_launch / (kernel_ms * 1e-3) / 1e9 / peaks["hbm_gbs"]}
+    roof["traffic"] = None
+    prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if os.path.exists(prof):
+        try:
+            with open(prof) as f:
+                ent = json.load(f).get(kernel) or {}
+            roof["traffic"] = ent.get("dram_bytes_per_launch")
+            m = ent.get("metrics", {})
+
+            def num(k):
+                return float(m[k].split()[0].replace(",", ""))
+            wf = num("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum")
+            dur = num("gpu__time_duration.sum") * {"ns": 1e-9, "us": 1e-6, "ms": 1e-3}.get(
+                m["gpu__time_duration.sum"].split()[-1][:2], 1e-6)
+            sm_hz = num("sm__cycles_elapsed.avg.per_second") * 1e9
+            roof["ncu"] = {"report": ent.get("report"), "smem_wavefront_frac": wf / (148 * dur * sm_hz),
+                           "issue_active_pct": num("smsp__issue_active.avg.pct_of_peak_sustained_active"),
+                           "lsu_pipe_pct": num("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active"),
+                           "fma_pipe_pct": num("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active")}
+        except Exception:
+            pass
+    roof["kernel"] = kernel
+    roof["algorithmic_per_unit"] = wl["insts"] if not stencil else wl["bytes"]
+    return roof
+
+
+def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_seconds: float,
+                   carveout_axis: bool, kernel: str | None = None, select: str = "fastest", world: int = 1,
+                   rank: int = 0, local: int = 0):
+    """Build, sweep, tune and time one configuration on this rank's GPU.  Returns the record
+    (rank 0) -- the same keys as the headline line."""
     import torch
     import torch.distributed as dist
     from paper_conf_middleware_hayeslcsz16_b200 import orion as O
 
-    world, rank, local = dist_env()
-    if not torch.cuda.is_available():
-        raise SystemExit("bench.py: no CUDA device (the product has no CPU path)")
-    local = init_dist(world, local)
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream
-    wl = WORKLOADS[args.workload]
-    kernel, W, H = args.kernel or wl["kernel"], wl["W"], wl["H"]
+    wl = WORKLOADS[key]
+    kernel, W, H = kernel or wl["kernel"], wl["W"], wl["H"]
     is_srad = kernel.startswith("srad_f32")
     is_stencil = kernel.startswith("hotspot") or is_srad
+    # launch-bound frames (C1 by default) replay their settled iterations as one CUDA graph,
+    # whose kernel nodes are plain launches: the whole configuration (sweep included) then runs
+    # without programmatic dependent launch, so every level is timed the way the loop runs it
+    graph_loop = (args.graph == "on" or (args.graph == "auto" and key == "c1")) and not is_stencil
+    pdl_prev = O.set_pdl(False) if graph_loop else None
 
     # ---- multi-version binary: probe -> levels -> build (offline, untimed) ----------------
     t_build = time.perf_counter()
@@ -368,23 +477,22 @@ def run_ours(args):
         if is_srad:
             O.srad_roi_stats(local, t_a.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
         sweep_args = grid_args(t_a, t_b)
-    ms = variants.sweep(sweep_args, sp, rounds=args.rounds)
+    ms = variants.sweep(sweep_args, sp, rounds=rounds)
     best = min(range(nlev), key=lambda i: ms[i])
-    # the carveout axis (Table 3 analogue): the same levels realised the other way
-    carveout_axis = None
-    if not args.no_carveout_axis:
+    worst = max(range(nlev), key=lambda i: ms[i])
+    caxis = None
+    if carveout_axis:   # the carveout axis (Table 3 analogue): the same levels realised the other way
         other = O.REALISE_MAX_SMEM if realise == O.REALISE_MIN_CARVEOUT else O.REALISE_MIN_CARVEOUT
         v2, _ = O.build_all_levels(local, kernel, mode=other)
-        ms2 = v2.sweep(sweep_args, sp, rounds=args.rounds)
-        carveout_axis = {"realise": "min_carveout" if other == O.REALISE_MIN_CARVEOUT else "max_smem",
-                         "levels": [{"k": v2.level(i).ctas_per_sm, "carveout_kb": v2.level(i).carveout_kb,
-                                     "pad": v2.level(i).smem_pad_bytes, "ms": round(ms2[i], 5)} for i in range(len(v2))],
-                         "ms_best": min(ms2)}
+        ms2 = v2.sweep(sweep_args, sp, rounds=rounds)
+        caxis = {"realise": "min_carveout" if other == O.REALISE_MIN_CARVEOUT else "max_smem",
+                 "levels": [{"k": v2.level(i).ctas_per_sm, "carveout_kb": v2.level(i).carveout_kb,
+                             "pad": v2.level(i).smem_pad_bytes, "ms": round(ms2[i], 5)} for i in range(len(v2))],
+                 "ms_best": min(ms2)}
         v2.close()
-    worst = max(range(nlev), key=lambda i: ms[i])
 
     # ---- the tuned loop: warmup (includes Fig. 9 exploration) then K timed steps ----------
-    cfg = O.default_cfg(select_mode=O.SELECT_LOWEST_WITHIN_TOL if args.select == "lowest" else O.SELECT_FASTEST,
+    cfg = O.default_cfg(select_mode=O.SELECT_LOWEST_WITHIN_TOL if select == "lowest" else O.SELECT_FASTEST,
                         samples_per_level=args.samples, async_timing=int(args.async_timing))
     tuner = O.Tuner(variants, cfg)
     direction, ladder = tuner.ladder()
@@ -392,8 +500,10 @@ def run_ours(args):
         state["a"], state["b"] = t_a, t_b
     step = 0
     explore_ms = []
-    for _ in range(args.warmup):
+    ran_levels = []
+    for _ in range(warmup):
         r = tuner.step(step_args(step), sp)
+        ran_levels.append(r.level_idx)
         if r.phase == 0 and r.ms >= 0:
             explore_ms.append(r.ms)
         step += 1
@@ -404,21 +514,17 @@ def run_ours(args):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     n_launch0 = O.launch_count()
     # launch-bound frames (C1 by default): the K settled iterations replay as one CUDA graph.
-    # --graph native issues them in one library call instead (orion_tune_steps, under
-    # programmatic dependent launch): measured 3.6-3.7 us per C1 frame against 3.4-3.5 us for the
-    # graph (each frame is a DRAM-cold 64 KiB read either way).
-    use_graph = (args.graph == "on" or (args.graph == "auto" and args.workload == "c1")) and not is_stencil \
-        and tuner.final()[0] >= 0
+    use_graph = graph_loop and tuner.final()[0] >= 0
     native = not use_graph and args.graph == "native"
     graph = None
     native_args = None
-    if use_graph:   # the K settled iterations replay as one CUDA graph
-        graph = tuner.capture([step_args(step + k) for k in range(args.steps)])
-        step += args.steps
+    if use_graph:
+        graph = tuner.capture([step_args(step + k) for k in range(steps)])
+        step += steps
         torch.cuda.synchronize()
     elif native:
-        native_args = [step_args(step + k) for k in range(args.steps)]
-        step += args.steps
+        native_args = [step_args(step + k) for k in range(steps)]
+        step += steps
     torch.cuda.nvtx.range_push("timed")   # the launch list (ncu --nvtx-include "timed/") covers only this
     with ClockSampler(local) as clk:
         e0.record(stream)
@@ -427,11 +533,12 @@ def run_ours(args):
         elif native_args is not None:
             tuner.steps(native_args, sp)
         else:
-            for _ in range(args.steps):
+            for _ in range(steps):
                 tuner.step(step_args(step), sp)
                 step += 1
         e1.record(stream)
         torch.cuda.synchronize()
+        clk.mark_end()
     torch.cuda.nvtx.range_pop()
     if graph is not None:
         graph.close()
@@ -447,20 +554,19 @@ def run_ours(args):
     final, iters_to_final = tuner.final()
     spl = O.STEPS_PER_LAUNCH.get(kernel, 1)                # stencil steps per launch (temporal blocking)
     units_per_step = W * H * spl
-    value = world * units_per_step * args.steps / (total_ms * 1e-3) / 1e6
-    ms_step = total_ms / args.steps
+    value = world * units_per_step * steps / (total_ms * 1e-3) / 1e6
+    ms_step = total_ms / steps
     t_final = ms[final] if final >= 0 else float("nan")
 
     # ---- end to end through the C ABI with pinned host buffers ---------------------------
-    # orion_host_pipe: every step copies its frame host->device, runs the tuned kernel and
-    # copies the result device->host; H2D(n+1) / kernel(n) / D2H(n-1) overlap on the pipe's
-    # three streams.  The synchronous orion_tune_step_host is reported beside it.
-    e2e = None
     if not is_stencil:
+        # orion_host_pipe: every step copies its frame host->device, runs the tuned kernel and
+        # copies the result device->host; H2D(n+1) / kernel(n) / D2H(n-1) overlap on the pipe's
+        # three streams.  The synchronous orion_tune_step_host is reported beside it.
         host_in = [srcs[f].cpu().pin_memory() for f in range(2)]
         host_out = [torch.empty((H, W, 4)).pin_memory() for _ in range(2)]
         has = [O.denoise_args(kernel, host_in[f].data_ptr(), host_out[f].data_ptr(), W, H) for f in range(2)]
-        n_e2e = max(4, min(args.steps, 60))
+        n_e2e = max(4, min(steps, 60 if frame_bytes > 1 << 20 else 2000))
         pipe = O.HostPipe(tuner, W, H, depth=3)
         for f in range(2):
             pipe.submit(has[f])                                                    # warm
@@ -487,6 +593,7 @@ def run_ours(args):
         e2e = {"value": world * W * H * n_e2e / dt / 1e6, "unit": wl["unit"], "h2d_bytes_per_step": hi,
                "d2h_bytes_per_step": ho, "steps": n_e2e, "api": "orion_host_pipe (depth 3, pinned host frames)",
                "sync_api_value": world * W * H * n_sync / dt_sync / 1e6}
+        del host_in, host_out
     else:
         # a whole run per job (orion_tune_run_host): host grids -> device, the config's 100
         # time steps under a FRESH tuner (its exploration included), final grid -> host
@@ -521,302 +628,497 @@ def run_ours(args):
                "api": f"orion_tune_run_host ({jobs} runs of {launches_per_job} launches from pinned host grids, "
                       f"a fresh tuner per run)"}
 
-    if rank != 0:
-        if world > 1:
-            dist.destroy_process_group()
-        return
+    rec = None
+    if rank == 0:
+        cpu = None
+        if world == 1 and cpu_seconds > 0:
+            cpu = cpu_baseline(kernel, wl, cpu_seconds, all_cores=True)
+        # Orion-Select (Fig. 11, P:L747-P:L755) = the tuned run INCLUDING its exploration: every
+        # iteration charged the sweep time of the level it ran (one timing method for all bars)
+        horizon = ran_levels + [final] * steps
+        select_ms = sum(ms[i] for i in horizon) / len(horizon)
+        lvl_rows = [{"k": lv[i].ctas_per_sm, "occ": lv[i].occupancy_permille / 1000, "reg_cap": lv[i].reg_cap,
+                     "regs": infos[i].regs, "pad": lv[i].smem_pad_bytes, "carveout_kb": lv[i].carveout_kb,
+                     "spill_st": infos[i].spill_store, "ms": round(ms[i], 5)} for i in range(nlev)]
+        rec = {
+            "metric": METRIC, "value": value, "unit": wl["unit"], "n_gpus": world, "steps": steps,
+            "warmup": warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": wl["name"], "baseline_config_index": wl["cfg_index"], "kernel": kernel,
+                       "block_threads": res.block_threads, "width": W, "height": H, "frames_in_pool": nframes,
+                       "l2": "inputs larger than L2: rotating pool of frames" if not is_stencil else
+                             "grids (3 x 256 MiB) > L2 (126 MB)",
+                       "parallelism": f"dp{world} (independent frames per GPU)",
+                       "cuda_graph": graph is not None,
+                       "issue": "graph" if graph is not None else ("orion_tune_steps" if native_args is not None
+                                                                   else "orion_tune_step per step")},
+            "roofline": _roofline(kernel, wl, W * H * spl, ms_step),
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
+            "energy": clk.energy(steps), "select_mode": select,
+            "resources": {"final_regs": infos[final].regs if final >= 0 else None,
+                          "natural_regs": res.regs_per_thread,
+                          "final_warps_per_sm": lv[final].warps_per_sm if final >= 0 else None,
+                          "best_warps_per_sm": lv[best].warps_per_sm,
+                          "register_file_used_frac": (infos[final].regs * lv[final].warps_per_sm * 32 / 65536)
+                          if final >= 0 else None},
+            "tuner": {"direction": "increasing" if direction == 1 else "decreasing",
+                      "ladder_k": [lv[i].ctas_per_sm for i in ladder],
+                      "final_k": lv[final].ctas_per_sm if final >= 0 else None,
+                      "final_occupancy": lv[final].occupancy_permille / 1000 if final >= 0 else None,
+                      "iterations_to_final": iters_to_final, "explore_ms": explore_ms,
+                      "explored_k": [lv[i].ctas_per_sm for i in ran_levels[:max(0, iters_to_final)]],
+                      "samples_per_level": args.samples, "async_timing": bool(args.async_timing)},
+            "sweep": {"rounds": rounds, "n_levels": nlev, "levels": lvl_rows, "best_k": lv[best].ctas_per_sm,
+                      "ms_best": ms[best], "worst_k": lv[worst].ctas_per_sm, "ms_worst": ms[worst],
+                      "maxocc_k": lv[kmax].ctas_per_sm, "ms_maxocc": ms[kmax],
+                      "nvcc_default_k": lv[orig].ctas_per_sm, "ms_nvcc_default": ms[orig]},
+            "regret": t_final / ms[best] - 1.0,
+            "fig11": {"orion_min_ms": ms[worst], "orion_max_ms": ms[best], "nvcc_ms": ms[orig],
+                      "orion_select_ms": select_ms, "speedup_select_vs_nvcc": ms[orig] / select_ms,
+                      "speedup_max_vs_nvcc": ms[orig] / ms[best], "speedup_min_vs_nvcc": ms[orig] / ms[worst],
+                      "note": "every bar timed by orion_sweep (interleaved rounds); Orion-Select charges each "
+                              "warm-up + timed iteration the sweep time of the level it ran"},
+            "vs_maxocc": ms[kmax] / t_final,
+            "vs_nvcc_default": ms[orig] / t_final,
+            "build_seconds": round(t_build, 2),
+            "realise": "min_carveout" if realise == O.REALISE_MIN_CARVEOUT else "max_smem",
+            "carveout_axis": caxis,
+        }
+    tuner.close()
+    variants.close()
+    if graph_loop:
+        O.set_pdl(pdl_prev)
+    torch.cuda.empty_cache()
+    return rec
 
-    # ---- roofline of the dominant kernel ----------------------------------------------------
-    peaks, peak_kind = load_peaks()
-    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
-    kernel_ms = ms_step  # one launch per steady-state step; the stream holds only our kernel
+
+# ---- NEXT-3: resource-saving selection and energy (Fig. 12 / 13 analogues) ---------------------
+def measure_energy(key: str, args, kernel: str, local: int = 0, window_s: float = 1.2):
+    """Fig. 12 (registers saved, P:L873-P:L939) and Fig. 13 (energy, P:L943-P:L979) analogues for
+    one configuration: the level LOWEST_WITHIN_TOL selects (the paper's resource-saving reading,
+    R-A4), the level FASTEST selects, the exhaustive-best and the max-occupancy level; each is
+    replayed as a CUDA graph of its settled iterations over NVML windows >= `window_s` s."""
+    import torch
+    from paper_conf_middleware_hayeslcsz16_b200 import orion as O
+
+    sp = torch.cuda.current_stream().cuda_stream
+    wl = WORKLOADS[key]
+    W, H = wl["W"], wl["H"]
+    is_srad = kernel.startswith("srad")
+    is_stencil = kernel.startswith("hotspot") or is_srad
+    realise = O.REALISE_MIN_CARVEOUT if args.realise == "min" else O.REALISE_MAX_SMEM
+    pdl_prev = O.set_pdl(False)          # every level below is replayed as a CUDA graph (plain launches)
+    v, res = O.build_all_levels(local, kernel, mode=realise)
+    n = len(v)
     if is_stencil:
-        achieved = wl["bytes"] * W * H / (kernel_ms * 1e-3) / 1e9   # bytes per launch (T, P in; T' out)
-        roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "frac": achieved / peaks["hbm_gbs"], "peak_kind": peak_kind + " (copy bandwidth)"}
-    else:
-        peak = 148 * 128 * sm_max * 1e6 / 1e12
-        achieved = wl["insts"] * units_per_step / (kernel_ms * 1e-3) / 1e12
-        roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tinst/s (FP32 pipe lane-ops)",
-                "frac": achieved / peak,
-                "peak_kind": f"derived: 148 SM x 128 FP32 lanes x {sm_max:.0f} MHz (sm_max_mhz, {peak_kind})",
-                "hbm_frac": wl["bytes"] * units_per_step / (kernel_ms * 1e-3) / 1e9 / peaks["hbm_gbs"]}
-    roof["traffic"] = None
-    prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
-    if os.path.exists(prof):
-        try:
-            with open(prof) as f:
-                pj = json.load(f)
-            ent = pj.get(kernel) or {}
-            roof["traffic"] = ent.get("dram_bytes_per_launch")
-            m = ent.get("metrics", {})
-
-            def num(k):
-                return float(m[k].split()[0].replace(",", ""))
-            # the resource that actually binds the denoisers: shared-memory wavefronts per SM
-            # cycle (1 / clk / SM peak) and the issue slots, from the committed ncu capture
-            wf = num("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum")
-            dur = num("gpu__time_duration.sum") * {"ns": 1e-9, "us": 1e-6, "ms": 1e-3}.get(
-                m["gpu__time_duration.sum"].split()[-1][:2], 1e-6)
-            sm_hz = num("sm__cycles_elapsed.avg.per_second") * 1e9
-            roof["ncu"] = {"report": ent.get("report"), "smem_wavefront_frac": wf / (148 * dur * sm_hz),
-                           "issue_active_pct": num("smsp__issue_active.avg.pct_of_peak_sustained_active"),
-                           "lsu_pipe_pct": num("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active"),
-                           "fma_pipe_pct": num("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active")}
-        except Exception:
-            pass
-    roof["kernel"] = kernel
-    roof["algorithmic_per_unit"] = wl["insts"] if not is_stencil else wl["bytes"]
-
-    # ---- CPU baseline (the oracle), rank 0, N=1 only ------------------------------------------
-    cpu = None
-    if world == 1 and not args.no_cpu_baseline:
-        if is_stencil:
-            u, dt, sample = (cpu_baseline_srad if is_srad else cpu_baseline_hotspot)(W, 1, args.cpu_seconds)
+        a_ = torch.empty((H, W), device="cuda")
+        b_ = torch.empty((H, W), device="cuda")
+        p_ = torch.empty((H, W), device="cuda")
+        O.generate_thermal(local, a_.data_ptr(), p_.data_ptr(), W, H, seed=1, stream=sp)
+        q0 = torch.empty(1, device="cuda")
+        if is_srad:
+            O.srad_roi_stats(local, a_.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
+            args_pp = [O.srad_args(a_.data_ptr(), b_.data_ptr(), q0.data_ptr(), W, H),
+                       O.srad_args(b_.data_ptr(), a_.data_ptr(), q0.data_ptr(), W, H)]
         else:
-            u, dt, sample = cpu_baseline_nlm("knn" if kernel.startswith("knn") else "nlm", W, H, wl["sigma"],
-                                             args.cpu_seconds)
-        cpu = {"value": u / dt / 1e6, "unit": wl["unit"], "cores": 1, "kind": "oracle", "sample": sample}
-        if not is_stencil and host_threads() > 1:   # also row-parallel on every host core
-            nt = host_threads()
-            u2, dt2, sample2 = cpu_baseline_nlm_threads("knn" if kernel.startswith("knn") else "nlm", W, H,
-                                                        wl["sigma"], args.cpu_seconds, nt)
-            cpu["all_cores"] = {"value": u2 / dt2 / 1e6, "unit": wl["unit"], "cores": nt, "kind": "oracle",
-                                "sample": sample2}
+            args_pp = [O.hotspot_args(a_.data_ptr(), b_.data_ptr(), p_.data_ptr(), W, H),
+                       O.hotspot_args(b_.data_ptr(), a_.data_ptr(), p_.data_ptr(), W, H)]
+    else:
+        nfr = max(2, math.ceil(2 * 126e6 / (2 * W * H * 16)) + 1)
+        srcs = [torch.empty((H, W, 4), device="cuda") for _ in range(nfr)]
+        dsts = [torch.empty((H, W, 4), device="cuda") for _ in range(nfr)]
+        for f, t in enumerate(srcs):
+            O.generate_rgba(local, t.data_ptr(), W, H, seed=1 + f, sigma=wl["sigma"], stream=sp)
+        args_pp = [O.denoise_args(kernel, srcs[f].data_ptr(), dsts[f].data_ptr(), W, H) for f in range(nfr)]
+    torch.cuda.synchronize()
+    ms = v.sweep(args_pp[0], sp, rounds=args.rounds)
 
-    lvl_rows = [{"k": lv[i].ctas_per_sm, "occ": lv[i].occupancy_permille / 1000, "reg_cap": lv[i].reg_cap,
-                 "regs": infos[i].regs, "pad": lv[i].smem_pad_bytes, "carveout_kb": lv[i].carveout_kb,
-                 "spill_st": infos[i].spill_store, "ms": round(ms[i], 5)} for i in range(nlev)]
-    line = {
-        "metric": METRIC, "value": value, "unit": wl["unit"], "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
-        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": wl["name"], "kernel": kernel, "block_threads": res.block_threads,
-                   "width": W, "height": H, "frames_in_pool": nframes,
-                   "l2": "inputs larger than L2: rotating pool of frames" if not is_stencil else
-                         "grid 768 MiB > L2 (126 MB)",
-                   "parallelism": f"dp{world} (independent frames per GPU)",
-                   "cuda_graph": graph is not None,
-                   "issue": "graph" if graph is not None else ("orion_tune_steps" if native_args is not None
-                                                               else "orion_tune_step per step")},
-        "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
-        "energy": clk.energy(args.steps),
-        "select_mode": args.select,
-        "resources": {"final_regs": infos[final].regs if final >= 0 else None,
-                      "natural_regs": res.regs_per_thread,
-                      "final_warps_per_sm": lv[final].warps_per_sm if final >= 0 else None,
-                      "best_warps_per_sm": lv[best].warps_per_sm,
-                      "register_file_used_frac": (infos[final].regs * lv[final].warps_per_sm * 32 / 65536)
-                      if final >= 0 else None},
-        "tuner": {"direction": "increasing" if direction == 1 else "decreasing", "ladder_k": [lv[i].ctas_per_sm
-                  for i in ladder], "final_k": lv[final].ctas_per_sm if final >= 0 else None,
-                  "final_occupancy": lv[final].occupancy_permille / 1000 if final >= 0 else None,
-                  "iterations_to_final": iters_to_final, "explore_ms": explore_ms,
-                  "samples_per_level": args.samples, "async_timing": bool(args.async_timing)},
-        "sweep": {"rounds": args.rounds, "levels": lvl_rows, "best_k": lv[best].ctas_per_sm, "ms_best": ms[best],
-                  "worst_k": lv[worst].ctas_per_sm, "ms_worst": ms[worst], "maxocc_k": lv[kmax].ctas_per_sm,
-                  "ms_maxocc": ms[kmax], "nvcc_default_k": lv[orig].ctas_per_sm, "ms_nvcc_default": ms[orig]},
-        "regret": t_final / ms[best] - 1.0,
-        # the paper's Fig. 11 report (P:L747-P:L755): worst level (Orion-Min), best level
-        # (Orion-Max), the nvcc build (the original), and Orion-Select = the tuned run
-        # INCLUDING its exploration iterations, over the warm-up + timed horizon
-        "fig11": {"orion_min_ms": ms[worst], "orion_max_ms": ms[best], "nvcc_ms": ms[orig],
-                  "orion_select_ms": (sum(explore_ms) + (args.warmup + args.steps - len(explore_ms)) * ms_step)
-                  / (args.warmup + args.steps),
-                  "speedup_select_vs_nvcc": ms[orig] / ((sum(explore_ms) + (args.warmup + args.steps
-                                                          - len(explore_ms)) * ms_step) / (args.warmup + args.steps)),
-                  "speedup_max_vs_nvcc": ms[orig] / ms[best], "speedup_min_vs_nvcc": ms[orig] / ms[worst]},
-        "vs_maxocc": ms[kmax] / t_final,
-        "paper_context": {"note": "context only, not a target: the paper's best speedup over nvcc (particles, "
-                                  "Table 3) on GTX680 / Tesla C2075; imageDenoising 1.08-1.12, hotspot 1.12-1.18",
-                          "paper_max_speedup_vs_nvcc": 1.61, "this_run_vs_nvcc": ms[orig] / t_final},
-        "vs_nvcc_default": ms[orig] / t_final,
-        "build_seconds": round(t_build, 2),
-        "realise": "min_carveout" if realise == O.REALISE_MIN_CARVEOUT else "max_smem",
-        "carveout_axis": carveout_axis,
-    }
-    print(json.dumps(line), flush=True)
-    if world > 1:
-        dist.destroy_process_group()
+    def tuned(mode):
+        t = O.Tuner(v, O.default_cfg(select_mode=mode, samples_per_level=args.samples))
+        for i in range(200):
+            t.step(args_pp[i % len(args_pp)], sp)
+            if t.final()[0] >= 0:
+                break
+        torch.cuda.synchronize()
+        f = t.final()[0]
+        t.close()
+        return f
+
+    lowest = tuned(O.SELECT_LOWEST_WITHIN_TOL)
+    fastest = tuned(O.SELECT_FASTEST)
+    best = min(range(n), key=lambda i: ms[i])
+    picks = {"lowest_within_tol": lowest, "fastest": fastest, "exhaustive_best": best, "max_occupancy": n - 1}
+    per_graph = max(1, min(2000, int(math.ceil(20.0 / max(ms[best], 1e-3)))))   # ~20 ms of work per replay
+    out = {}
+    for name, lvl in picks.items():
+        if lvl < 0:
+            out[name] = None
+            continue
+        t = O.Tuner(v, O.default_cfg())
+        t.resume(lvl)
+        g = t.capture([args_pp[i % len(args_pp)] for i in range(per_graph)])
+        g.launch(sp)                                   # warm
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = 0
+        with ClockSampler(local) as clk:
+            e0.record()
+            t0 = time.perf_counter()
+            while True:
+                g.launch(sp)
+                reps += 1
+                if reps % 8 == 0:
+                    torch.cuda.synchronize()
+                    if time.perf_counter() - t0 >= window_s:
+                        break
+            e1.record()
+            torch.cuda.synchronize()
+            clk.mark_end()
+        g.close()
+        t.close()
+        iters = reps * per_graph
+        en = clk.energy(iters)
+        L, inf = v.level(lvl), v.info(lvl)
+        out[name] = {"k": L.ctas_per_sm, "occupancy": L.occupancy_permille / 1000, "regs": inf.regs,
+                     "register_file_frac": inf.regs * L.warps_per_sm * 32 / 65536,
+                     "ms_per_iteration": e0.elapsed_time(e1) / iters, "sweep_ms": ms[lvl],
+                     "joules_per_iteration": en["joules_per_step"] if en else None,
+                     "mean_watts": en["mean_watts"] if en else None, "window_s": en.get("window_s") if en else None,
+                     "clocks": clk.summary()}
+    rec = {"kernel": kernel, "workload": wl["name"], "natural_regs": res.regs_per_thread, "levels": out,
+           "iterations_per_graph": per_graph}
+    lo, fa = out.get("lowest_within_tol"), out.get("exhaustive_best")
+    if lo and fa:
+        rec["registers_saved_frac"] = 1.0 - lo["register_file_frac"] / fa["register_file_frac"]
+        rec["runtime_change"] = lo["ms_per_iteration"] / fa["ms_per_iteration"] - 1.0
+        if lo["joules_per_iteration"] and fa["joules_per_iteration"]:
+            rec["energy_change"] = lo["joules_per_iteration"] / fa["joules_per_iteration"] - 1.0
+    v.close()
+    O.set_pdl(pdl_prev)
+    torch.cuda.empty_cache()
+    return rec
 
 
-def run_c5(args):
-    """C5: one 16384^2 NLM frame row-sharded over the ranks (strong scaling).  A step =
-    every rank's tuned NLM launch on its band (input slab + 6-row halo generated in place
-    before the timed region) followed by the NCCL all-gather of the output bands."""
+# ---- C5: the row-sharded frame -------------------------------------------------------------
+def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: int, group=None, size: int = 0,
+               mode_req: str = "auto", chunks_req: int = 4, e2e: bool = True):
+    """One 16384^2 NLM frame row-sharded over the `world` ranks of `group` (strong scaling).  A
+    step = every rank's tuned NLM launch on its band (input slab + 6-row halo generated in
+    place before the timed region) and the exchange of the output bands into every rank's full
+    image.  Returns the record on rank 0 of the group, else None."""
     import torch
     import torch.distributed as dist
     from paper_conf_middleware_hayeslcsz16_b200 import orion as O
     from paper_conf_middleware_hayeslcsz16_b200 import shard
 
-    world, rank, local = dist_env()
-    local = init_dist(world, local)
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream
     wl = WORKLOADS["c5"]
-    kernel = args.kernel or wl["kernel"]
-    W = H = args.size or wl["W"]
+    kernel = args.kernel if args.kernel and args.workload == "c5" else wl["kernel"]
+    W = H = size or wl["W"]
     b = shard.band(rank, world, H, 6)
     src = torch.empty((b.src_rows, W, 4), device=dev)
     O.generate_rgba(local, src.data_ptr(), W, H, b.src_begin, b.src_end, seed=1, sigma=wl["sigma"], stream=sp)
     out = torch.empty((b.rows_per_rank, W, 4), device=dev)
-    full = torch.empty((world * b.rows_per_rank, W, 4), device=dev) if world > 1 else out
-    variants, res = O.build_all_levels(local, kernel)
+    variants, res = O.build_all_levels(local, kernel, mode=O.REALISE_MIN_CARVEOUT if args.realise == "min"
+                                       else O.REALISE_MAX_SMEM)
     nlev = len(variants)
     a = O.denoise_args(kernel, src.data_ptr(), out.data_ptr(), W, H, b.row_begin, b.row_end, b.src_begin,
                        b.src_end, b.row_begin)
     ms = variants.sweep(a, sp, rounds=max(3, args.rounds // 3))
-    tuner = O.Tuner(variants)
-    # the exchange: the kernels' fan-out stores into every rank's symmetric-memory image
-    # (compute + gather in one kernel over NVLink), else chunked NCCL all-gathers
-    mode, fan, fan_note = ("none" if world == 1 and args.c5_mode != "fanout" else args.c5_mode), None, None
-    if mode == "fanout" and world == 1 and not dist.is_initialized():
-        # P = 1 with an explicit fan-out: a one-rank NCCL group exercises the symmetric-memory path
-        import socket
-        with socket.socket() as so:
-            so.bind(("127.0.0.1", 0))
-            port = so.getsockname()[1]
-        dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", world_size=1, rank=0,
-                                device_id=dev)
+    tuner = O.Tuner(variants, O.default_cfg(samples_per_level=args.samples))
+    # the exchange: the kernels' fan-out stores into every rank's symmetric-memory image (compute
+    # + gather in one kernel over NVLink), else chunked all-gathers overlapped with compute
+    mode, fan, fan_note = ("none" if world == 1 else mode_req), None, None
+    full = None
     if mode in ("auto", "fanout"):
         try:
-            fan = shard.FanoutImage((H, W, 4), dev)
+            if backend_name() != "nccl":
+                raise RuntimeError("symmetric memory needs the nccl backend")
+            fan = shard.FanoutImage((H, W, 4), dev, group)
             a = O.with_fanout(type(a).from_buffer_copy(a), fan.ptrs)
             mode = "fanout"
         except Exception as ex:   # no symmetric memory on this group / backend
             if mode == "fanout":
                 raise
-            mode, fan_note = "gather", f"fan-out unavailable ({type(ex).__name__}); chunked all-gather used"
-    for _ in range(args.warmup):
-        tuner.step(a, sp)
+            mode, fan_note = "gather", f"fan-out unavailable ({type(ex).__name__}: {ex}); chunked all-gather used"
+    if mode == "gather":
+        full = torch.empty((world * b.rows_per_rank, W, 4), device=dev)
+    chunks = max(1, chunks_req) if mode == "gather" else 1
+    per = -(-b.rows // chunks) if b.rows else 0
+    comm = torch.cuda.Stream() if mode == "gather" else None
+
+    def one_step(ev=None, recorded=None):
+        """Compute the band (as `chunks` row chunks when gathering) and exchange it."""
         if mode == "fanout":
-            fan.barrier()
-        elif world > 1:
-            shard.gather_bands(out, full)
+            tuner.step(a, sp)                 # stores its band into every rank's image
+            if ev is not None:
+                ev[1].record(stream)
+            fan.barrier()                     # every rank's stores have landed
+            return
+        if mode == "none":
+            tuner.step(a, sp)
+            if ev is not None:
+                ev[1].record(stream)
+            return
+        for c in range(chunks):
+            r0, r1 = min(b.rows, c * per), min(b.rows, (c + 1) * per)
+            if r0 >= r1:
+                continue
+            ca = O.denoise_args(kernel, src.data_ptr(), out.data_ptr(), W, H, b.row_begin + r0, b.row_begin + r1,
+                                b.src_begin, b.src_end, b.row_begin)
+            ce = None
+            if recorded is not None:
+                ce = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                ce[0].record(stream)
+            tuner.step(ca, sp)
+            if ce is not None:
+                ce[1].record(stream)
+                recorded.append(ce)
+            comm.wait_stream(stream)
+            with torch.cuda.stream(comm):
+                shard.gather_rows(out, full, b.rows_per_rank, r0, r1, group=group)
+        if ev is not None:
+            ev[1].record(stream)
+        stream.wait_stream(comm)
+
+    for _ in range(warmup):
+        one_step()
     torch.cuda.synchronize()
     if world > 1:
-        dist.barrier()
+        dist.barrier(group=group)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
-           torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    chunks = max(1, args.c5_chunks) if mode == "gather" else 1
+           torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    recorded = [] if mode == "gather" else None
     n0 = O.launch_count()
-    if mode == "fanout":
-        with ClockSampler(local) as clk:
-            for e0, e1, e2 in ev:
-                e0.record(stream)
-                tuner.step(a, sp)            # stores its band into every rank's image
-                e1.record(stream)
-                fan.barrier()                # every rank's stores have landed
-                e2.record(stream)
-            torch.cuda.synchronize()
-        comp = sum(e0.elapsed_time(e1) for e0, e1, _ in ev)
-        gat = sum(e1.elapsed_time(e2) for _, e1, e2 in ev)
-    elif chunks == 1:
-        with ClockSampler(local) as clk:
-            for e0, e1, e2 in ev:
-                e0.record(stream)
-                tuner.step(a, sp)
-                e1.record(stream)
-                if world > 1:
-                    shard.gather_bands(out, full)
-                e2.record(stream)
-            torch.cuda.synchronize()
-        comp = sum(e0.elapsed_time(e1) for e0, e1, _ in ev)
-        gat = sum(e1.elapsed_time(e2) for _, e1, e2 in ev)
-    else:
-        # overlap: the band is split into row chunks (kernel splitting); chunk c's all-gather
-        # runs on a side stream while chunk c+1 is being computed
-        comm = torch.cuda.Stream()
-        per = -(-b.rows // chunks)
-        cev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-                for _ in range(chunks)] for _ in range(args.steps)]
-        recorded = []
-        with ClockSampler(local) as clk:
-            for s_, (e0, e1, e2) in enumerate(ev):
-                e0.record(stream)
-                for c in range(chunks):
-                    r0, r1 = min(b.rows, c * per), min(b.rows, (c + 1) * per)
-                    if r0 >= r1:
-                        continue
-                    ca = O.denoise_args(kernel, src.data_ptr(), out.data_ptr(), W, H, b.row_begin + r0,
-                                        b.row_begin + r1, b.src_begin, b.src_end, b.row_begin)
-                    cev[s_][c][0].record(stream)
-                    tuner.step(ca, sp)
-                    cev[s_][c][1].record(stream)
-                    recorded.append(cev[s_][c])
-                    comm.wait_stream(stream)
-                    with torch.cuda.stream(comm):
-                        shard.gather_rows(out, full, b.rows_per_rank, r0, r1)
-                e1.record(stream)
-                stream.wait_stream(comm)
-                e2.record(stream)
-            torch.cuda.synchronize()
-        comp = sum(x.elapsed_time(y) for (x, y) in recorded)
-        gat = sum(e1.elapsed_time(e2) for _, e1, e2 in ev)   # the gather tail not hidden by compute
+    with ClockSampler(local) as clk:
+        for e in ev:
+            e[0].record(stream)
+            one_step(e, recorded)
+            e[2].record(stream)
+        torch.cuda.synchronize()
+        clk.mark_end()
     launches = O.launch_count() - n0
     tot = ev[0][0].elapsed_time(ev[-1][2])
-    t = torch.tensor([tot, comp, gat], device=dev)
+    if recorded is not None:
+        comp = sum(x.elapsed_time(y) for (x, y) in recorded)
+    else:
+        comp = sum(e0.elapsed_time(e1) for e0, e1, _ in ev)
+    gat = sum(e1.elapsed_time(e2) for _, e1, e2 in ev)   # the exchange tail not hidden by compute
+
+    # ---- end to end: pinned host slab -> device, tuned step + exchange, own band -> host -------
+    e2e_rec = None
+    if e2e:
+        h_src = torch.empty((b.src_rows, W, 4), pin_memory=True)
+        h_src.copy_(src)
+        h_out = torch.empty((b.rows, W, 4), pin_memory=True)
+        n_e2e = max(2, min(steps, 4))
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier(group=group)
+        t0 = time.perf_counter()
+        for _ in range(n_e2e):
+            src.copy_(h_src, non_blocking=True)
+            one_step()
+            h_out.copy_(out[:b.rows], non_blocking=True)
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        e2e_rec = [dt, float(b.src_rows * W * 16), float(b.rows * W * 16), n_e2e]
+        del h_src, h_out
+    t = torch.tensor([tot, comp, gat] + ([e2e_rec[0]] if e2e_rec else [0.0]), device=dev)
     final, it = tuner.final()
-    chosen = [variants.level(final).ctas_per_sm if final >= 0 else -1, it, t_best_k(variants, ms)]
+    chosen = [variants.level(final).ctas_per_sm if final >= 0 else -1, it,
+              variants.level(min(range(nlev), key=lambda k: ms[k])).ctas_per_sm, b.row_begin, b.row_end]
+    byts = torch.tensor([e2e_rec[1], e2e_rec[2]] if e2e_rec else [0.0, 0.0], device=dev, dtype=torch.float64)
     if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+        dist.all_reduce(byts, op=dist.ReduceOp.SUM, group=group)
         allc = [None] * world
-        dist.all_gather_object(allc, chosen)
+        dist.all_gather_object(allc, chosen, group=group)
     else:
         allc = [chosen]
-    tot, comp, gat = (float(x) for x in t.tolist())
+    tot, comp, gat, e2e_dt = (float(x) for x in t.tolist())
+    rec = None
     if rank == 0:
-        peaks, peak_kind = load_peaks()
-        kernel_ms = comp / args.steps
-        peak = 148 * 128 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6 / 1e12
-        achieved = wl["insts"] * b.rows * W / (kernel_ms * 1e-3) / 1e12
-        line = {
-            "metric": METRIC, "value": H * W * args.steps / (tot * 1e-3) / 1e6, "unit": "Mpix/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot / args.steps, "higher_is_better": True,
+        kernel_ms = comp / steps
+        roof = _roofline(kernel, wl, b.rows * W, kernel_ms)
+        roof["note"] = "per rank: rank 0's band of rows per kernel millisecond"
+        rec = {
+            "metric": METRIC, "value": H * W * steps / (tot * 1e-3) / 1e6, "unit": "Mpix/s", "n_gpus": world,
+            "steps": steps, "warmup": warmup, "ms_per_step": tot / steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": wl["name"], "kernel": kernel, "width": W, "height": H,
+            "config": {"workload": wl["name"], "baseline_config_index": 4, "kernel": kernel, "width": W, "height": H,
                        "rows_per_rank": b.rows_per_rank, "halo_rows": 6,
                        "collective": ("kernel fan-out stores into every rank's symmetric-memory image over NVLink "
                                       "+ device barrier" if mode == "fanout" else
                                       f"all_gather of {chunks} row chunks on a side stream, overlapped with the "
-                                      f"next chunk's kernel" if chunks > 1 else "all_gather_into_tensor (NCCL)")
-                       if world > 1 else "none (P=1)", "collective_note": fan_note, "l2": "4 GiB frame >> L2",
-                       "parallelism": f"row-sharded x{world}"},
-            "compute_only": {"value": H * W * args.steps / (comp * 1e-3) / 1e6, "unit": "Mpix/s",
-                             "ms_per_step": comp / args.steps},
-            "allgather_ms_per_step": gat / args.steps,
-            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tinst/s (FP32 pipe lane-ops)",
-                         "frac": achieved / peak, "kernel": kernel, "peak_kind": peak_kind},
-            "per_rank": [{"rank": r, "final_k": c[0], "iterations_to_final": c[1], "sweep_best_k": c[2]}
-                         for r, c in enumerate(allc)],
+                                      f"next chunk's kernel" if mode == "gather" else "none (P=1)"),
+                       "collective_note": fan_note, "l2": "4 GiB frame >> L2",
+                       "parallelism": f"row-sharded x{world}", "backend": backend_name() if world > 1 else None},
+            "compute_only": {"value": H * W * steps / (comp * 1e-3) / 1e6, "unit": "Mpix/s",
+                             "ms_per_step": comp / steps},
+            "exchange_ms_per_step": gat / steps,
+            "roofline": roof,
+            "per_rank": [{"rank": r, "final_k": c[0], "iterations_to_final": c[1], "sweep_best_k": c[2],
+                          "rows": [c[3], c[4]]} for r, c in enumerate(allc)],
             "sweep_rank0": [{"k": variants.level(i).ctas_per_sm, "ms": round(ms[i], 4)} for i in range(nlev)],
-            "gpu_launches": launches, "clocks": clk.summary(), "energy": clk.energy(args.steps),
-            "e2e": {"value": None, "unit": "Mpix/s", "note": "C5 inputs are generated in place per rank"},
+            "regret_rank0": (ms[final] / min(ms) - 1.0) if final >= 0 else None,
+            "gpu_launches": launches, "clocks": clk.summary(), "energy": clk.energy(steps),
+            "e2e": ({"value": H * W * e2e_rec[3] / e2e_dt / 1e6, "unit": "Mpix/s",
+                     "h2d_bytes_per_step": float(byts[0]), "d2h_bytes_per_step": float(byts[1]),
+                     "steps": e2e_rec[3],
+                     "api": "per rank: pinned host slab (+ halo) -> device, orion_tune_step + exchange, "
+                            "own output band -> pinned host; bytes summed over ranks"} if e2e_rec else None),
             "cpu_baseline": None,
         }
+    tuner.close()
+    variants.close()
+    del src, out, full, fan
+    torch.cuda.empty_cache()
+    return rec
+
+
+# ---- drivers ------------------------------------------------------------------------------------
+def run_single(args):
+    """N = 1: the headline configuration and (unless --only) every other one as a sub-record."""
+    import torch
+    world, rank, local = dist_env()
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py: no CUDA device (the product has no CPU path)")
+    local = init_dist(world, local)
+    key = args.workload
+    wl = WORKLOADS[key]
+    steps = args.steps or wl["steps"]
+    if key == "c5":
+        line = measure_c5(args, world=1, rank=0, local=local, steps=steps, warmup=args.warmup, size=args.size,
+                          mode_req=args.c5_mode, chunks_req=args.c5_chunks)
         print(json.dumps(line), flush=True)
+        return
+    t0 = time.perf_counter()
+    line = measure_single(key, args, steps=steps, warmup=args.warmup, rounds=args.rounds,
+                          cpu_seconds=0 if args.no_cpu_baseline else args.cpu_seconds,
+                          carveout_axis=not args.no_carveout_axis, kernel=args.kernel or None, select=args.select,
+                          local=local)
+    line["seconds"] = round(time.perf_counter() - t0, 1)
+    if not args.only:
+        subs = {}
+        for sub in SUB_RECORDS:
+            if sub == key:
+                continue
+            t1 = time.perf_counter()
+            try:
+                if sub == "c5":
+                    r = measure_c5(args, world=1, rank=0, local=local, steps=WORKLOADS["c5"]["steps"], warmup=3)
+                else:
+                    r = measure_single(sub, args, steps=WORKLOADS[sub]["steps"], warmup=max(args.warmup, 12),
+                                       rounds=5 if sub == "c4" else args.rounds,
+                                       cpu_seconds=0 if args.no_cpu_baseline else args.sub_cpu_seconds,
+                                       carveout_axis=sub != "c4", select="fastest", local=local)
+                r["seconds"] = round(time.perf_counter() - t1, 1)
+            except Exception as ex:                           # reported, never silently dropped
+                r = {"error": f"{type(ex).__name__}: {ex}"}
+            subs[sub] = r
+        line["configs"] = subs
+        if not args.no_energy:
+            nx = {}
+            for sub, kern in (("srad", "srad_f32h"), ("c3", "hotspot_f32"), ("c1", "knn_f4_t16"), ("c4", "nlm_f4_regheavy")):
+                try:
+                    nx[f"{sub}:{kern}"] = measure_energy(sub, args, kern, local=local)
+                except Exception as ex:
+                    nx[f"{sub}:{kern}"] = {"error": f"{type(ex).__name__}: {ex}"}
+            line["next3_energy"] = nx
+    line["seconds_total"] = round(time.perf_counter() - t0, 1)
+    print(json.dumps(line), flush=True)
+
+
+def run_multi(args):
+    """N > 1 (one process per GPU): C5 row-sharded over every rank, with C5 at P = 1 (rank 0
+    alone, the curve's anchor) in the same line."""
+    import torch
+    import torch.distributed as dist
+    world, rank, local = dist_env()
+    if args.gpus and args.gpus != world:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}")
+    local = init_dist(world, local)
+    steps = args.steps or WORKLOADS["c5"]["steps"]
+    anchor = None
+    if not args.no_anchor:
+        if rank == 0:
+            anchor = measure_c5(args, world=1, rank=0, local=local, steps=steps, warmup=3, size=args.size,
+                                e2e=False)
+        dist.barrier()
+    line = measure_c5(args, world=world, rank=rank, local=local, steps=steps, warmup=args.warmup, size=args.size,
+                      mode_req=args.c5_mode, chunks_req=args.c5_chunks)
+    if rank == 0:
+        if anchor is not None:
+            line["c5_p1_anchor"] = {k: anchor[k] for k in ("value", "ms_per_step", "compute_only", "per_rank",
+                                                           "roofline", "clocks")}
+            line["speedup_vs_p1"] = line["value"] / anchor["value"]
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def run_plumbing_check(args):
+    """CPU-only check of the multi-rank plumbing (tests/test_bench_host.py, gloo): the spawn, the
+    row bands + halos, the gather and the max-over-ranks reduction, with the per-band compute
+    replaced by a COPY of the band's own input rows (a stand-in, not the method: no kernel runs,
+    nothing is measured).  Rank 0 prints one JSON line saying whether the gathered image equals
+    the generated one."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import synth
+    from paper_conf_middleware_hayeslcsz16_b200 import shard
+    world, rank, _ = dist_env()
     if world > 1:
+        dist.init_process_group("gloo")
+    W, H = 23, args.size or 37
+    b = shard.band(rank, world, H, 6)
+    slab = torch.from_numpy(synth.noisy_rgba(W, H, seed=5, row_begin=b.src_begin, row_end=b.src_end))
+    out = torch.zeros((b.rows_per_rank, W, 4))
+    out[:b.rows] = slab[b.row_begin - b.src_begin:b.row_end - b.src_begin]     # stand-in for the kernel
+    full = torch.empty((world * b.rows_per_rank, W, 4))
+    t0 = time.perf_counter()
+    if world > 1:
+        shard.gather_bands(out, full)
+    else:
+        full = out
+    dt = torch.tensor([time.perf_counter() - t0 + rank * 1e-3])
+    if world > 1:
+        dist.all_reduce(dt, op=dist.ReduceOp.MAX)
+        allb = [None] * world
+        dist.all_gather_object(allb, [b.row_begin, b.row_end, b.src_begin, b.src_end])
+    else:
+        allb = [[b.row_begin, b.row_end, b.src_begin, b.src_end]]
+    if rank == 0:
+        ok = bool(np.array_equal(full[:H].numpy(), synth.noisy_rgba(W, H, seed=5)))
+        print(json.dumps({"plumbing_check": True, "n_gpus": world, "ok": ok, "bands": allb,
+                          "max_over_ranks_s": float(dt.item()), "spawned": os.environ.get("ORION_BENCH_SPAWNED")}),
+              flush=True)
+    if world > 1:
+        dist.barrier()
         dist.destroy_process_group()
 
 
-def t_best_k(variants, ms):
-    i = min(range(len(ms)), key=lambda k: ms[k])
-    return variants.level(i).ctas_per_sm
-
-
-def main():
+def main(argv=None):
+    argv = sys.argv[1:] if argv is None else argv
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=300)
+    ap.add_argument("--steps", type=int, default=0, help="timed steps (0: the workload's default)")
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", choices=sorted(WORKLOADS), default="c2")
+    ap.add_argument("--only", action="store_true", help="the headline workload alone (no sub-records)")
     ap.add_argument("--rounds", type=int, default=11, help="interleaved rounds of the exhaustive sweep")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--sub-cpu-seconds", type=float, default=3.0)
+    ap.add_argument("--no-energy", action="store_true", help="skip the NEXT-3 energy record")
+    ap.add_argument("--no-anchor", action="store_true", help="N > 1: skip C5 at P = 1 on rank 0")
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
-    ap.add_argument("--kernel", default="", help="override the workload's kernel id (same family)")
+    ap.add_argument("--kernel", default="", help="override the headline workload's kernel id (same family)")
     ap.add_argument("--c5-chunks", type=int, default=4, help="C5: row chunks per band whose all-gathers overlap compute")
     ap.add_argument("--c5-mode", default="auto", choices=("auto", "fanout", "gather"),
                     help="C5 exchange: kernel fan-out into symmetric memory (auto: when available) or all-gather")
@@ -825,9 +1127,7 @@ def main():
                          "issue them in one library call (orion_tune_steps); off: one Python call per "
                          "iteration; auto = on for the launch-bound C1 frames, off otherwise")
     ap.add_argument("--async-timing", type=int, default=0, choices=(0, 1),
-                    help="1: the tuner reads its event pairs without host synchronisation "
-                         "(orion_tuner_cfg.async_timing; exploration then spans as many iterations as the host "
-                         "runs ahead of the GPU)")
+                    help="1: the tuner reads its event pairs without host synchronisation")
     ap.add_argument("--samples", type=int, default=2,
                     help="timed launches per explored level, the fastest kept (paper: 1; reading R-A11)")
     ap.add_argument("--select", choices=["fastest", "lowest"], default="fastest",
@@ -835,19 +1135,26 @@ def main():
     ap.add_argument("--realise", choices=["max", "min"], default="min",
                     help="level realisation: max = pad against 228 KB smem; min = smallest carveout (more L1)")
     ap.add_argument("--no-carveout-axis", action="store_true", help="skip the sweep of the other realisation")
-    args = ap.parse_args()
+    ap.add_argument("--plumbing-check", action="store_true", help=argparse.SUPPRESS)
+    args = ap.parse_args(argv)
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
-    if args.graph == "on" or (args.graph == "auto" and args.workload == "c1"):
-        # graph kernel nodes are plain launches; the sweep must time the levels the same way, so
-        # this process launches without programmatic dependent launch (liborion reads it once)
-        os.environ.setdefault("ORION_PDL", "0")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        if not args.plumbing_check and backend_name() == "nccl":
+            import torch
+            if torch.cuda.device_count() < args.gpus:
+                raise SystemExit(f"bench.py: --gpus {args.gpus} but {torch.cuda.device_count()} CUDA device(s)")
+        sys.exit(spawn(args.gpus, argv))
+    if args.plumbing_check:
+        run_plumbing_check(args)
+        return
+    world = int(os.environ.get("WORLD_SIZE", "1"))
     if args.impl == "reference":
         run_reference(args)
-    elif args.workload == "c5":
-        run_c5(args)
+    elif world > 1:
+        run_multi(args)
     else:
-        run_ours(args)
+        run_single(args)
 
 
 if __name__ == "__main__":

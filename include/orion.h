@@ -179,7 +179,8 @@ void orion_variants_destroy(orion_variants *v);
  *  hotspot:   src = T (float), aux = power (same rows as src), dst = T'; fparam[0..4] =
  *             sdc (step/Cap), rx = 1/Rx, ry = 1/Ry, rz = 1/Rz, amb (reading R-O3/R-A15).
  *             src must hold rows row_begin-1 .. row_end (clamped).
- *  fan-out (kernels "knn_f4", "nlm_f4", "nlm_f4_i", "nlm_f4_w8", "nlm_f4_g1"): every output
+ *  fan-out (every box-sum NLM kernel "nlm_f4*" except "nlm_f4_direct", every KNN kernel
+ *             "knn_f4*"; not the stencils or "nlm_f4_regheavy"): every output
  *             pixel is also stored into fanout[0 .. n_fanout) -- full width x height images
  *             (global row y at y * width), device pointers in this GPU's memory or a peer's
  *             reachable over NVLink (P2P / symmetric memory) -- so a row-sharded frame is
@@ -198,8 +199,17 @@ typedef struct {
     int n_fanout;
 } orion_args;
 
-/* Launch variant `level_idx` (realising its occupancy level) on `stream` (async). */
+/* Launch variant `level_idx` (realising its occupancy level, P:L649, P:L757-P:L759) on
+ * `stream` (async).  An empty row range (row_begin == row_end) is a no-op returning ORION_OK.
+ * Every launch uses programmatic dependent launch unless it is disabled (ORION_PDL=0 in the
+ * environment, or orion_set_pdl(0, ..)); results are the same bits either way. */
 orion_status orion_launch(orion_variants *v, int level_idx, const orion_args *a, void *stream);
+
+/* Process-wide switch of programmatic dependent launch for every later launch (initially
+ * from ORION_PDL; default on).  `on` is 0 or 1 (else ORION_E_INVALID); *previous (may be
+ * NULL) receives the setting it replaces.  A loop that will be replayed as a CUDA graph (graph
+ * nodes are plain launches) turns it off so that the sweep times the levels the same way. */
+orion_status orion_set_pdl(int on, int *previous);
 
 /* Exhaustive occupancy sweep (Fig. 11's Orion-Min / Orion-Max methodology, P:L747-P:L755):
  * `rounds` rounds, each launching every level once in round-robin order (interleaving

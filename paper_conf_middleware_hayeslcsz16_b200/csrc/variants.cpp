@@ -17,6 +17,8 @@
 #include <string>
 #include <vector>
 
+#include <atomic>
+
 #include "orion_internal.h"
 
 using namespace orion;
@@ -29,6 +31,7 @@ int warps_of(const orion_device_limits &d, int T) { return (T + d.warp_size - 1)
 // the source slab holds every row the kernel reaches (clamped to the image).
 orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *k)
 {
+    std::memset(k, 0, sizeof *k);          // an empty launch still hands back a defined block
     if (!a) return fail(ORION_E_INVALID, "orion_launch: NULL args");
     if (a->width <= 0 || a->height <= 0 || a->row_begin < 0 || a->row_end > a->height || a->row_begin > a->row_end)
         return fail(ORION_E_INVALID, "orion_launch: bad image geometry");
@@ -47,7 +50,6 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
         return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + ": bad n_fanout");
     for (int f = 0; f < a->n_fanout; ++f)
         if (!a->fanout[f]) return fail(ORION_E_INVALID, "orion_launch: NULL fanout buffer");
-    std::memset(k, 0, sizeof *k);
     for (int f = 0; f < a->n_fanout; ++f) k->fan[f] = a->fanout[f];
     k->nfan = a->n_fanout;
     k->src = a->src;
@@ -78,13 +80,28 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
 // Launches use programmatic stream serialization (PDL) unless ORION_PDL=0, and never while a
 // graph is being captured.  Measured A/B on one box (same library, ORION_PDL=0 vs 1): C2
 // 0.2217 -> 0.2197 ms, SRAD 0.1044 -> 0.1029 ms, C3 0.1571 -> 0.1564 ms per launch.
+// -1: not yet read from ORION_PDL; orion_set_pdl() overrides it at run time.
+static std::atomic<int> g_pdl{-1};
+
 static bool pdl_enabled()
 {
-    static const bool on = [] {
+    int on = g_pdl.load();
+    if (on < 0) {
         const char *e = std::getenv("ORION_PDL");
-        return !(e && e[0] == '0');
-    }();
+        int want = (e && e[0] == '0') ? 0 : 1;
+        g_pdl.compare_exchange_strong(on, want);
+        on = g_pdl.load();
+    }
     return on && !t_capturing;
+}
+
+static int pdl_enabled_setting()
+{
+    const bool cap = t_capturing;
+    t_capturing = false;
+    const int on = pdl_enabled() ? 1 : 0;
+    t_capturing = cap;
+    return on;
 }
 
 // Programmatic dependent launch when enabled: this grid may be scheduled while the previous
@@ -323,11 +340,24 @@ orion_status orion_launch(orion_variants *v, int i, const orion_args *a, void *s
     return launch_fn(*v->def, w.fn, w.dyn_bytes, k, (CUstream)stream);
 }
 
+orion_status orion_set_pdl(int on, int *previous)
+{
+    if (on != 0 && on != 1) return fail(ORION_E_INVALID, "orion_set_pdl: on must be 0 or 1");
+    const int was = pdl_enabled_setting();
+    g_pdl.store(on);
+    if (previous) *previous = was;
+    return ORION_OK;
+}
+
 orion_status orion_sweep(orion_variants *v, const orion_args *a, void *stream, int rounds, float *ms_median)
 {
     if (!v || !a || rounds <= 0 || !ms_median) return fail(ORION_E_INVALID, "orion_sweep: bad argument");
     orion_kargs k;
     ORION_TRY(make_kargs(*v->def, a, &k));
+    if (a->row_begin == a->row_end) {     // nothing to time: an empty launch is a no-op at every level
+        for (size_t i = 0; i < v->vars.size(); ++i) ms_median[i] = 0.0f;
+        return ORION_OK;
+    }
     ORION_TRY(ensure_context(v->device));
     const Driver &D = drv();
     const int n = (int)v->vars.size();

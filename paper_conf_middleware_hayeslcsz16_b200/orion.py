@@ -155,6 +155,7 @@ def lib() -> ctypes.CDLL:
                 "orion_tuner_ladder": [V, P(I), P(I), I, P(I)],
                 "orion_tuner_final": [V, P(I), P(I)],
                 "orion_tuner_tried": [V, P(ctypes.c_float), I],
+                "orion_set_pdl": [I, P(I)],
                 "orion_tuner_replay": [P(TunerCfg), P(Level), I, I, P(ctypes.c_float), I, P(I), P(I), P(I)],
                 "orion_generate_rgba": [I, V, I, I, I, I, ctypes.c_uint, ctypes.c_float, V],
                 "orion_generate_thermal": [I, V, V, I, I, ctypes.c_uint, V],
@@ -546,6 +547,14 @@ def srad_roi_stats(device: int, j: int, width: int, height: int, roi, q0: int, s
 
 def flush_l2(device: int, buf: int, nbytes: int, stream=None):
     _check(lib().orion_flush_l2(device, ctypes.c_void_p(buf), nbytes, _s(stream)), "orion_flush_l2")
+
+
+def set_pdl(on: bool) -> bool:
+    """orion_set_pdl: programmatic dependent launch on / off for later launches; returns the
+    previous setting."""
+    prev = ctypes.c_int()
+    _check(lib().orion_set_pdl(1 if on else 0, ctypes.byref(prev)), "orion_set_pdl")
+    return bool(prev.value)
 
 
 def launch_count() -> int:

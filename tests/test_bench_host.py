@@ -36,3 +36,34 @@ def test_energy_long_window(bench):
 
 def test_energy_unavailable(bench):
     assert _sampler(bench, None, 5, 0.0, 1.0).energy(1) is None
+
+
+def test_spawn_command_is_one_process_per_gpu(bench):
+    cmd = bench.spawn_command(4, ["--steps", "3"], 29555)
+    assert cmd[1:3] == ["-m", "torch.distributed.run"]
+    assert "--nproc-per-node=4" in cmd and "--master-addr=127.0.0.1" in cmd and "--master-port=29555" in cmd
+    assert cmd[-3:] == [os.path.join(ROOT, "bench.py"), "--steps", "3"]
+
+
+@pytest.mark.parametrize("n,height", [(2, 37), (3, 20), (1, 9)])
+def test_gpus_flag_spawns_ranks_gloo_plumbing(n, height):
+    # `bench.py --gpus N` without torchrun re-launches itself on N ranks; the plumbing check
+    # (CPU, gloo: bands + halos, gather, max over ranks; the kernel replaced by a copy) must
+    # print exactly ONE JSON line, from rank 0, with n_gpus = N and the gathered image intact.
+    import json
+    import subprocess
+    import sys
+    env = dict(os.environ, ORION_BENCH_BACKEND="gloo", OMP_NUM_THREADS="1")
+    env.pop("WORLD_SIZE", None)
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", str(n), "--plumbing-check",
+                        "--size", str(height)], capture_output=True, text=True, env=env, timeout=300, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["plumbing_check"] and d["ok"] and d["n_gpus"] == n
+    if n > 1:
+        assert d["spawned"] == "1"
+        rows = [b[:2] for b in d["bands"]]
+        assert rows[0][0] == 0 and rows[-1][1] == height
+        assert all(rows[k][1] == rows[k + 1][0] for k in range(n - 1))
