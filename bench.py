@@ -86,6 +86,8 @@ class ClockSampler:
                0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
                0x100: "display_clock_setting"}
 
+    MIN_WINDOW_S = 1.0
+
     def __init__(self, index: int, period: float = 0.02):
         self.samples, self.reasons, self.ok = [], set(), False
         self.period = period
@@ -146,11 +148,12 @@ class ClockSampler:
             return None
         j = (self.e1 - self.e0) / 1e3
         window = self.t1 - self.t0
-        if j <= 0 or window < 0.05:
-            # The board counter advances in coarse ticks: a short timed region reads 0 J,
-            # which is not a measurement.
+        if j <= 0 or window < self.MIN_WINDOW_S:
+            # The board counter advances in coarse ticks: a short timed region reads 0 J or a
+            # few ticks, which is not a measurement (next3_energy uses >= 1.2 s windows).
             return {"joules_per_step": None, "mean_watts": None, "source": "nvml total energy",
-                    "note": f"timed region {window * 1e3:.1f} ms is below the counter's update period"}
+                    "note": f"timed region {window * 1e3:.1f} ms is below the {self.MIN_WINDOW_S:.1f} s "
+                            f"energy window"}
         return {"joules_per_step": j / steps, "mean_watts": j / window, "window_s": window,
                 "source": "nvml total energy"}
 
@@ -652,7 +655,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
                        "cuda_graph": graph is not None,
                        "issue": "graph" if graph is not None else ("orion_tune_steps" if native_args is not None
                                                                    else "orion_tune_step per step")},
-            "roofline": _roofline(kernel, wl, W * H * spl, ms_step),
+            "roofline": _roofline(kernel, wl, W * H, ms_step),      # bytes / instructions per cell or pixel per launch
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
             "energy": clk.energy(steps), "select_mode": select,
             "resources": {"final_regs": infos[final].regs if final >= 0 else None,
@@ -787,12 +790,16 @@ def measure_energy(key: str, args, kernel: str, local: int = 0, window_s: float 
                      "clocks": clk.summary()}
     rec = {"kernel": kernel, "workload": wl["name"], "natural_regs": res.regs_per_thread, "levels": out,
            "iterations_per_graph": per_graph}
-    lo, fa = out.get("lowest_within_tol"), out.get("exhaustive_best")
-    if lo and fa:
-        rec["registers_saved_frac"] = 1.0 - lo["register_file_frac"] / fa["register_file_frac"]
-        rec["runtime_change"] = lo["ms_per_iteration"] / fa["ms_per_iteration"] - 1.0
-        if lo["joules_per_iteration"] and fa["joules_per_iteration"]:
-            rec["energy_change"] = lo["joules_per_iteration"] / fa["joules_per_iteration"] - 1.0
+    lo = out.get("lowest_within_tol")
+    for ref in ("exhaustive_best", "max_occupancy"):
+        fa = out.get(ref)
+        if lo and fa:
+            c = {"registers_saved_frac": 1.0 - lo["register_file_frac"] / fa["register_file_frac"],
+                 "warps_saved_frac": 1.0 - lo["occupancy"] / fa["occupancy"],
+                 "runtime_change": lo["ms_per_iteration"] / fa["ms_per_iteration"] - 1.0}
+            if lo["joules_per_iteration"] and fa["joules_per_iteration"]:
+                c["energy_change"] = lo["joules_per_iteration"] / fa["joules_per_iteration"] - 1.0
+            rec[f"lowest_vs_{ref}"] = c
     v.close()
     O.set_pdl(pdl_prev)
     torch.cuda.empty_cache()

@@ -28,10 +28,12 @@ def test_energy_short_window_is_null(bench):
 
 
 def test_energy_long_window(bench):
-    # 600 J over 1 s and 100 steps: 6 J per step, 600 W
-    e = _sampler(bench, 1_000_000, 1_600_000, 10.0, 11.0).energy(100)
-    assert e["joules_per_step"] == pytest.approx(6.0)
+    # 720 J over 1.2 s and 100 steps: 7.2 J per step, 600 W
+    e = _sampler(bench, 1_000_000, 1_720_000, 10.0, 11.2).energy(100)
+    assert e["joules_per_step"] == pytest.approx(7.2)
     assert e["mean_watts"] == pytest.approx(600.0)
+    # a 0.3 s window is below the 1 s energy window: null, not a number
+    assert _sampler(bench, 1_000_000, 1_300_000, 10.0, 10.3).energy(100)["joules_per_step"] is None
 
 
 def test_energy_unavailable(bench):
