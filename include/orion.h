@@ -153,8 +153,9 @@ typedef struct orion_variants orion_variants;   /* opaque, library-owned */
  * SM; the driver may run a padded launch in a larger carveout configuration than requested,
  * which the API does not model).  A level whose planned configuration does not measure k is
  * retried in each larger configuration; none -> ORION_E_OCCUPANCY_MISMATCH.  The probe
- * launches (148 x 32 CTAs, ~1 ms) run on the legacy default stream during the build.  Every variant is launched once (warm-up, defeats lazy
- * loading) only when orion_launch is first called with it. */
+ * launches (148 x 32 CTAs, ~1 ms) run on the legacy default stream during the build; they
+ * also load every module (no lazy loading inside a later timed launch).  orion_sweep warms
+ * and times each level once more before its timed rounds. */
 orion_status orion_build_variants(int device, const char *kernel_id, int block_threads,
                                   const orion_level *levels, int n, orion_variants **out);
 orion_status orion_variants_count(const orion_variants *v, int *n);
@@ -204,6 +205,17 @@ typedef struct {
  * Every launch uses programmatic dependent launch unless it is disabled (ORION_PDL=0 in the
  * environment, or orion_set_pdl(0, ..)); results are the same bits either way. */
 orion_status orion_launch(orion_variants *v, int level_idx, const orion_args *a, void *stream);
+
+/* The method parameters of a kernel family, written into fparam[0 .. n) (n >= 8; the rest
+ * zero) -- what orion_args.fparam holds for a launch with the defaults:
+ *   "knn_f4*": Noise = 1/0.32^2, lerpC = 0.2, weight threshold 0.02, lerp threshold 0.79;
+ *   "nlm_f4*": Noise = 1/1.45^2, 0.2, 0.10, 0.10  (CUDA-SDK imageDenoising [20], P:L91,
+ *              the paper names the benchmark, not its math: reading R-O2);
+ *   "hotspot*": sdc = step/Cap, rx, ry, rz, amb = 80 -- Rodinia hotspot ([6], Table 2
+ *              P:L731) at the 512-grid's 31.25 um cell for every grid size (readings R-O3, R-A15);
+ *   "srad*":   lambda = 0.5 (Rodinia srad_v2, Table 2; reading R-SRAD).
+ * ORION_E_INVALID for an unknown id or n < 8.  Host-only. */
+orion_status orion_default_params(const char *kernel_id, float *fparam, int n);
 
 /* Process-wide switch of programmatic dependent launch for every later launch (initially
  * from ORION_PDL; default on).  `on` is 0 or 1 (else ORION_E_INVALID); *previous (may be
@@ -264,7 +276,9 @@ typedef struct {
  * first iteration runs the original; then the next ladder level while runtimes do not
  * degrade ("Worse runtime?" when increasing, "Slowdown > .02?" vs the best when
  * decreasing); then the final kernel every iteration.  Exploration iterations record a
- * CUDA event pair and synchronise on it; final iterations only enqueue the launch. */
+ * CUDA event pair and synchronise on it; final iterations only enqueue the launch.  An empty
+ * row range (row_begin == row_end) is not an iteration: nothing runs, *out reports
+ * iteration = level_idx = phase = -1, ORION_OK. */
 orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, orion_step_report *out);
 /* The measured time of an exploring iteration is work-normalised (ns per output element,
  * P:L975) before Fig. 9 compares it, so iterations of different sizes compare fairly. */

@@ -2,6 +2,7 @@
 #include <dlfcn.h>
 
 #include <cstdio>
+#include <map>
 #include <mutex>
 
 #include "orion_internal.h"
@@ -74,10 +75,23 @@ orion_status ensure_context(int device)
         ORION_CU(d.cuDeviceGet(&want, device));
         if (cd == want) return ORION_OK;
     }
-    CUdevice dev;
-    ORION_CU(d.cuDeviceGet(&dev, device));
-    CUcontext ctx;
-    ORION_CU(d.cuDevicePrimaryCtxRetain(&ctx, dev));
+    // each device's primary context is retained ONCE per process (the reference is held for
+    // the library's lifetime and released at unload); later switches reuse the cached handle
+    static std::mutex mu;
+    static std::map<int, CUcontext> retained;
+    CUcontext ctx = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = retained.find(device);
+        if (it != retained.end()) {
+            ctx = it->second;
+        } else {
+            CUdevice dev;
+            ORION_CU(d.cuDeviceGet(&dev, device));
+            ORION_CU(d.cuDevicePrimaryCtxRetain(&ctx, dev));
+            retained[device] = ctx;
+        }
+    }
     ORION_CU(d.cuCtxSetCurrent(ctx));
     return ORION_OK;
 }

@@ -103,7 +103,6 @@ struct orion_variants {
         CUmodule mod = nullptr;
         CUfunction fn = nullptr;
         int regs = 0, local_bytes = 0, verified = 0, dyn_bytes = 0, carveout_pct = -1;
-        bool warmed = false;
     };
     std::vector<Var> vars;
 };

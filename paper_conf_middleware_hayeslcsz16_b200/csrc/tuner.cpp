@@ -246,7 +246,7 @@ static void feed_sample(orion_tuner *t, int lvl, float ms, double work)
     Fig9 &f = t->f;
     // work-normalised runtime: ns per output element, so iterations of
     // different sizes -- the bands of a split frame -- compare fairly
-    const float per = work > 0 ? (float)(ms * 1e6 / work) : ms;
+    const float per = (float)(ms * 1e6 / work);      // work > 0: empty bands never reach here
     const float m = (t->samples == 0) ? per : std::min(t->sample_best, per);
     t->samples += 1;
     t->sample_best = m;
@@ -266,6 +266,18 @@ orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, 
     CUstream s = (CUstream)stream;
     const Driver &D = drv();
     const double work = (double)(a->row_end - a->row_begin) * (double)a->width;
+    if (a->row_begin == a->row_end && a->width > 0 && a->row_begin >= 0 && a->row_end <= a->height) {
+        // an empty band is not an iteration: nothing is launched, timed or fed to Fig. 9 (a
+        // zero-work sample would be in other units than ns per output element)
+        if (out) {
+            out->iteration = -1;
+            out->level_idx = -1;
+            out->phase = -1;
+            out->final_level_idx = f.final_idx;
+            out->ms = -1.0f;
+        }
+        return ORION_OK;
+    }
     float ms = -1.0f;
     auto report = [&](int lvl, int phase) {
         if (out) {

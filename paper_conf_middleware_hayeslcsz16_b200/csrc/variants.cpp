@@ -340,6 +340,50 @@ orion_status orion_launch(orion_variants *v, int i, const orion_args *a, void *s
     return launch_fn(*v->def, w.fn, w.dyn_bytes, k, (CUstream)stream);
 }
 
+orion_status orion_default_params(const char *kernel_id, float *fparam, int n)
+{
+    if (!kernel_id || !fparam || n < 8) return fail(ORION_E_INVALID, "orion_default_params: bad argument");
+    const KernelDef *def = find_kernel(kernel_id, 0);
+    if (!def) return fail(ORION_E_INVALID, std::string("orion_default_params: unknown kernel ") + kernel_id);
+    for (int i = 0; i < n; ++i) fparam[i] = 0.0f;
+    switch (def->kind) {
+    case K_KNN:      // CUDA-SDK imageDenoising KNN (reading R-O2): Noise = 1/h^2, h = 0.32
+        fparam[0] = (float)(1.0 / (0.32 * 0.32));
+        fparam[1] = 0.2f;          // lerpC
+        fparam[2] = 0.02f;         // weight threshold
+        fparam[3] = 0.79f;         // lerp threshold on cnt / 49
+        break;
+    case K_NLM:      // CUDA-SDK imageDenoising NLM (reading R-O2): h = 1.45
+        fparam[0] = (float)(1.0 / (1.45 * 1.45));
+        fparam[1] = 0.2f;
+        fparam[2] = 0.10f;
+        fparam[3] = 0.10f;
+        break;
+    case K_STENCIL: {  // Rodinia hotspot at the 512-grid cell size for every N (readings R-O3, R-A15)
+        const double cell = 0.016 / 512.0;       // 16 mm chip / 512 cells = 31.25 um
+        const double t_chip = 0.0005, k_si = 100.0, spec_heat_si = 1.75e6, factor_chip = 0.5;
+        const double max_pd = 3.0e6, precision = 0.001, amb = 80.0;
+        const double cap = factor_chip * spec_heat_si * t_chip * cell * cell;
+        const double r_x = cell / (2.0 * k_si * t_chip * cell);
+        const double r_y = cell / (2.0 * k_si * t_chip * cell);
+        const double r_z = t_chip / (k_si * cell * cell);
+        const double step = precision / (max_pd / (factor_chip * t_chip * spec_heat_si));
+        fparam[0] = (float)(step / cap);         // sdc = step / Cap
+        fparam[1] = (float)(1.0 / r_x);          // rx = 1 / Rx
+        fparam[2] = (float)(1.0 / r_y);          // ry = 1 / Ry
+        fparam[3] = (float)(1.0 / r_z);          // rz = 1 / Rz
+        fparam[4] = (float)amb;
+        break;
+    }
+    case K_SRAD:     // Rodinia srad_v2 (reading R-SRAD): lambda = 0.5
+        fparam[0] = 0.5f;
+        break;
+    default:
+        return fail(ORION_E_INVALID, "orion_default_params: kernel without method parameters");
+    }
+    return ORION_OK;
+}
+
 orion_status orion_set_pdl(int on, int *previous)
 {
     if (on != 0 && on != 1) return fail(ORION_E_INVALID, "orion_set_pdl: on must be 0 or 1");

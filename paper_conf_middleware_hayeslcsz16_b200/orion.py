@@ -27,10 +27,6 @@ LIM_REGS, LIM_SMEM, LIM_WARPS, LIM_BLOCKS = 1, 2, 4, 8
 DIR_DECREASING, DIR_INCREASING = -1, 1
 SELECT_FASTEST, SELECT_LOWEST_WITHIN_TOL = 0, 1
 
-# SDK imageDenoising parameters (reading R-O2): Noise = 1/h^2, lerpC, weight
-# threshold, lerp threshold (fraction of the 49 window taps).
-KNN_PARAMS = (1.0 / (0.32 * 0.32), 0.2, 0.02, 0.79)
-NLM_PARAMS = (1.0 / (1.45 * 1.45), 0.2, 0.10, 0.10)
 HALO = {"knn_f4": 3, "knn_f4_p1": 3, "knn_f4_t8": 3, "knn_f4_t16": 3, "nlm_f4": 6, "nlm_f4_g1": 6, "nlm_f4_i": 6, "nlm_f4_q": 6, "nlm_f4_w": 6, "nlm_f4_w8": 6, "nlm_f4_direct": 6, "nlm_f4_regheavy": 6, "hotspot_f32": 1, "hotspot2_f32": 2,
         "hotspot2h_f32": 2, "hotspot4h_f32": 4, "srad_f32": 2, "srad_f32h": 2, "srad_f32_tile": 2}
 # stencil steps one launch advances (temporal blocking); every other kernel: 1
@@ -156,6 +152,7 @@ def lib() -> ctypes.CDLL:
                 "orion_tuner_final": [V, P(I), P(I)],
                 "orion_tuner_tried": [V, P(ctypes.c_float), I],
                 "orion_set_pdl": [I, P(I)],
+                "orion_default_params": [ctypes.c_char_p, P(ctypes.c_float), I],
                 "orion_tuner_replay": [P(TunerCfg), P(Level), I, I, P(ctypes.c_float), I, P(I), P(I), P(I)],
                 "orion_generate_rgba": [I, V, I, I, I, I, ctypes.c_uint, ctypes.c_float, V],
                 "orion_generate_thermal": [I, V, V, I, I, ctypes.c_uint, V],
@@ -246,30 +243,27 @@ def denoise_args(kernel_id: str, src: int, dst: int, width: int, height: int, ro
     row_end = height if row_end is None else row_end
     src_row_end = height if src_row_end is None else src_row_end
     dst_row_begin = row_begin if dst_row_begin is None else dst_row_begin
-    p = params or (KNN_PARAMS if kernel_id.startswith("knn") else NLM_PARAMS)
+    p = params or default_params(kernel_id)[:4]
     a = Args(src, dst, None, width, height, row_begin, row_end, src_row_begin, src_row_end, dst_row_begin)
     for i, x in enumerate(p):
         a.fparam[i] = x
     return a
 
 
-def hotspot_constants(cell: float = 0.016 / 512) -> tuple:
-    """Rodinia hotspot coefficients at a fixed cell size (reading R-A15):
-    (sdc = step/Cap, rx = 1/Rx, ry = 1/Ry, rz = 1/Rz, amb)."""
-    t_chip, k_si, spec_heat, factor_chip, max_pd, precision = 0.0005, 100.0, 1.75e6, 0.5, 3.0e6, 0.001
-    cap = factor_chip * spec_heat * t_chip * cell * cell
-    r_x = cell / (2.0 * k_si * t_chip * cell)
-    r_y = cell / (2.0 * k_si * t_chip * cell)
-    r_z = t_chip / (k_si * cell * cell)
-    step = precision / (max_pd / (factor_chip * t_chip * spec_heat))
-    return (step / cap, 1.0 / r_x, 1.0 / r_y, 1.0 / r_z, 80.0)
+def default_params(kernel_id: str) -> tuple:
+    """orion_default_params: the kernel family's method parameters (fparam[0..8)) as liborion
+    defines them -- SDK imageDenoising (Noise, lerpC, wthr, lthr), Rodinia hotspot (sdc, rx, ry,
+    rz, amb) or SRAD (lambda)."""
+    buf = (ctypes.c_float * 8)()
+    _check(lib().orion_default_params(kernel_id.encode(), buf, 8), "orion_default_params")
+    return tuple(buf)
 
 
 def hotspot_args(t_in: int, t_out: int, power: int, width: int, height: int, row_begin: int = 0,
                  row_end: int | None = None, consts=None) -> Args:
     row_end = height if row_end is None else row_end
     a = Args(t_in, t_out, power, width, height, row_begin, row_end, 0, height, 0)
-    for i, x in enumerate(consts or hotspot_constants()):
+    for i, x in enumerate(consts or default_params("hotspot_f32")[:5]):
         a.fparam[i] = x
     return a
 
@@ -532,10 +526,11 @@ def generate_thermal(device: int, t0: int, power: int, width: int, height: int, 
                                         _s(stream)), "orion_generate_thermal")
 
 
-def srad_args(j_in: int, j_out: int, q0: int, width: int, height: int, lam: float = 0.5) -> Args:
-    """Arguments of one "srad_f32" iteration; q0 = device address of the float q0sqr."""
+def srad_args(j_in: int, j_out: int, q0: int, width: int, height: int, lam: float | None = None) -> Args:
+    """Arguments of one "srad_f32" iteration; q0 = device address of the float q0sqr; lam
+    None = liborion's default (orion_default_params)."""
     a = Args(j_in, j_out, q0, width, height, 0, height, 0, height, 0)
-    a.fparam[0] = lam
+    a.fparam[0] = default_params("srad_f32h")[0] if lam is None else lam
     return a
 
 

@@ -153,3 +153,25 @@ def test_device_entry_points_fail_cleanly_without_gpu():
     with pytest.raises(O.OrionError) as e:
         O.query_limits(0)
     assert e.value.status == -5
+
+
+def test_default_params_match_the_oracles_constants():
+    # liborion's method parameters (orion_default_params, C++) and the oracle's (Python) are
+    # written independently; they must agree to fp32 (the kernels' parameter precision)
+    import numpy as np
+    import oracle
+    f32 = np.float32
+    for k in ("knn_f4", "knn_f4_t16"):
+        p = O.default_params(k)
+        assert p[:4] == (f32(oracle.KNN["noise"]), f32(oracle.KNN["lerpc"]), f32(oracle.KNN["wthr"]),
+                         f32(oracle.KNN["lthr"]))
+    for k in ("nlm_f4_w", "nlm_f4_regheavy"):
+        p = O.default_params(k)
+        assert p[:4] == (f32(oracle.NLM["noise"]), f32(oracle.NLM["lerpc"]), f32(oracle.NLM["wthr"]),
+                         f32(oracle.NLM["lthr"]))
+    c = oracle.hotspot_constants()
+    for k in ("hotspot_f32", "hotspot4h_f32"):
+        assert O.default_params(k)[:5] == tuple(f32(c[n]) for n in ("sdc", "rx", "ry", "rz", "amb"))
+    assert O.default_params("srad_f32h")[0] == 0.5
+    with pytest.raises(O.OrionError):
+        O.default_params("no_such_kernel")
