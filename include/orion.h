@@ -86,10 +86,15 @@ enum { ORION_REALISE_MAX_SMEM = 0, ORION_REALISE_MIN_CARVEOUT = 1 };
 
 /* ---- occupancy levels (question 1; host-only, pure) -------------------------------------- */
 
-/* Nominal B200 (cc 10.0, 148 SMs) limits, for planning without a GPU. */
+/* Nominal B200 (cc 10.0, 148 SMs) limits -- the Eq. (1) inputs (P:L121-P:L127: registers,
+ * shared memory and thread slots per SM) for planning without a GPU; the B200 figures are
+ * BASELINE.json's north star (64K regs, 228 KB, 64 warps, 148 SMs), the granularities those of
+ * the calculator the paper uses ([19]). */
 orion_status orion_b200_limits(orion_device_limits *out);
 
-/* Limits of CUDA device `device`, read from the driver (cuDeviceGetAttribute). */
+/* Limits of CUDA device `device` read from the driver (cuDeviceGetAttribute): the same Eq. (1)
+ * inputs (P:L121-P:L127) as orion_b200_limits, measured instead of assumed.  ORION_E_CUDA
+ * without a driver / device. */
 orion_status orion_query_limits(int device, orion_device_limits *out);
 
 /* Eq. (1) evaluated with the calculator's granularities (P:L125-P:L127): CTAs/SM of a
@@ -107,36 +112,45 @@ orion_status orion_ctas_per_sm(const orion_device_limits *dev, int block_threads
  * -> ORION_E_CAPACITY with *n_out = the number needed.  `out` may be NULL if capacity = 0. */
 orion_status orion_levels(const orion_device_limits *dev, const orion_kernel_resources *res,
                           orion_level *out, int capacity, int *n_out);
-/* orion_levels with an explicit realisation mode (ORION_REALISE_*); orion_levels = MAX_SMEM.
- * Same k_max and register caps in both modes; padding and carveout differ. */
+/* orion_levels with an explicit realisation mode (ORION_REALISE_*; the small- vs large-cache
+ * axis of P:L757-P:L761, Table 3); orion_levels = MAX_SMEM.  Same k_max and register caps in
+ * both modes; padding and carveout differ. */
 orion_status orion_levels_ex(const orion_device_limits *dev, const orion_kernel_resources *res, int mode,
                              orion_level *out, int capacity, int *n_out);
-/* orion_ctas_per_sm under a carveout preference of `carveout_pct` percent of the maximum
- * shared memory (< 0: the default, treated as the maximum), rounded up to a configuration
- * and raised to fit one CTA, as the driver does. */
+/* orion_ctas_per_sm (Eq. (1) with granularities, P:L125-P:L127) under a carveout preference of
+ * `carveout_pct` percent of the maximum shared memory (< 0: the default, treated as the
+ * maximum), rounded up to a configuration and raised to fit one CTA, as the driver does
+ * (reading R-CARVE). */
 orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int block_threads, int regs,
                                         int smem_static, int smem_dyn, int carveout_pct, int *ctas,
                                         int *limiter);
 
 /* ---- code generation (question 1; host-only, no GPU needed) ------------------------------ */
 
-/* Kernel ids: "knn_f4" (T = 128 / 256 / 64), "knn_f4_p1" (one pixel per thread), "knn_f4_t8" / "knn_f4_t16" (the
- * 49 taps of a pixel split over 8 / 16 lanes), "nlm_f4" (box sums, 3 offset pairs per pass), "nlm_f4_w" (same,
- * 128-column tiles), "nlm_f4_q" (float4 tile plane, 2 pairs per pass),
- * "nlm_f4_i" (same, exact fixed-point integer windows), "nlm_f4_w8" (same tile, 256 threads),
- * "nlm_f4_g1" (1 pair per pass), "nlm_f4_direct", "nlm_f4_regheavy" (T = 128 / 64),
- * "hotspot_f32" (T = 256 / 128), "hotspot2_f32" (two stencil steps per launch, edge lanes fetch
- * the outer columns; width % 4 == 0), "hotspot2h_f32" (two steps per launch, whole halo lanes:
- * 120 output columns per warp; width % 4 == 0), "hotspot4h_f32" (four steps per launch, the same
- * halo-lane warps as a 4-stage register pipeline; width % 4 == 0; the C3 default),
- * "srad_f32" (register-sliding, any width), "srad_f32h" (same with whole halo lanes; width % 4 == 0),
- * "srad_f32_tile" (shared-memory form, same bits).
- * block_threads = 0 selects the kernel's default CTA size.  Fills the natural resources
- * (compiles the kernel's PTX once, uncapped, with the embedded ptxas). */
+/* The kernel's natural resources -- Vreg, Vsmem of Eq. (1) (P:L121-P:L127) and MAXLIVE's proxy
+ * for Fig. 8 (reading R-A5) -- from compiling its PTX once, uncapped, with the embedded
+ * ptxas (the "original" build).  Kernel ids (the paper's benchmarks, Table 2 P:L725-
+ * P:L739; their math per readings R-O2, R-O3, R-SRAD):
+ *   imageDenoising KNN: "knn_f4" (T = 128 / 256 / 64), "knn_f4_p1" (one pixel per
+ *       thread, same bits), "knn_f4_t16" (the 49 taps of a pixel over 16 lanes; the C1 default);
+ *   imageDenoising NLM: "nlm_f4_w" (box sums + symmetric pairs, 3 pairs per pass,
+ *       128-column tiles; the C2 / C5 default), "nlm_f4" (same, 122-column tiles),
+ *       "nlm_f4_direct" (the direct 2401-term definition, cross-check form), "nlm_f4_regheavy"
+ *       (direct form, centre patch in registers: the register-heavy C4 kernel; T = 128 / 64);
+ *   hotspot: "hotspot_f32" (one step per launch; T = 256 / 128), "hotspot2h_f32" (two
+ *       steps per launch, whole halo lanes), "hotspot4h_f32" (four steps per launch as a 4-stage
+ *       register pipeline; the C3 default) -- width % 4 == 0 for the multi-step forms;
+ *   srad: "srad_f32h" (float4 strips, whole halo lanes, width % 4 == 0; the default),
+ *       "srad_f32" (register-sliding, any width), "srad_f32_tile" (shared-memory form; both
+ *       cross-check forms, same bits).
+ * block_threads = 0 selects the kernel's default CTA size.  ORION_E_INVALID for an unknown id /
+ * CTA size, ORION_E_COMPILE when ptxas fails.  Host-only. */
 orion_status orion_kernel_probe(const char *kernel_id, int block_threads, orion_kernel_resources *out);
 
 /* Compile the kernel at register cap `reg_cap` (0 = uncapped) and report what ptxas did:
- * registers used, spill store / load bytes, local (stack) bytes per thread. */
+ * registers used, spill store / load bytes, local (stack) bytes per thread -- the spill cost a
+ * register-capped level pays ("avoid excessive spilling"; C4's trade-off).  Memoised per
+ * (kernel, T, cap).  Host-only; ORION_E_COMPILE with the ptxas log in orion_last_error(). */
 orion_status orion_compile_info(const char *kernel_id, int block_threads, int reg_cap, int *regs,
                                 int *spill_store_bytes, int *spill_load_bytes, int *local_bytes);
 
@@ -158,13 +172,18 @@ typedef struct orion_variants orion_variants;   /* opaque, library-owned */
  * and times each level once more before its timed rounds. */
 orion_status orion_build_variants(int device, const char *kernel_id, int block_threads,
                                   const orion_level *levels, int n, orion_variants **out);
+/* Number of variants (= levels) of the multi-version binary. */
 orion_status orion_variants_count(const orion_variants *v, int *n);
-/* The realised level (pad recomputed from actual registers) of variant `level_idx`. */
+/* The realised level (pad recomputed from actual registers, P:L649) of variant `level_idx`. */
 orion_status orion_variant_level(const orion_variants *v, int level_idx, orion_level *out);
-/* verified_ctas_per_sm = the residency MEASURED by the probe launch (equal to the level's k). */
+/* What ptxas and the hardware did with variant `level_idx` (P:L215, P:L227-P:L229 realising a
+ * level): registers, spill store / load bytes and local bytes per thread, and
+ * verified_ctas_per_sm = the residency MEASURED by the probe launch (equal to the level's k).
+ * Any output pointer may be NULL.  ORION_E_INVALID for a bad index. */
 orion_status orion_variant_info(const orion_variants *v, int level_idx, int *regs, int *spill_store_bytes,
                                 int *spill_load_bytes, int *local_bytes, int *verified_ctas_per_sm);
-/* The kernel's natural resources (what orion_kernel_probe returned when building). */
+/* The kernel's natural resources (what orion_kernel_probe returned when building; Eq. (1)'s
+ * Vreg / Vsmem, P:L121-P:L127). */
 orion_status orion_variants_resources(const orion_variants *v, orion_kernel_resources *out);
 void orion_variants_destroy(orion_variants *v);
 
@@ -217,7 +236,8 @@ orion_status orion_launch(orion_variants *v, int level_idx, const orion_args *a,
  * ORION_E_INVALID for an unknown id or n < 8.  Host-only. */
 orion_status orion_default_params(const char *kernel_id, float *fparam, int n);
 
-/* Process-wide switch of programmatic dependent launch for every later launch (initially
+/* Launch plumbing of the P:L653 loop (not a method step): process-wide switch of
+ * programmatic dependent launch for every later launch (initially
  * from ORION_PDL; default on).  `on` is 0 or 1 (else ORION_E_INVALID); *previous (may be
  * NULL) receives the setting it replaces.  A loop that will be replayed as a CUDA graph (graph
  * nodes are plain launches) turns it off so that the sweep times the levels the same way. */
@@ -253,6 +273,9 @@ typedef struct {
                                      launch runs back to back with its neighbours                   */
 } orion_tuner_cfg;
 
+/* The defaults: the paper's constants (MAXLIVE threshold 32; slowdown 0.02, P:L615;
+ * worse_eps 0 and one sample per level) plus the readings' defaults (FASTEST, R-A4;
+ * direction switch on, R-A12; synchronous timing). */
 orion_status orion_tuner_default_cfg(orion_tuner_cfg *cfg);
 
 typedef struct orion_tuner orion_tuner;   /* opaque, library-owned (holds CUDA events) */
@@ -260,7 +283,8 @@ typedef struct orion_tuner orion_tuner;   /* opaque, library-owned (holds CUDA e
 /* Fig. 8 (P:L589-P:L603) applied to the variants' levels: direction from MAXLIVE (the
  * natural register count), ladder = original + conservative..max (increasing) or
  * original, original-1, .. 1 by padding (decreasing), with the opposite direction kept
- * as the fail-safe. */
+ * as the fail-safe.  The tuner holds two CUDA events; ORION_E_INVALID for a bad cfg or
+ * levels without the original (uncapped) version. */
 orion_status orion_tuner_create(orion_variants *v, const orion_tuner_cfg *cfg, orion_tuner **out);
 
 typedef struct {
@@ -283,7 +307,8 @@ orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, 
 /* The measured time of an exploring iteration is work-normalised (ns per output element,
  * P:L975) before Fig. 9 compares it, so iterations of different sizes compare fairly. */
 
-/* n consecutive iterations, exactly n calls of orion_tune_step on args[0..n-1] (host array of n
+/* n consecutive Fig. 9 iterations (P:L605-P:L643), exactly n calls of orion_tune_step on
+ * args[0..n-1] (host array of n
  * orion_args, caller-owned), issued from the library in one call: launch-bound frames (C1) do not
  * pay a foreign-function call per iteration.  *last (may be NULL) = the report of the last
  * iteration.  Errors: ORION_E_INVALID for NULL / n < 0; otherwise the first failing
@@ -299,7 +324,7 @@ orion_status orion_tune_steps(orion_tuner *t, const orion_args *args, int n, voi
 orion_status orion_tune_split(orion_tuner *t, const orion_args *a, int bands, void *stream,
                               orion_step_report *reports);
 
-/* Same iteration end to end from HOST buffers: copies a->src (host, pinned for async)
+/* Same iteration (Fig. 9, P:L605-P:L643) end to end from HOST buffers: copies a->src (host, pinned for async)
  * into dev_src, runs orion_tune_step with device pointers, copies dev_dst back into
  * a->dst (host) -- all on `stream`, then synchronises it.  dev_src / dev_dst are
  * caller-owned device buffers at least as large as the host regions (and dev_aux for the
@@ -311,7 +336,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
 /* A whole iterative stencil run end to end from HOST buffers -- the Rodinia driver shape
  * (copy the grid in, iterate, copy it out), the iterations being the ones
  * Fig. 9 tunes across (P:L651-P:L653).  Kernels of kind hotspot ("hotspot_f32",
- * "hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32") and srad ("srad_f32", "srad_f32h", "srad_f32_tile") only, whole grids only
+ * "hotspot2h_f32", "hotspot4h_f32") and srad ("srad_f32", "srad_f32h", "srad_f32_tile") only, whole grids only
  * (a->row_begin = a->src_row_begin = a->dst_row_begin = 0, a->row_end = a->src_row_end =
  * a->height).
  *   a->src  host initial grid (fp32, width x height, row-major; pinned for async copies)
@@ -320,7 +345,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
  *   dev_a, dev_b  caller-owned device grids (ping-pong), width x height fp32 each
  *   dev_aux hotspot: device power map buffer (filled here); srad: the device float q0sqr
  *   roi     srad only: {r1, r2, c1, c2} of the ROI statistics run before every iteration
- * Copies in, runs `iterations` orion_tune_step iterations on `stream` (hotspot2_f32 / hotspot2h_f32 advance
+ * Copies in, runs `iterations` orion_tune_step iterations on `stream` (hotspot2h_f32 advances
  * two time steps per iteration, hotspot4h_f32 four), copies the final grid out and synchronises the stream.
  * Bytes copied are returned in *h2d_bytes / *d2h_bytes.  ORION_E_INVALID on other kernels,
  * partial row ranges or missing buffers. */
@@ -328,7 +353,8 @@ orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterat
                                  void *dev_aux, const int *roi, void *stream, long long *h2d_bytes,
                                  long long *d2h_bytes);
 
-/* Pipelined end-to-end iterations from HOST buffers.  The pipe owns `depth` slots of device
+/* Pipelined end-to-end iterations from HOST buffers (the P:L653 tuned loop fed from the host:
+ * what an application streaming frames sees; bench.py's e2e figure).  The pipe owns `depth` slots of device
  * staging buffers (width x max_rows elements each for src, dst and -- stencil -- aux;
  * allocated here, never in submit) and three non-blocking streams: the H2D copy of frame n,
  * the kernel of frame n-1 (orion_tune_step on the pipe's compute stream) and the D2H copy of
@@ -336,18 +362,26 @@ orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterat
  * stay untouched until orion_host_pipe_drain returns.  Errors: ORION_E_INVALID when a frame
  * does not fit the pipe's width / max_rows; driver errors as ORION_E_CUDA. */
 typedef struct orion_host_pipe orion_host_pipe;   /* opaque, library-owned */
+/* Create a pipe over tuner t (its Fig. 9 walk, P:L605-P:L643, runs inside submit); depth 1..8. */
 orion_status orion_host_pipe_create(orion_tuner *t, int width, int max_rows, int depth, orion_host_pipe **out);
-/* Enqueue one iteration: a->src / a->aux / a->dst are HOST pointers laid out as for
+/* Enqueue one tuned iteration (orion_tune_step, Fig. 9 P:L605-P:L643): a->src / a->aux /
+ * a->dst are HOST pointers laid out as for
  * orion_launch (src rows [src_row_begin, src_row_end), dst rows from dst_row_begin).
  * Returns without waiting; bytes copied are reported in *h2d_bytes / *d2h_bytes. */
 orion_status orion_host_pipe_submit(orion_host_pipe *p, const orion_args *a, orion_step_report *out,
                                     long long *h2d_bytes, long long *d2h_bytes);
-/* Wait until every submitted iteration's output is in host memory. */
+/* Wait until every submitted iteration's output is in host memory (end of the P:L653 loop). */
 orion_status orion_host_pipe_drain(orion_host_pipe *p);
+/* Synchronise the pipe's streams and free its staging buffers, events and streams (SURVEY §8(b)
+ * ownership: library-owned objects have a create / destroy pair). */
 void orion_host_pipe_destroy(orion_host_pipe *p);
 
-/* Current ladder: *direction, ladder level indices (ladder[0] = original) -> out[]. */
+/* Current Fig. 8 candidate ladder (P:L589-P:L603): *direction (ORION_DIR_*), ladder level
+ * indices (ladder[0] = the original) -> out[capacity]; capacity protocol as
+ * orion_levels.  After a P:L689 direction switch it is the opposite ladder. */
 orion_status orion_tuner_ladder(const orion_tuner *t, int *direction, int *out, int capacity, int *n_out);
+/* The final kernel of Fig. 9 ("set final kernel"): its level index (-1 while exploring)
+ * and the iteration it was set at. */
 orion_status orion_tuner_final(const orion_tuner *t, int *final_level_idx, int *iterations_to_final);
 /* The runtime table Fig. 9 has seen so far (P:L605-P:L643; work-normalised per P:L975):
  * out[i] = the value observed for level i -- ns per output element, the fastest of its
@@ -388,10 +422,15 @@ orion_status orion_tuner_replay(const orion_tuner_cfg *cfg, const orion_level *l
 
 /* ---- synthetic inputs on the device (the generator's GPU twin; no method arithmetic) ---- */
 
-/* Rows [row_begin, row_end) of the W x H seeded noisy RGBA image into dst (pitch W). */
+/* Rows [row_begin, row_end) of the W x H seeded noisy RGBA image into dst (pitch W): the device
+ * twin of synth.noisy_rgba (SURVEY §8(d) generator; DESIGN §5 input recipe -- the paper
+ * publishes no inputs, P:L85-P:L91), bit-identical to it, so a row slab of a sharded frame (C5)
+ * is the same bits as those rows of the full image.  seed < 2^24. */
 orion_status orion_generate_rgba(int device, void *dst, int width, int height, int row_begin, int row_end,
                                  unsigned seed, float sigma, void *stream);
-/* Thermal T0 and power map (W x H) into t0 / power. */
+/* Thermal T0 and power map (W x H) into t0 / power: the device twin of synth.thermal_inputs
+ * (T0 = 323.15 + U[0,1) * 20, P = U[0,1) * 0.05; Rodinia hotspot's
+ * inputs are unpublished).  Also SRAD's positive image. */
 orion_status orion_generate_thermal(int device, void *t0, void *power, int width, int height, unsigned seed,
                                     void *stream);
 /* SRAD's per-iteration ROI statistics (Rodinia srad_v2, reading R-SRAD; Table 2
@@ -401,14 +440,19 @@ orion_status orion_generate_thermal(int device, void *t0, void *power, int width
  * (whose fparam[0] = lambda).  Asynchronous on `stream`. */
 orion_status orion_srad_roi_stats(int device, const void *J, int width, int height, int r1, int r2, int c1, int c2,
                                   void *q0, void *stream);
-/* Write `bytes` of `buf` (a device scratch buffer larger than L2) to evict the L2. */
+/* Write `bytes` of `buf` (a device scratch buffer larger than L2) to evict the L2: a
+ * measurement utility (cold-cache timing, SURVEY §8(d) timing protocol); no method math. */
 orion_status orion_flush_l2(int device, void *buf, long long bytes, void *stream);
 
-/* ---- diagnostics -------------------------------------------------------------------------- */
+/* ---- diagnostics (SURVEY §5 failure detection; not method steps) ---------------------------- */
+/* Name of a status code ("ORION_OK", "ORION_E_INVALID", ...). */
 const char *orion_status_str(orion_status s);
+/* The calling thread's last error message (driver string, ptxas log, argument check). */
 const char *orion_last_error(void);
-/* Number of kernel launches liborion has enqueued in this process (all kernels). */
+/* Number of kernel launches liborion has enqueued in this process (all kernels; graph replays
+ * count their captured launches): the evidence bench.py reports as gpu_launches. */
 long long orion_launch_count(void);
+/* Library name and version string. */
 const char *orion_version(void);
 
 #ifdef __cplusplus

@@ -122,219 +122,23 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot_f32_256(orion_ka
 // T = 128 threads (32 x 4 warps): 128 columns x 4 strips of 16 rows per CTA.
 extern "C" __global__ void __launch_bounds__(128) orion_hotspot_f32_128(orion_kargs a) { ORION_PROBE(a); hotspot_body<4, 16>(a); }
 
-// ---- two explicit steps per launch (temporal blocking) -------------------------------------
-// T2 = step(step(T0)) with the intermediate T1 kept in registers: per 2 cell-steps the kernel
-// reads T0 and P once and writes T2 once (12 B instead of 24 B of DRAM traffic).  Each warp
-// walks a strip of rows computing T1 one row ahead of T2; E / W neighbours come by shuffle,
-// and lanes 0 / 31 also compute the T1 cell just outside the warp's 128 columns (the halo
-// the outer T2 cells need), from predicated scalar loads.  Every cell value is produced by
-// the same hs_cell() as the one-step kernel, with the same clamp-to-edge neighbours, so two
-// one-step launches and one two-step launch give identical bits.  Rows must be 16-byte
-// aligned (width % 4 == 0; the launcher rejects other widths for this kernel).
-struct Row4 {
-    float4 v;      // own columns cx .. cx+3
-    float x;       // the edge lane's outer column: xx (lane 0: base-1, lane 31: base+128, clamped)
-    float xo;      // one further out: lane 0: base-2 (1 at the west edge), lane 31: base+129 (clamped)
-};
-
-// The rows a warp walks are streamed through a ring in shared memory: fetched NB-1 rows
-// ahead with cp.async (LDGSTS: global -> shared without registers), so the bytes in flight
-// per SM do not depend on the register budget of the occupancy level.  Each lane copies its
-// own 16 bytes of the T0 and P rows (the edge lanes also their outer columns) into its warp's
-// ring slot and later reads back exactly what it copied, so no warp barrier is needed.  Six
-// slots and a six-row loop body: every slot offset in the body is a compile-time constant.
-namespace {
-#ifndef H2_NB_SLOTS
-#define H2_NB_SLOTS 6
-#endif
+// ---- temporal blocking: rows streamed through a shared-memory ring ------------------------
+// A warp's T0 / P rows are fetched ahead with cp.async (LDGSTS: global -> shared without
+// registers), so the bytes in flight per SM do not depend on the register budget of the
+// occupancy level.  Each lane copies its own 16 bytes of a row into its warp's ring slot and
+// later reads back exactly what it copied: no warp barrier is needed.
 #ifndef H2_ROWS
 #define H2_ROWS 32
 #endif
-constexpr int H2_NB = H2_NB_SLOTS;          // ring slots per warp (NB-1 rows in flight); multiple of 6
-static_assert(H2_NB % 6 == 0, "the loop body rotates rows through 6 register sets");
-constexpr int H2_SLOT = 136 + 136;          // floats: T0 segment [base-4, base+132), P segment
-}  // namespace
 
 __device__ __forceinline__ void cp_async16(float *sdst, const float *gsrc)
 {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
                  "l"(gsrc) : "memory");
 }
-__device__ __forceinline__ void cp_async4(float *sdst, const float *gsrc)
-{
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
-                 "l"(gsrc) : "memory");
-}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
-
-// Edge handling without per-row selects on the block position: the edge lanes' outer columns
-// are clamped in global coordinates, and at the west edge lane 0's outer T1 cell is made to be
-// T1(column 0) itself -- outer column xx = 0 with neighbours {T(0), T(1)} (xo = 1): the update
-// only uses E + W, one commutative IEEE addition, so the cell is bit-identical to the main
-// cell of column 0, and T2's west neighbour of column 0 (clamp-to-edge: column 0) is lane 0's
-// outer cell like everywhere else.  At the east edge the lane holding column W-1 takes its own
-// value as E (eclamp); lanes past the edge write nothing and feed no written cell.
-template <int RY, bool BOTTOM>
-__device__ __forceinline__ void hotspot2_strip(const orion_kargs &a, int ys, int ye)
-{
-    extern __shared__ float4 smem4[];
-    const int W = a.width, H = a.height;
-    const int lane = threadIdx.x;
-    const float c[5] = {a.fparam[0], a.fparam[1], a.fparam[2], a.fparam[3], a.fparam[4]};
-    const int base = blockIdx.x * 128;
-    const int cx = base + lane * 4;
-    const int cxl = min(cx, W - 4);
-    const bool lane0 = lane == 0, lane31 = lane == 31, edge = lane0 || lane31;
-    const bool eclamp = cx + 4 >= W;
-    const int xx = lane0 ? (base == 0 ? 0 : base - 1) : min(base + 128, W - 1);
-    const int xo = lane0 ? (base == 0 ? min(1, W - 1) : base - 2) : min(base + 129, W - 1);
-    const float *t0 = (const float *)a.src - (size_t)a.src_row_begin * (size_t)W;
-    const float *p0 = (const float *)a.aux - (size_t)a.src_row_begin * (size_t)W;
-    float *ring = reinterpret_cast<float *>(smem4) + threadIdx.y * (H2_NB * H2_SLOT);
-    // slot offsets: own float4 at 4 + 4*lane; lane 0's outer columns at 3 (xx) and 2 (xo);
-    // lane 31's at 132 (xx) and 133 (xo); the P segment follows at +136.  The other lanes read
-    // their "outer" words (unused) from their own float4, so every lane reads back only words
-    // it copied itself.
-    const int own = 4 + 4 * lane;
-    const int oxx = lane0 ? 3 : (lane31 ? 132 : own), oxo = lane0 ? 2 : (lane31 ? 133 : own + 1);
-    const int dxx = xx - cxl, dxo = xo - cxl;
-
-    auto load = [&](const float *row) {
-        Row4 r;
-        r.v = __ldg(reinterpret_cast<const float4 *>(row + cxl));
-        r.x = __ldg(row + xx);
-        r.xo = __ldg(row + xo);
-        return r;
-    };
-    auto step = [&](const Row4 &N, const Row4 &T, const Row4 &S, float4 P, float Pe) {
-        float Wv = __shfl_up_sync(0xffffffffu, T.v.w, 1);
-        float Ev = __shfl_down_sync(0xffffffffu, T.v.x, 1);
-        if (lane0) Wv = T.x;
-        if (lane31) Ev = T.x;
-        if (eclamp) Ev = T.v.w;
-        Row4 out;
-        out.v = hs_cell4(T.v, N.v, S.v, Ev, Wv, P, c);
-        out.x = hs_cell(T.x, N.x, S.x, lane0 ? T.v.x : T.xo, lane0 ? T.xo : T.v.w, Pe, c);
-        out.xo = 0.0f;
-        return out;
-    };
-    auto rowp = [&](const float *b, int y) { return b + (size_t)clampi(y, 0, H - 1) * (size_t)W; };
-    // issue() is called for q = 0, 1, 2, ... in order; slot q % NB holds T0(clamp(ys+2+q)) and
-    // P(ys+1+q) (P rows never pass H-1: q < nq).  Rows advance by pointer increments; only the
-    // bottom strip clamps.
-    const float *tn = rowp(t0, ys + 2) + cxl, *pn = rowp(p0, ys + 1) + cxl;
-    int rt = ys + 2;                               // unclamped row of tn
-    auto issue = [&](float *sl) {
-        cp_async16(sl + own, tn);
-        cp_async16(sl + 136 + own, pn);
-        if (edge) {
-            cp_async4(sl + oxx, tn + dxx);
-            cp_async4(sl + oxo, tn + dxo);
-            cp_async4(sl + 136 + oxx, pn + dxx);
-        }
-        if (!BOTTOM || rt < H - 1) tn += W;
-        pn += W;
-        ++rt;
-    };
-
-    const int yb = min(ye, H - 1);                 // rows whose south T1 row is distinct
-    const int nq = yb - ys;                        // loop iterations
-#pragma unroll
-    for (int q = 0; q < H2_NB - 1; ++q) {
-        if (q < nq) issue(ring + q * H2_SLOT);
-        cp_async_commit();
-    }
-    // prologue: T1 of rows clamp(ys-1) (ua) and ys (ub)
-    const bool top = ys == 0;
-    Row4 tm2 = load(rowp(t0, ys - 2)), tm1 = load(rowp(t0, ys - 1));
-    Row4 tc0 = load(rowp(t0, ys)), tc1 = load(rowp(t0, ys + 1));
-    const float *pa_row = rowp(p0, ys - 1), *pc_row = rowp(p0, ys);
-    const float4 Pa = __ldg(reinterpret_cast<const float4 *>(pa_row + cxl));
-    const float4 Pc = __ldg(reinterpret_cast<const float4 *>(pc_row + cxl));
-    const float Pea = __ldg(pa_row + xx), Pec = __ldg(pc_row + xx);
-    Row4 ua = top ? step(tc0, tc0, tc1, Pc, Pec) : step(tm2, tm1, tc0, Pa, Pea);
-    Row4 ub = step(tm1, tc0, tc1, Pc, Pec);
-    float *orow = (float *)a.dst + (size_t)cx + ((size_t)ys - (size_t)a.dst_row_begin) * (size_t)W;
-    const bool writer = cx < W;
-    // one output row y = ys + q: T0 rows y, y+1 (A, B) and y+2 (C, from the ring), T1 rows
-    // clamp(y-1), y (X, Y) and y+1 (Z, computed), P rows y (Pcur) and y+1 (Pnext, from the ring).
-    // T0 and T1 rows rotate through three variables and P rows through two, so six consecutive
-    // rows are written out with permuted arguments -- no register moves between rows.
-    struct PRow {
-        float4 v;
-        float e;
-    };
-    PRow pa{Pc, Pec}, pb;
-    Row4 tcx;
-    auto row = [&](int q, float *sl_read, float *sl_issue, const Row4 &A, const Row4 &B, Row4 &C, const Row4 &X,
-                   const Row4 &Y, Row4 &Z, const PRow &Pcur, PRow &Pnext) {
-        if (q + H2_NB - 1 < nq) issue(sl_issue);
-        cp_async_commit();
-        cp_async_wait<H2_NB - 1>();                // slot q has landed (this lane's copies)
-        C.v = *reinterpret_cast<const float4 *>(sl_read + own);
-        Pnext.v = *reinterpret_cast<const float4 *>(sl_read + 136 + own);
-        C.x = sl_read[oxx];                        // meaningful on the edge lanes only (no branch)
-        C.xo = sl_read[oxo];
-        Pnext.e = sl_read[136 + oxx];
-        Z = step(A, B, C, Pnext.v, Pnext.e);       // T1(y+1)
-        const Row4 o = step(X, Y, Z, Pcur.v, Pcur.e);   // T2(y)
-        if (writer) *reinterpret_cast<float4 *>(orow) = o.v;
-        orow += W;
-    };
-    Row4 uz;
-    int q = 0;
-#define H2_S(k) (ring + (k) * H2_SLOT)
-#define H2_I(k) H2_S(((k) + H2_NB - 1) % H2_NB)
-#pragma unroll 1
-    for (; q + H2_NB <= nq; q += H2_NB) {          // slot of row q + k is k (q % NB == 0)
-#pragma unroll
-        for (int g = 0; g < H2_NB; g += 6) {
-            row(q + g, H2_S(g), H2_I(g), tc0, tc1, tcx, ua, ub, uz, pa, pb);
-            row(q + g + 1, H2_S(g + 1), H2_I(g + 1), tc1, tcx, tc0, ub, uz, ua, pb, pa);
-            row(q + g + 2, H2_S(g + 2), H2_I(g + 2), tcx, tc0, tc1, uz, ua, ub, pa, pb);
-            row(q + g + 3, H2_S(g + 3), H2_I(g + 3), tc0, tc1, tcx, ua, ub, uz, pb, pa);
-            row(q + g + 4, H2_S(g + 4), H2_I(g + 4), tc1, tcx, tc0, ub, uz, ua, pa, pb);
-            row(q + g + 5, H2_S(g + 5), H2_I(g + 5), tcx, tc0, tc1, uz, ua, ub, pb, pa);
-        }
-    }
-#undef H2_I
-#pragma unroll 1
-    for (; q < nq; ++q) {                          // the last < 6 rows
-        row(q, H2_S(q % H2_NB), H2_S((q + H2_NB - 1) % H2_NB), tc0, tc1, tcx, ua, ub, uz, pa, pb);
-        tc0 = tc1;
-        tc1 = tcx;
-        ua = ub;
-        ub = uz;
-        pa = pb;
-    }
-#undef H2_S
-    cp_async_wait<0>();
-    if (ye == H) {                                 // bottom image row: its south T1 row is itself
-        const Row4 o = step(ua, ub, ub, pa.v, pa.e);
-        if (writer) *reinterpret_cast<float4 *>(orow) = o.v;
-    }
-}
-
-template <int BY, int RY>
-__device__ __forceinline__ void hotspot2_body(const orion_kargs &a)
-{
-    const int ys = a.row_begin + (blockIdx.y * BY + threadIdx.y) * RY;
-    if (ys >= a.row_end) return;
-    const int ye = min(ys + RY, a.row_end);
-    if (ye + 1 < a.height)                         // every T0 row the strip streams is < H-1 + 1
-        hotspot2_strip<RY, false>(a, ys, ye);
-    else
-        hotspot2_strip<RY, true>(a, ys, ye);
-}
-
-// T = 256 threads (32 x 8 warps): 128 columns x 8 strips of 16 rows per CTA; 2 steps per launch.
-extern "C" __global__ void __launch_bounds__(256) orion_hotspot2_f32_256(orion_kargs a)
-{
-    ORION_PROBE(a);
-    hotspot2_body<8, H2_ROWS>(a);
-}
 
 // ---- two steps per launch, halo lanes (hotspot2h) ------------------------------------------
 // The same two-step update with the warp's column halo carried by whole lanes instead of edge
@@ -344,7 +148,8 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2_f32_256(orion_k
 // shuffle away), so there are no scalar outer-column loads, no extra T1 cell and no per-lane
 // edge copies: per row two 16-byte cp.async, two 16-byte ring reads, four shuffles.  6.7 % of
 // the lanes' cells are recomputed halo (the neighbouring warp's), traded for half the
-// memory-pipe instructions of hotspot2_f32.  Clamp-to-edge: the lane holding column 0 takes
+// memory-pipe instructions of an edge-lane form (round 1's hotspot2_f32, measured 0.142 vs
+// 0.140 ms and removed).  Clamp-to-edge: the lane holding column 0 takes
 // its own value as W, the lane holding column W-1 its own value as E; lanes past either edge
 // load clamped columns, write nothing and feed no written cell.  Bit-identical to one-step
 // launches (every cell is hs_cell4's operation sequence, = hs_cell's).

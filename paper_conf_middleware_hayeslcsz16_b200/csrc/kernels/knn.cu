@@ -82,20 +82,21 @@ extern "C" __global__ void __launch_bounds__(64) orion_knn_f4_64(orion_kargs a) 
 extern "C" __global__ void __launch_bounds__(128) orion_knn1_f4_128(orion_kargs a) { ORION_PROBE(a); knn_body<32, 4, 1>(a); }
 extern "C" __global__ void __launch_bounds__(64) orion_knn1_f4_64(orion_kargs a) { ORION_PROBE(a); knn_body<8, 8, 1>(a); }
 
-// ---- tap-split form (knn_f4_t8): 8 threads per pixel ------------------------------------------
+// ---- tap-split form (knn_f4_t16): 16 threads per pixel -----------------------------------------
 // Small frames (C1: 64 x 64 = 4096 pixels) are latency-bound: one pixel per thread still walks
-// a serial chain of 49 taps on 32 of 148 SMs.  Here the 49 taps of a pixel are split over the 8
-// lanes of a lane group (lane g takes taps k = g, g+8, ..., k -> (i, j) = (k/7 - 3, k%7 - 3)),
+// a serial chain of 49 taps on 32 of 148 SMs.  Here the 49 taps of a pixel are split over the LP
+// lanes of a lane group (lane g takes taps k = g, g+LP, ..., k -> (i, j) = (k/7 - 3, k%7 - 3)),
 // read straight from global memory (clamp-to-edge in global coordinates; the frame is L1 / L2
-// resident), and the 8 partial sums are combined by a fixed xor-shuffle tree (offsets 4, 2, 1)
-// whose result lane 0 of the group writes.  Every weight is computed exactly as in knn_body
-// (same tap arithmetic), so the counts -- hence the lerp branch -- are the same; only the order
-// of the weighted sums differs (within the 1e-5 tolerance; bit-identical across occupancy
-// levels, which share this code).  CTA = 128 threads = 16 pixels of one row.
+// resident), and the LP partial sums are combined by a fixed xor-shuffle tree whose result lane
+// 0 of the group writes.  Every weight is computed exactly as in knn_body (same tap arithmetic),
+// so the counts -- hence the lerp branch -- are the same; only the order of the weighted sums
+// differs (within the 1e-5 tolerance; bit-identical across occupancy levels, which share this
+// code).  CTA = 128 threads = 128 / LP pixels of one row.  (LP = 8, round 1's knn_f4_t8, measured
+// 3.4-3.6 vs 3.0-3.07 us per C1 frame and removed.)
 template <int LP>
 __device__ __forceinline__ void knn_tap_split_body(const orion_kargs &a)
 {
-    static_assert(LP == 8 || LP == 16, "lanes per pixel");
+    static_assert(LP == 8 || LP == 16, "lanes per pixel: a power of two dividing 32");
     const int g = threadIdx.x & (LP - 1);
     const int x = blockIdx.x * (128 / LP) + (threadIdx.x / LP);
     const int y = a.row_begin + blockIdx.y;
@@ -135,6 +136,5 @@ __device__ __forceinline__ void knn_tap_split_body(const orion_kargs &a)
         fanout_column(a, x, y, y + 1);
     }
 }
-extern "C" __global__ void __launch_bounds__(128) orion_knn8_f4_128(orion_kargs a) { ORION_PROBE(a); knn_tap_split_body<8>(a); }
 // 16 lanes per pixel (3-4 taps each), 8 pixels of one row per CTA.
 extern "C" __global__ void __launch_bounds__(128) orion_knn16_f4_128(orion_kargs a) { ORION_PROBE(a); knn_tap_split_body<16>(a); }

@@ -21,7 +21,7 @@
 // CTA = 128 threads (4 warps); output tile TW = 122 columns x TH = 23 rows.
 // Shared memory: the input tile (TW+18) x (TH+12) with a 9-column / 6-row
 // clamp-to-edge halo as an (r, g) float2 plane and a b plane (odd pitch; one LDS.64 + one
-// LDS per pixel, conflict-free for both access patterns below), and GMAX buffers of
+// LDS per pixel, conflict-free for both access patterns below), and three buffers of
 // H_o, 32 rows x 128 columns each (odd pitch).  Per pass:
 //   phase A: warp w computes H_o for columns [32w, 32w+32) of each buffer; lane = row
 //            (32 rows = TH + 9), sliding along the row over 38 difference values per
@@ -31,8 +31,10 @@
 //            rows, give D_{-o}(x, .); weights w = 2^(D * (-Noise log2 e) + geo) and
 //            the accumulation of w*p, w and [w > wthr] for both offsets.  Lanes touch
 //            consecutive columns: conflict-free.
-// Two __syncthreads per pass.  GMAX = 1: 24 passes, 75.7 KB smem (3 CTAs/SM);
-// GMAX = 3: 10 passes, 108.8 KB smem (2 CTAs/SM), ~2.4x fewer phase-A loads.
+// Two __syncthreads per pass; eight passes of three pairs, 108.8 KB of shared memory (2 CTAs/SM).
+// (Round 1 measured and removed: one pair per pass in 24 passes at 3 CTAs/SM, 0.295 ms at C2;
+// exact fixed-point integer windows, 0.27 ms; a 256-thread CTA, 0.28 ms; a (r, g, b, 1)
+// float4 tile plane with two pairs per pass, 0.272 ms -- against 0.234 ms for this form.)
 #include "common.cuh"
 
 #define PB_R 3   // window radius
@@ -203,131 +205,17 @@ ORION_DEVICE void phase_b(const float2 *prg, const float *pb, const float *hb, i
     }
 }
 
-// ---- integer box sums ------------------------------------------------------------------
-// d in [0, 3] (pixels in [0, 1]) is quantised once to a fixed-point integer with 21 fraction
-// bits by a single rounding: bits(fma(d, 2^21, 2^23)) = bits(2^23) + round(d 2^21).  Box sums of
-// those integers are exact, so the 7-term windows slide with one IADD3 per output (the 2^23
-// offsets cancel in the slides; the first window subtracts 7 of them, in wrapping uint32
-// arithmetic).  |error| per difference <= 2^-22, per patch sum <= 49 * 2^-22 = 1.2e-5: a weight
-// error <= 5.7e-6 relative, inside the R-AMB band and the 1e-5 output tolerance.
-constexpr float kQScale = 2097152.0f;            // 2^21
-constexpr float kQMagic = 8388608.0f;            // 2^23
-constexpr unsigned kQMagicBits = 0x4B000000u;    // bits of 2^23
-
-ORION_DEVICE unsigned quant(float d) { return __float_as_uint(__fmaf_rn(d, kQScale, kQMagic)); }
-
-// Sliding 7-term sums of the raw quantised words q[0 .. N+5] (each = magic + value).
-template <int N>
-ORION_DEVICE void window7_q(const unsigned (&q)[N + 6], unsigned (&out)[N])
-{
-    unsigned s = q[0] + q[1] + q[2] + q[3] + q[4] + q[5] + q[6] - 7u * kQMagicBits;
-    out[0] = s;
-#pragma unroll
-    for (int k = 1; k < N; ++k) {
-        s = s + q[k + 6] - q[k - 1];
-        out[k] = s;
-    }
-}
-
-// Sliding 7-term sums of exact integers h[0 .. N+5].
-template <int N>
-ORION_DEVICE void window7_i(const unsigned (&h)[N + 6], unsigned (&out)[N])
-{
-    unsigned s = h[0] + h[1] + h[2] + h[3] + h[4] + h[5] + h[6];
-    out[0] = s;
-#pragma unroll
-    for (int k = 1; k < N; ++k) {
-        s = s + h[k + 6] - h[k - 1];
-        out[k] = s;
-    }
-}
-
-template <int G>
-ORION_DEVICE void phase_a_int(const float2 *prg, const float *pb, unsigned *hs, int lane, int warp,
-                              int i, int j1)
-{
-    const int cb = 3 + HWARP * warp;
-    const int rowc = lane * PW + cb;
-    const int rows = rowc + i * PW + j1;
-    float2 wrg[G];
-    float wb[G];
-#pragma unroll
-    for (int g = 0; g < G - 1; ++g) {
-        wrg[g + 1] = prg[rows + g];
-        wb[g + 1] = pb[rows + g];
-    }
-    unsigned q[G][ND];
-#pragma unroll
-    for (int c = 0; c < ND; ++c) {
-#pragma unroll
-        for (int g = 0; g < G - 1; ++g) {
-            wrg[g] = wrg[g + 1];
-            wb[g] = wb[g + 1];
-        }
-        wrg[G - 1] = prg[rows + c + G - 1];
-        wb[G - 1] = pb[rows + c + G - 1];
-        const float2 ncrg = neg2(prg[rowc + c]);
-        const float cbv = pb[rowc + c];
-#pragma unroll
-        for (int g = 0; g < G; ++g) q[g][c] = quant(diff2rg(wrg[g], wb[g], ncrg, cbv));
-    }
-#pragma unroll
-    for (int g = 0; g < G; ++g) {
-        unsigned h[HWARP];
-        window7_q<HWARP>(q[g], h);
-        unsigned *hrow = hs + g * HBUF + lane * HP + HWARP * warp;
-#pragma unroll
-        for (int c = 0; c < HWARP; ++c) hrow[c] = h[c];
-    }
-}
-
-ORION_DEVICE void phase_b_int(const float2 *prg, const float *pb, const unsigned *hb, int t, int i,
-                              int j, float nl2q, float wthr, Acc &A)
-{
-    const float geo = geo_l2_rt(i, j);
-    unsigned hp[TH + 6], hm[TH + 6], Dp[TH], Dm[TH];
-#pragma unroll
-    for (int c = 0; c < TH + 6; ++c) {
-        hp[c] = hb[(c + 3) * HP + t + 3];           // +o: H column t+3, rows 3 .. TH+8
-        hm[c] = hb[(c + 3 - i) * HP + t + 3 - j];   // -o: H column t+3-j, rows 3-i .. TH+8-i
-    }
-    window7_i<TH>(hp, Dp);
-    window7_i<TH>(hm, Dm);
-#pragma unroll
-    for (int r = 0; r < TH; ++r) {
-        const float wp = ex2(__fmaf_rn(__uint2float_rn(Dp[r]), nl2q, geo));
-        const float wm = ex2(__fmaf_rn(__uint2float_rn(Dm[r]), nl2q, geo));
-        const int pp = (r + 6 + i) * PW + t + 9 + j;      // p(x+j, y+i)
-        const int pm = (r + 6 - i) * PW + t + 9 - j;      // p(x-j, y-i)
-        A.axy[r] = fma2(make_float2(wp, wp), prg[pp], A.axy[r]);
-        A.azs[r] = fma2(make_float2(wp, wp), make_float2(pb[pp], 1.0f), A.azs[r]);
-        A.axy[r] = fma2(make_float2(wm, wm), prg[pm], A.axy[r]);
-        A.azs[r] = fma2(make_float2(wm, wm), make_float2(pb[pm], 1.0f), A.azs[r]);
-        count_above(A, r, wp, wthr);
-        count_above(A, r, wm, wthr);
-    }
-}
-
-// Pass tables: (i, j1, G).  Together they cover the 24 half-plane pairs exactly once.
-__constant__ int kPass1[24][3] = {
-    {0, 1, 1}, {0, 2, 1}, {0, 3, 1},
-    {1, -3, 1}, {1, -2, 1}, {1, -1, 1}, {1, 0, 1}, {1, 1, 1}, {1, 2, 1}, {1, 3, 1},
-    {2, -3, 1}, {2, -2, 1}, {2, -1, 1}, {2, 0, 1}, {2, 1, 1}, {2, 2, 1}, {2, 3, 1},
-    {3, -3, 1}, {3, -2, 1}, {3, -1, 1}, {3, 0, 1}, {3, 1, 1}, {3, 2, 1}, {3, 3, 1}};
-__constant__ int kPass3[10][3] = {
-    {0, 1, 3}, {1, -3, 3}, {1, 0, 2}, {1, 2, 2}, {2, -3, 3}, {2, 0, 2}, {2, 2, 2}, {3, -3, 3}, {3, 0, 2}, {3, 2, 2}};
-// Float path, three offsets per pass in 8 passes: (i, j1, vert) -- seven sliding passes
-// (i, j1 .. j1+2) and one vertical pass (1 .. 3, 3).
+// The 24 half-plane pairs in eight passes of three offsets, (i, j1, vert): seven sliding passes
+// (i, j1 .. j1+2) and one vertical pass (1 .. 3, 3) -- every pair exactly once.
 __constant__ int kPass8[8][3] = {
     {0, 1, 0}, {1, -3, 0}, {1, 0, 0}, {2, -3, 0}, {2, 0, 0}, {3, -3, 0}, {3, 0, 0}, {1, 3, 1}};
 
-template <int GMAX, bool INT>
 __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 {
     extern __shared__ float4 smem4[];
     float2 *prg = reinterpret_cast<float2 *>(smem4);             // (r, g) plane
     float *pb = reinterpret_cast<float *>(prg + PR * PW);         // b plane
-    float *hs = pb + PR * PW;               // GMAX buffers of H_o: AR rows x HP
+    float *hs = pb + PR * PW;               // 3 buffers of H_o: AR rows x HP
 
     const int tid = threadIdx.x;
     const int lane = tid & 31, warp = tid >> 5;
@@ -365,44 +253,19 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
         for (int q = 0; q < (TH + 3) / 4; ++q) A.cnt[q] = c1 * 0x01010101u;
     }
 
-    constexpr bool P8 = GMAX == 3 && !INT;        // the 8-pass float schedule
-    constexpr int NPASS = GMAX == 1 ? 24 : (P8 ? 8 : 10);
 #pragma unroll 1
-    for (int ps = 0; ps < NPASS; ++ps) {
-        const int i = GMAX == 1 ? kPass1[ps][0] : (P8 ? kPass8[ps][0] : kPass3[ps][0]);
-        const int j1 = GMAX == 1 ? kPass1[ps][1] : (P8 ? kPass8[ps][1] : kPass3[ps][1]);
-        const int G = GMAX == 1 ? 1 : (P8 ? 3 : kPass3[ps][2]);
-        const int vert = P8 ? kPass8[ps][2] : 0;
-        unsigned *hi = reinterpret_cast<unsigned *>(hs);
-        if (INT) {
-            if (GMAX == 1 || G == 1)
-                phase_a_int<1>(prg, pb, hi, lane, warp, i, j1);
-            else if (G == 2)
-                phase_a_int<2>(prg, pb, hi, lane, warp, i, j1);
-            else
-                phase_a_int<(GMAX >= 3 ? 3 : 1)>(prg, pb, hi, lane, warp, i, j1);
-        } else if (P8) {
-            if (vert)
-                phase_a<3, true>(prg, pb, hs, lane, warp, i, j1);
-            else
-                phase_a<3>(prg, pb, hs, lane, warp, i, j1);
-        } else {
-            if (GMAX == 1 || G == 1)
-                phase_a<1>(prg, pb, hs, lane, warp, i, j1);
-            else if (G == 2)
-                phase_a<2>(prg, pb, hs, lane, warp, i, j1);
-            else
-                phase_a<(GMAX >= 3 ? 3 : 1)>(prg, pb, hs, lane, warp, i, j1);
-        }
+    for (int ps = 0; ps < 8; ++ps) {
+        const int i = kPass8[ps][0], j1 = kPass8[ps][1], vert = kPass8[ps][2];
+        if (vert)
+            phase_a<3, true>(prg, pb, hs, lane, warp, i, j1);
+        else
+            phase_a<3>(prg, pb, hs, lane, warp, i, j1);
         __syncthreads();
         if (t < TW) {
 #pragma unroll 1
-            for (int g = 0; g < G; ++g) {
+            for (int g = 0; g < 3; ++g) {
                 const int ig = vert ? i + g : i, jg = vert ? j1 : j1 + g;
-                if (INT)
-                    phase_b_int(prg, pb, hi + g * HBUF, t, ig, jg, nl2 * (1.0f / kQScale), wthr, A);
-                else
-                    phase_b(prg, pb, hs + g * HBUF, t, ig, jg, nl2, wthr, A);
+                phase_b(prg, pb, hs + g * HBUF, t, ig, jg, nl2, wthr, A);
             }
         }
         __syncthreads();
@@ -424,13 +287,9 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 }  // namespace
 
 #ifndef NLMB_WIDE
-// One pair per pass: 3 planar planes + 1 H buffer = 75 732 B of shared memory.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_box_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<1, false>(a); }
-// Up to three pairs per pass: 3 planar planes + 3 H buffers = 108 756 B of shared memory.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_box3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<3, false>(a); }
-// Integer (fixed-point, exact) box sums, up to three pairs per pass.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_boxi3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<3, true>(a); }
+// 122-column tiles, three pairs per pass: 3 planar planes + 3 H buffers = 108 756 B of shared memory.
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_box3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body(a); }
 #else
-// 128-column tiles, up to three pairs per pass: 115 188 B of shared memory.
-extern "C" __global__ void __launch_bounds__(128) orion_nlm_boxw3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body<3, false>(a); }
+// 128-column tiles, three pairs per pass: 115 188 B of shared memory.
+extern "C" __global__ void __launch_bounds__(128) orion_nlm_boxw3_f4_128(orion_kargs a) { ORION_PROBE(a); nlm_box_body(a); }
 #endif

@@ -26,8 +26,6 @@ extern "C" const char liborion_ptx_nlm_regheavy[];
 extern "C" const char liborion_ptx_hotspot[];
 extern "C" const char liborion_ptx_gen[];
 extern "C" const char liborion_ptx_srad[];
-extern "C" const char liborion_ptx_nlm_box256[];
-extern "C" const char liborion_ptx_nlm_box4[];
 extern "C" const char liborion_ptx_nlm_boxw[];
 
 namespace orion {
@@ -41,8 +39,6 @@ static const char *module_ptx(const char *module)
     if (!std::strcmp(module, "hotspot")) return liborion_ptx_hotspot;
     if (!std::strcmp(module, "gen")) return liborion_ptx_gen;
     if (!std::strcmp(module, "srad")) return liborion_ptx_srad;
-    if (!std::strcmp(module, "nlm_box256")) return liborion_ptx_nlm_box256;
-    if (!std::strcmp(module, "nlm_box4")) return liborion_ptx_nlm_box4;
     if (!std::strcmp(module, "nlm_boxw")) return liborion_ptx_nlm_boxw;
     return nullptr;
 }
@@ -56,38 +52,23 @@ static const KernelDef kKernels[] = {
     // one pixel per thread: small (launch-bound) frames
     {"knn_f4_p1", 128, "orion_knn1_f4_128", "knn", 32, 4, 32, 4, 3, K_KNN, 1, 0, 1, 1, 1},
     {"knn_f4_p1", 64, "orion_knn1_f4_64", "knn", 8, 8, 8, 8, 3, K_KNN, 1, 0, 1, 1, 1},
-    // 8 threads per pixel (taps split, shuffle-tree combine), 16 pixels of one row per CTA, no tile
-    {"knn_f4_t8", 128, "orion_knn8_f4_128", "knn", 128, 1, 16, 1, 3, K_KNN, 0, 0, 1, 1, 1},
     // 16 threads per pixel, 8 pixels of one row per CTA
     {"knn_f4_t16", 128, "orion_knn16_f4_128", "knn", 128, 1, 8, 1, 3, K_KNN, 0, 0, 1, 1, 1},
-    // nlm_box: 3 planar (122+18) x (23+12) fp32 planes (pitch 141) + 32 x 129 floats of H_o
-    // up to 3 offset pairs per pass: 3 H_o buffers (2 CTAs/SM) -- the C2 / C5 default
+    // nlm_box: 3 planar (122+18) x (23+12) fp32 planes (pitch 141) + 3 H_o buffers of 32 x 129
+    // floats, 3 offset pairs per pass (2 CTAs/SM)
     {"nlm_f4", 128, "orion_nlm_box3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
      3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},
-    // (r, g, b, 1) float4 tile plane (pitch 141) + 2 H_o buffers, two pairs per pass (2 CTAs/SM)
-    {"nlm_f4_q", 128, "orion_nlm_box4_f4_128", "nlm_box4", 128, 1, 122, 23, 6, K_NLM, 0,
-     35 * 141 * 16 + 2 * 32 * 129 * 4, 1, 1, 1},
-    // 128-column tiles: planes (128+20) x 35 (pitch 149) + 3 H buffers of 32 x 137 floats
+    // 128-column tiles: planes (128+20) x 35 (pitch 149) + 3 H buffers of 32 x 137 floats -- the
+    // C2 / C5 default
     {"nlm_f4_w", 128, "orion_nlm_boxw3_f4_128", "nlm_boxw", 128, 1, 128, 23, 6, K_NLM, 0,
      3 * 35 * 149 * 4 + 3 * 32 * 137 * 4, 1, 1, 1},
-    // same, integer (fixed-point, exact) box sums
-    {"nlm_f4_i", 128, "orion_nlm_boxi3_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
-     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},
-    // same tile, 256 threads (8 warps per CTA)
-    {"nlm_f4_w8", 256, "orion_nlm_box256_f4_256", "nlm_box256", 256, 1, 122, 23, 6, K_NLM, 0,
-     3 * 35 * 141 * 4 + 3 * 32 * 129 * 4, 1, 1, 1},
-    // one offset pair per pass: 1 H_o buffer (3 CTAs/SM)
-    {"nlm_f4_g1", 128, "orion_nlm_box_f4_128", "nlm_box", 128, 1, 122, 23, 6, K_NLM, 0,
-     3 * 35 * 141 * 4 + 32 * 129 * 4, 1, 1, 1},
+    // the direct 2401-term definition (cross-check form), and the register-heavy C4 kernel
     {"nlm_f4_direct", 128, "orion_nlm_direct_f4_128", "nlm_direct", 32, 4, 32, 4, 6, K_NLM, 1, 0},
     {"nlm_f4_regheavy", 128, "orion_nlm_regheavy_f4_128", "nlm_regheavy", 32, 4, 32, 4, 6, K_NLM, 1, 0},
     {"nlm_f4_regheavy", 64, "orion_nlm_regheavy_f4_64", "nlm_regheavy", 8, 8, 8, 8, 6, K_NLM, 1, 0},
     {"hotspot_f32", 256, "orion_hotspot_f32_256", "hotspot", 32, 8, 128, 128, 1, K_STENCIL, 0, 0},
     {"hotspot_f32", 128, "orion_hotspot_f32_128", "hotspot", 32, 4, 128, 64, 1, K_STENCIL, 0, 0},
-    // two steps per launch (temporal blocking): reads 2 rows beyond its strip; width % 4 == 0
-    // the rows each warp walks stream through a 6-slot cp.async ring: 8 warps x 6 x 272 floats
-    {"hotspot2_f32", 256, "orion_hotspot2_f32_256", "hotspot", 32, 8, 128, 256, 2, K_STENCIL, 0, 8 * 6 * 272 * 4, 4, 2},
-    // two steps per launch with whole halo lanes: 120 output columns per warp, 6-slot ring of
+    // two steps per launch (temporal blocking) with whole halo lanes: 120 output columns per warp, 6-slot ring of
     // 8 warps x 6 x 256 floats
     {"hotspot2h_f32", 256, "orion_hotspot2h_f32_256", "hotspot", 32, 8, 120, 256, 2, K_STENCIL, 0, 8 * 6 * 256 * 4, 4, 2},
     // four steps per launch, whole halo lanes: the same 120-column warps walking 64-row strips as

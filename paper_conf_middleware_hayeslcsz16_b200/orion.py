@@ -27,12 +27,12 @@ LIM_REGS, LIM_SMEM, LIM_WARPS, LIM_BLOCKS = 1, 2, 4, 8
 DIR_DECREASING, DIR_INCREASING = -1, 1
 SELECT_FASTEST, SELECT_LOWEST_WITHIN_TOL = 0, 1
 
-HALO = {"knn_f4": 3, "knn_f4_p1": 3, "knn_f4_t8": 3, "knn_f4_t16": 3, "nlm_f4": 6, "nlm_f4_g1": 6, "nlm_f4_i": 6, "nlm_f4_q": 6, "nlm_f4_w": 6, "nlm_f4_w8": 6, "nlm_f4_direct": 6, "nlm_f4_regheavy": 6, "hotspot_f32": 1, "hotspot2_f32": 2,
-        "hotspot2h_f32": 2, "hotspot4h_f32": 4, "srad_f32": 2, "srad_f32h": 2, "srad_f32_tile": 2}
+HALO = {"knn_f4": 3, "knn_f4_p1": 3, "knn_f4_t16": 3, "nlm_f4": 6, "nlm_f4_w": 6, "nlm_f4_direct": 6,
+        "nlm_f4_regheavy": 6, "hotspot_f32": 1, "hotspot2h_f32": 2, "hotspot4h_f32": 4, "srad_f32": 2,
+        "srad_f32h": 2, "srad_f32_tile": 2}
 # stencil steps one launch advances (temporal blocking); every other kernel: 1
-STEPS_PER_LAUNCH = {"hotspot2_f32": 2, "hotspot2h_f32": 2, "hotspot4h_f32": 4}
-KERNELS = ("knn_f4", "knn_f4_p1", "knn_f4_t8", "knn_f4_t16", "nlm_f4", "nlm_f4_w", "nlm_f4_q", "nlm_f4_g1", "nlm_f4_i", "nlm_f4_w8", "nlm_f4_direct", "nlm_f4_regheavy", "hotspot_f32", "hotspot2_f32", "hotspot2h_f32",
-           "hotspot4h_f32", "srad_f32", "srad_f32h", "srad_f32_tile")
+STEPS_PER_LAUNCH = {"hotspot2h_f32": 2, "hotspot4h_f32": 4}
+KERNELS = tuple(HALO)
 
 
 class OrionError(RuntimeError):

@@ -175,3 +175,20 @@ def test_default_params_match_the_oracles_constants():
     assert O.default_params("srad_f32h")[0] == 0.5
     with pytest.raises(O.OrionError):
         O.default_params("no_such_kernel")
+
+
+def test_every_header_entry_cites_its_passage():
+    # each declaration in include/orion.h is preceded by a comment citing the passage (PAPER.md
+    # line, figure / equation, SURVEY section or DESIGN reading) that defines the operation
+    txt = open(os.path.join(ROOT, "include", "orion.h")).read()
+    missing = []
+    for m in re.finditer(r"\n(orion_status|void|const char \*|long long) (orion_[a-z0-9_]+)\(", txt):
+        before = txt[:m.start()].rstrip()
+        end = before.rfind("*/")
+        if before[end:].count(";") > 2:        # no comment block within the last declarations
+            missing.append(m.group(2))
+            continue
+        com = before[before.rfind("/*", 0, end):end]
+        if not re.search(r"P:L|SURVEY|reading|Fig\.|Eq\.", com):
+            missing.append(m.group(2))
+    assert not missing, missing

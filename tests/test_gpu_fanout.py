@@ -22,7 +22,7 @@ def dev():
     return 0
 
 
-@pytest.mark.parametrize("kernel,halo", [("nlm_f4", 6), ("knn_f4", 3), ("knn_f4_t8", 3), ("knn_f4_t16", 3), ("nlm_f4_i", 6), ("nlm_f4_q", 6), ("nlm_f4_w", 6)])
+@pytest.mark.parametrize("kernel,halo", [("nlm_f4", 6), ("knn_f4", 3), ("knn_f4_t16", 3), ("nlm_f4_w", 6)])
 @pytest.mark.parametrize("P", [2, 3])
 def test_fanout_gathers_bands_bit_exact(dev, kernel, halo, P):
     W, H = 250, 131

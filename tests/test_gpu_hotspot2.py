@@ -1,6 +1,6 @@
-"""hotspot2_f32 / hotspot2h_f32 (two explicit steps per launch, the intermediate step kept in
-registers; edge lanes vs whole halo lanes) and hotspot4h_f32 (four steps per launch, a 4-stage
-register pipeline on the halo-lane warps):
+"""hotspot2h_f32 (two explicit steps per launch, the intermediate step kept in registers, whole
+halo lanes) and hotspot4h_f32 (four steps per launch, a 4-stage register pipeline on the
+halo-lane warps):
 bit-identical to two launches of the one-step kernel and to the oracle's fp32 form, at every
 occupancy level, on ragged heights and at the image borders."""
 import numpy as np
@@ -15,7 +15,7 @@ pytestmark = pytest.mark.gpu
 from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
 
 
-@pytest.fixture(scope="module", params=["hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32"])
+@pytest.fixture(scope="module", params=["hotspot2h_f32", "hotspot4h_f32"])
 def v2(request):
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")

@@ -45,7 +45,6 @@ def _run(kernel, t0, pw, iterations, roi=None):
 
 @pytest.mark.parametrize("kernel,shape,launches,steps", [("hotspot_f32", (300, 203), 9, 9),
                                                           ("hotspot_f32", (97, 1), 4, 4),
-                                                          ("hotspot2_f32", (260, 131), 6, 12),
                                                           ("hotspot2h_f32", (244, 131), 6, 12),
                                                           ("hotspot4h_f32", (244, 131), 5, 20)])
 def test_hotspot_run_host_bit_exact(dev, kernel, shape, launches, steps):

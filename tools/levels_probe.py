@@ -8,7 +8,7 @@ import time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
 
-kernels = sys.argv[1:] or ["srad_f32", "hotspot_f32", "hotspot2_f32", "knn_f4", "nlm_f4_regheavy", "nlm_f4"]
+kernels = sys.argv[1:] or ["srad_f32", "hotspot_f32", "hotspot2h_f32", "knn_f4", "nlm_f4_regheavy", "nlm_f4"]
 for k in kernels:
     for mode in (O.REALISE_MIN_CARVEOUT, O.REALISE_MAX_SMEM):
         t = time.time()

@@ -15,13 +15,13 @@ sp = torch.cuda.current_stream().cuda_stream
 W, H = 70, 45                                     # ragged: not a multiple of any tile
 img = torch.empty((H, W, 4), device="cuda")
 O.generate_rgba(0, img.data_ptr(), W, H, sigma=0.13, stream=sp)
-for k in ("knn_f4", "knn_f4_t8", "knn_f4_t16", "nlm_f4", "nlm_f4_w", "nlm_f4_q", "nlm_f4_i", "nlm_f4_g1", "nlm_f4_w8", "nlm_f4_direct", "nlm_f4_regheavy"):
+for k in ("knn_f4", "knn_f4_p1", "knn_f4_t16", "nlm_f4", "nlm_f4_w", "nlm_f4_direct", "nlm_f4_regheavy"):
     v, _ = O.build_all_levels(0, k)
     out = torch.empty_like(img)
     full = torch.empty_like(img)
     for i in (0, len(v) - 1):
         a = O.denoise_args(k, img.data_ptr(), out.data_ptr(), W, H)
-        if k in ("knn_f4", "knn_f4_t8", "knn_f4_t16", "nlm_f4", "nlm_f4_w", "nlm_f4_q", "nlm_f4_i", "nlm_f4_g1", "nlm_f4_w8"):
+        if k in ("knn_f4", "knn_f4_p1", "knn_f4_t16", "nlm_f4", "nlm_f4_w"):
             a = O.with_fanout(a, [full.data_ptr()])
         v.launch(i, a, sp)
     torch.cuda.synchronize()
@@ -32,7 +32,7 @@ pw = torch.empty_like(t0)
 t1 = torch.empty_like(t0)
 O.generate_thermal(0, t0.data_ptr(), pw.data_ptr(), WT, HT, stream=sp)
 q0 = torch.empty(1, device="cuda")
-for k in ("hotspot_f32", "hotspot2_f32", "hotspot2h_f32", "hotspot4h_f32", "srad_f32", "srad_f32h", "srad_f32_tile"):
+for k in ("hotspot_f32", "hotspot2h_f32", "hotspot4h_f32", "srad_f32", "srad_f32h", "srad_f32_tile"):
     v, _ = O.build_all_levels(0, k)
     for w in ((WT, WT - 3) if k in ("srad_f32", "srad_f32_tile") else (WT,)):
         for i in (0, len(v) - 1):

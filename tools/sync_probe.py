@@ -2,7 +2,7 @@
 
 The Fig. 9 tuner times one launch per explored level; this probe shows how far a launch
 timed after a host sync is from the same level timed back to back (the steady state the
-final kernel runs in).  Usage: python tools/sync_probe.py [hotspot2_f32|srad_f32|nlm_f4]
+final kernel runs in).  Usage: python tools/sync_probe.py [hotspot2h_f32|srad_f32|nlm_f4]
 """
 import os
 import statistics
@@ -13,7 +13,7 @@ import torch  # noqa: E402
 
 from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
 
-kern = sys.argv[1] if len(sys.argv) > 1 else "hotspot2_f32"
+kern = sys.argv[1] if len(sys.argv) > 1 else "hotspot2h_f32"
 torch.cuda.set_device(0)
 sp = torch.cuda.current_stream().cuda_stream
 if kern.startswith("hotspot") or kern.startswith("srad"):
