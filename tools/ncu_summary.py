@@ -40,7 +40,7 @@ KEYS = [
 
 def main():
     kid, rep = sys.argv[1], sys.argv[2]
-    rnd = sys.argv[3] if len(sys.argv) > 3 else "r01"
+    rnd = sys.argv[3] if len(sys.argv) > 3 else "r02"
     out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     hdr, units, data = rows[0], rows[1], rows[2:]
