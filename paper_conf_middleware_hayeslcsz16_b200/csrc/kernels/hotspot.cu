@@ -140,6 +140,7 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
 
+
 // ---- two steps per launch, halo lanes (hotspot2h) ------------------------------------------
 // The same two-step update with the warp's column halo carried by whole lanes instead of edge
 // lanes: a warp loads 128 consecutive columns [base-4, base+124) as float4 lanes and writes the
@@ -293,6 +294,11 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2h_f32_256(orion_
 // by DRAM (long-scoreboard 1.9 stalls per issue on the ring waits, FMA pipe 56 % busy).  64-row
 // strips also make a strip's 72 iterations exactly the 9 prologue/fill iterations + 7 bodies of 9
 // (no slow remainder loop): 61-row strips (3.96 instead of 3.73 waves) measured 0.159 vs 0.156.
+// Round 2: the ring rows moved by TMA bulk copies (cp.async.bulk of each warp's 512-byte T0 and
+// P segments by one elected lane, completing on per-slot mbarriers; edge column blocks kept
+// LDGSTS) measured 0.176 vs 0.157 ms per launch (three A/B pairs on one box), and a 12-slot TMA
+// ring 0.218 ms: at this granularity the per-row elect / expect_tx / try_wait / warp-sync cost
+// more than the 2 LDGSTS they replace.  Removed.
 #ifndef HS_ROWS
 #define HS_ROWS 64
 #endif
