@@ -62,10 +62,11 @@ WORKLOADS = {
                name="imageDenoising NLM 16384x16384 RGBA row-sharded with halos + all-gather",
                insts=24 * 30 + 10, bytes=32, steps=10, cfg_index=4),
     # NEXT-4: a second Rodinia stencil (srad), 8 B/cell-iteration (read J, write J')
-    "srad": dict(kernel="srad_f32h", W=8192, H=8192, unit="Mcell-steps/s", name="SRAD 8192x8192 fp32 (NEXT-4)",
+    "srad": dict(kernel="srad_f32hs", W=8192, H=8192, unit="Mcell-steps/s", name="SRAD 8192x8192 fp32 (NEXT-4)",
                  insts=60, bytes=8, steps=100, cfg_index=None),
 }
 SUB_RECORDS = ("c1", "c3", "c4", "srad", "c5")
+ROI = (0, 127, 0, 127)     # SRAD's ROI statistics window (reading R-SRAD: Rodinia's default)
 
 
 def load_peaks():
@@ -421,6 +422,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     kernel, W, H = kernel or wl["kernel"], wl["W"], wl["H"]
     is_srad = kernel.startswith("srad_f32")
     is_stencil = kernel.startswith("hotspot") or is_srad
+    fused = kernel == "srad_f32hs"
     # launch-bound frames (C1 by default) replay their settled iterations as one CUDA graph,
     # whose kernel nodes are plain launches: the whole configuration (sweep included) then runs
     # without programmatic dependent launch, so every level is timed the way the loop runs it
@@ -444,21 +446,26 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     nframes = max(2, math.ceil(2 * 126e6 / (2 * frame_bytes)) + 1)
     if is_stencil:
         nframes = 1
-        t_a = torch.empty((H, W), device=dev)
-        t_b = torch.empty((H, W), device=dev)
+        # srad_f32hs: the ROI statistics slots travel behind each grid
+        extra = O.SRAD_STATS_FLOATS if fused else 0
+        t_a = torch.empty(H * W + extra, device=dev)[:H * W].view(H, W)
+        t_b = torch.empty(H * W + extra, device=dev)[:H * W].view(H, W)
         pw = torch.empty((H, W), device=dev)
         O.generate_thermal(local, t_a.data_ptr(), pw.data_ptr(), W, H, seed=1 + rank, stream=sp)
+        if fused:
+            O.srad_stats_init(local, t_a.data_ptr(), W, H, ROI, sp)
         state = {"a": t_a, "b": t_b}
         q0 = torch.empty(1, device=dev)   # srad: the ROI statistic of the current iteration
 
         def grid_args(src, dst):
             if is_srad:
-                return O.srad_args(src.data_ptr(), dst.data_ptr(), q0.data_ptr(), W, H)
+                return O.srad_args(src.data_ptr(), dst.data_ptr(), 0 if fused else q0.data_ptr(), W, H,
+                                   roi=ROI if fused else None)
             return O.hotspot_args(src.data_ptr(), dst.data_ptr(), pw.data_ptr(), W, H)
 
         def step_args(s):
-            if is_srad:   # the iteration's ROI statistics precede the tuned update kernel
-                O.srad_roi_stats(local, state["a"].data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
+            if is_srad and not fused:   # the iteration's ROI statistics precede the tuned update kernel
+                O.srad_roi_stats(local, state["a"].data_ptr(), W, H, ROI, q0.data_ptr(), sp)
             a = grid_args(state["a"], state["b"])
             state["a"], state["b"] = state["b"], state["a"]
             return a
@@ -477,8 +484,8 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     sweep_args = step_args(0)
     if is_stencil:
         state["a"], state["b"] = t_a, t_b
-        if is_srad:
-            O.srad_roi_stats(local, t_a.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
+        if is_srad and not fused:
+            O.srad_roi_stats(local, t_a.data_ptr(), W, H, ROI, q0.data_ptr(), sp)
         sweep_args = grid_args(t_a, t_b)
     ms = variants.sweep(sweep_args, sp, rounds=rounds)
     best = min(range(nlev), key=lambda i: ms[i])
@@ -606,7 +613,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
         h_o = torch.empty((H, W)).pin_memory()
         if is_srad:
             ja = O.srad_args(h_t.data_ptr(), h_o.data_ptr(), 0, W, H)
-            aux_dev, roi = q0, (0, 127, 0, 127)
+            aux_dev, roi = q0, ROI
         else:
             ja = O.hotspot_args(h_t.data_ptr(), h_o.data_ptr(), h_p.data_ptr(), W, H)
             aux_dev, roi = pw, None
@@ -709,18 +716,25 @@ def measure_energy(key: str, args, kernel: str, local: int = 0, window_s: float 
     W, H = wl["W"], wl["H"]
     is_srad = kernel.startswith("srad")
     is_stencil = kernel.startswith("hotspot") or is_srad
+    fused = kernel == "srad_f32hs"
     realise = O.REALISE_MIN_CARVEOUT if args.realise == "min" else O.REALISE_MAX_SMEM
     pdl_prev = O.set_pdl(False)          # every level below is replayed as a CUDA graph (plain launches)
     v, res = O.build_all_levels(local, kernel, mode=realise)
     n = len(v)
     if is_stencil:
-        a_ = torch.empty((H, W), device="cuda")
-        b_ = torch.empty((H, W), device="cuda")
+        extra = O.SRAD_STATS_FLOATS if fused else 0
+        a_ = torch.empty(H * W + extra, device="cuda")[:H * W].view(H, W)
+        b_ = torch.empty(H * W + extra, device="cuda")[:H * W].view(H, W)
         p_ = torch.empty((H, W), device="cuda")
         O.generate_thermal(local, a_.data_ptr(), p_.data_ptr(), W, H, seed=1, stream=sp)
         q0 = torch.empty(1, device="cuda")
-        if is_srad:
-            O.srad_roi_stats(local, a_.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
+        if fused:
+            O.srad_stats_init(local, a_.data_ptr(), W, H, ROI, sp)
+            O.srad_stats_init(local, b_.data_ptr(), W, H, ROI, sp)
+            args_pp = [O.srad_args(a_.data_ptr(), b_.data_ptr(), 0, W, H, roi=ROI),
+                       O.srad_args(b_.data_ptr(), a_.data_ptr(), 0, W, H, roi=ROI)]
+        elif is_srad:
+            O.srad_roi_stats(local, a_.data_ptr(), W, H, ROI, q0.data_ptr(), sp)
             args_pp = [O.srad_args(a_.data_ptr(), b_.data_ptr(), q0.data_ptr(), W, H),
                        O.srad_args(b_.data_ptr(), a_.data_ptr(), q0.data_ptr(), W, H)]
         else:
@@ -1029,7 +1043,7 @@ def run_single(args):
         line["configs"] = subs
         if not args.no_energy:
             nx = {}
-            for sub, kern in (("srad", "srad_f32h"), ("c3", "hotspot_f32"), ("c1", "knn_f4_t16"), ("c4", "nlm_f4_regheavy")):
+            for sub, kern in (("srad", "srad_f32hs"), ("c3", "hotspot_f32"), ("c1", "knn_f4_t16"), ("c4", "nlm_f4_regheavy")):
                 try:
                     nx[f"{sub}:{kern}"] = measure_energy(sub, args, kern, local=local)
                 except Exception as ex:

@@ -140,7 +140,9 @@ orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int bloc
  *   hotspot: "hotspot_f32" (one step per launch; T = 256 / 128), "hotspot2h_f32" (two
  *       steps per launch, whole halo lanes), "hotspot4h_f32" (four steps per launch as a 4-stage
  *       register pipeline; the C3 default) -- width % 4 == 0 for the multi-step forms;
- *   srad: "srad_f32h" (float4 strips, whole halo lanes, width % 4 == 0; the default),
+ *   srad: "srad_f32hs" (float4 strips, whole halo lanes, the ROI statistics fused in;
+ *       width % 4 == 0; the default), "srad_f32h" (the same strips after a separate statistics
+ *       kernel),
  *       "srad_f32" (register-sliding, any width), "srad_f32_tile" (shared-memory form; both
  *       cross-check forms, same bits).
  * block_threads = 0 selects the kernel's default CTA size.  ORION_E_INVALID for an unknown id /
@@ -336,7 +338,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
 /* A whole iterative stencil run end to end from HOST buffers -- the Rodinia driver shape
  * (copy the grid in, iterate, copy it out), the iterations being the ones
  * Fig. 9 tunes across (P:L651-P:L653).  Kernels of kind hotspot ("hotspot_f32",
- * "hotspot2h_f32", "hotspot4h_f32") and srad ("srad_f32", "srad_f32h", "srad_f32_tile") only, whole grids only
+ * "hotspot2h_f32", "hotspot4h_f32") and srad ("srad_f32", "srad_f32h", "srad_f32hs", "srad_f32_tile") only, whole grids only
  * (a->row_begin = a->src_row_begin = a->dst_row_begin = 0, a->row_end = a->src_row_end =
  * a->height).
  *   a->src  host initial grid (fp32, width x height, row-major; pinned for async copies)
@@ -344,6 +346,9 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
  *   a->dst  host buffer receiving the grid after `iterations` launches
  *   dev_a, dev_b  caller-owned device grids (ping-pong), width x height fp32 each
  *   dev_aux hotspot: device power map buffer (filled here); srad: the device float q0sqr
+ *           ("srad_f32hs": unused, may be NULL -- dev_a / dev_b then hold width x height +
+ *           ORION_SRAD_STATS_FLOATS floats each, and the slots of the initial grid are written
+ *           once with orion_srad_stats_init before the first iteration)
  *   roi     srad only: {r1, r2, c1, c2} of the ROI statistics run before every iteration
  * Copies in, runs `iterations` orion_tune_step iterations on `stream` (hotspot2h_f32 advances
  * two time steps per iteration, hotspot4h_f32 four), copies the final grid out and synchronises the stream.
@@ -440,6 +445,22 @@ orion_status orion_generate_thermal(int device, void *t0, void *power, int width
  * (whose fparam[0] = lambda).  Asynchronous on `stream`. */
 orion_status orion_srad_roi_stats(int device, const void *J, int width, int height, int r1, int r2, int c1, int c2,
                                   void *q0, void *stream);
+/* SRAD with the ROI statistics fused into the update ("srad_f32hs"): every grid it reads or writes
+ * is width x height floats FOLLOWED by ORION_SRAD_STATS_FLOATS floats of statistics slots (the
+ * ROI's partial sums, in double).  A launch derives q0sqr (reading R-SRAD, Table 2) from
+ * the slots behind src and writes its output ROI's slots behind dst, so an iteration is ONE
+ * kernel (the tuner's iteration, P:L651-P:L653) instead of statistics + update.  Its orion_args:
+ * whole grids (row ranges 0 .. height), fparam[0] = lambda, fparam[1..4] = r1, r2, c1, c2
+ * (inclusive ROI, exact integers), aux unused; width % 4 == 0. */
+#define ORION_SRAD_STAT_SLOTS 64
+#define ORION_SRAD_STATS_FLOATS (4 * ORION_SRAD_STAT_SLOTS)
+/* The first iteration's input: write the statistics slots of grid J (device, width x height +
+ * ORION_SRAD_STATS_FLOATS floats) for ROI rows [r1, r2] x cols [c1, c2] in "srad_f32hs"'s
+ * partition, asynchronously on `stream` (reading R-SRAD's ROI statistics).
+ * ORION_E_INVALID for a ROI outside the grid or spanning more than ORION_SRAD_STAT_SLOTS
+ * (42-row strip, 120-column block) slots, or width % 4 != 0. */
+orion_status orion_srad_stats_init(int device, void *J, int width, int height, int r1, int r2, int c1, int c2,
+                                   void *stream);
 /* Write `bytes` of `buf` (a device scratch buffer larger than L2) to evict the L2: a
  * measurement utility (cold-cache timing, SURVEY §8(d) timing protocol); no method math. */
 orion_status orion_flush_l2(int device, void *buf, long long bytes, void *stream);

@@ -108,6 +108,96 @@ ORION_DEVICE SradConsts srad_consts(const orion_kargs &a)
     return k;
 }
 
+// ---- ROI statistics carried by the grids (srad_f32hs) ------------------------------------------
+// The fused kernel reads q0sqr of ITS input from partial sums stored behind the input grid and
+// writes the partial sums of its output's ROI behind the output grid, so the next iteration needs
+// no separate statistics kernel.  Partition (shared with orion_srad_stats_init): the warp
+// (strip g = y / SRADH_RY, column block b = x / 120) owning a ROI cell sums, in double, the ROI
+// cells it writes -- each lane its own columns row by row, then a fixed xor-shuffle tree -- into
+// slot (g - g1) * nb + (b - b1), g1 / b1 the first strip / block the ROI touches.  Every launch
+// reduces the slots in index order, so q0sqr is deterministic and the same at every level.
+#ifndef SRADH_RY
+#define SRADH_RY 42
+#endif
+constexpr int SRAD_STAT_SLOTS = 64;           // (sum, sum of squares) doubles per slot
+
+struct SradRoi {
+    int r1, r2, c1, c2;      // inclusive ROI
+    int g1, b1, nb, nslots;  // first strip / block, blocks per strip row, slots used
+};
+ORION_DEVICE SradRoi srad_roi(const orion_kargs &a)
+{
+    SradRoi r;
+    r.r1 = (int)a.fparam[1];
+    r.r2 = (int)a.fparam[2];
+    r.c1 = (int)a.fparam[3];
+    r.c2 = (int)a.fparam[4];
+    r.g1 = r.r1 / SRADH_RY;
+    r.b1 = r.c1 / 120;
+    r.nb = r.c2 / 120 - r.b1 + 1;
+    r.nslots = (r.r2 / SRADH_RY - r.g1 + 1) * r.nb;
+    return r;
+}
+// The statistics area behind a width x height grid (16-byte aligned: width % 4 == 0).
+ORION_DEVICE double *srad_stats_area(const void *grid, const orion_kargs &a, int row_begin)
+{
+    return (double *)((float *)grid + ((size_t)a.height - (size_t)row_begin) * (size_t)a.width);
+}
+// q0sqr from the slots of the input grid: lane k reduces slots k, k+32 (fixed order), then a
+// fixed xor tree; every lane returns the same value.
+ORION_DEVICE float srad_q0_from_slots(const double *slots, const SradRoi &r, int lane)
+{
+    double s = 0.0, s2 = 0.0;
+    for (int k = lane; k < r.nslots; k += 32) {
+        s += slots[2 * k];
+        s2 += slots[2 * k + 1];
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        s += __shfl_xor_sync(0xffffffffu, s, o);
+        s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+    }
+    const double n = (double)(r.r2 - r.r1 + 1) * (double)(r.c2 - r.c1 + 1);
+    const double mean = s / n;
+    const double var = s2 / n - mean * mean;
+    return (float)(var / (mean * mean));
+}
+ORION_DEVICE SradConsts srad_consts_q0(float q0, float lam)
+{
+    SradConsts k;
+    k.lam4 = __fmul_rn(0.25f, lam);
+    k.iqden = __frcp_rn(__fmul_rn(q0, __fadd_rn(1.0f, q0)));
+    k.nq = -__fmul_rn(q0, k.iqden);
+    return k;
+}
+// A lane's running ROI sums over the float4 it holds at columns cx .. cx+3 of row y.
+ORION_DEVICE void srad_roi_acc(double &s, double &s2, const float4 &v, int cx, int y, const SradRoi &r, bool own)
+{
+    if (!own || y < r.r1 || y > r.r2) return;
+    const float e[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+        if (cx + k >= r.c1 && cx + k <= r.c2) {
+            const double d = (double)e[k];
+            s += d;
+            s2 = fma(d, d, s2);
+        }
+}
+// Close a warp's sums: fixed xor tree, lane 0 stores its slot (warps outside the ROI store nothing).
+ORION_DEVICE void srad_roi_store(double s, double s2, double *area, int g, int b, const SradRoi &r, int lane)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        s += __shfl_xor_sync(0xffffffffu, s, o);
+        s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+    }
+    if (lane == 0) {
+        const int k = (g - r.g1) * r.nb + (b - r.b1);
+        area[2 * k] = s;
+        area[2 * k + 1] = s2;
+    }
+}
+
 constexpr int SX = 32, SY = 8, RY = 4;        // threads, rows per thread
 constexpr int TW = SX, TH = SY * RY;          // output tile 32 x 32
 constexpr int JW = TW + 3, JH = TH + 3;       // J tile: x0-1 .. x0+TW+1, y0-1 .. y0+TH+1
@@ -451,7 +541,7 @@ namespace {
 constexpr int SRADH_SLOT = 128;   // floats per ring slot: the warp's 128 columns of one J row
 }  // namespace
 
-template <bool CEDGE>
+template <bool CEDGE, bool STATS = false>
 __device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int ys, int ye)
 {
     const int W = a.width, H = a.height;
@@ -460,7 +550,8 @@ __device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int
     const int cxl = clampi(cx, 0, W - 4);
     const bool wclamp = cx == 0, eclamp = cx + 4 >= W;
     const bool writer = lane >= 1 && lane <= 30 && cx < W;
-    const SradConsts kc = srad_consts(a);
+    SradConsts kc;                  // STATS: set after the ring's first rows are in flight (below)
+    if (!STATS) kc = srad_consts(a);
     const float *J = (const float *)a.src - (size_t)a.src_row_begin * (size_t)W + cxl;   // row 0, own columns
     float *Jo = (float *)a.dst + (size_t)cx - (size_t)a.dst_row_begin * (size_t)W;
 
@@ -508,6 +599,9 @@ __device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int
         if (q < nq) issue(ring + q * SRADH_SLOT);
         srad_commit();
     }
+    if (STATS)   // the input's q0sqr from its statistics slots, while the ring rows are in flight
+        kc = srad_consts_q0(srad_q0_from_slots(srad_stats_area(a.src, a, a.src_row_begin), srad_roi(a), lane),
+                            a.fparam[0]);
     float4 j0 = load(ys), j1 = load(min(ys + 1, H - 1)), j2;
     CRow<4> c0 = coeff_row(load(max(ys - 1, 0)), j0, j1), c1;
     auto row = [&](int q, float *sl_read, float *sl_issue, const float4 &N, const float4 &T, float4 &S,
@@ -542,22 +636,70 @@ __device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int
 #undef SH_I
     srad_wait<0>();
     if (ye == H) update_row(H - 1, j0, c0, c0);               // last image row: c_S = own c
+    if (STATS) {
+        // the output ROI's slot: a warp holding ROI cells reads back the cells its lanes just
+        // wrote (same-thread global RAW; off the hot loop, so no registers live across it)
+        const SradRoi roi = srad_roi(a);
+        if (ys <= roi.r2 && ye - 1 >= roi.r1 && base <= roi.c2 && base + 119 >= roi.c1) {
+            double rs = 0.0, rs2 = 0.0;
+            for (int y = max(ys, roi.r1); y <= min(ye - 1, roi.r2); ++y)
+                if (writer)
+                    srad_roi_acc(rs, rs2, *reinterpret_cast<const float4 *>(Jo + (size_t)y * (size_t)W), cx, y, roi,
+                                 true);
+            srad_roi_store(rs, rs2, srad_stats_area(a.dst, a, a.dst_row_begin), ys / SRADH_RY, base / 120, roi, lane);
+        }
+    }
 }
 
 // T = 256 threads (32 x 8 warps), output tile 120 x (8 * SRADH_RY); width % 4 == 0.  42-row
 // strips: a multiple of the 6-row loop body (no remainder iterations), 25 x 69 CTAs at 8192^2.
-#ifndef SRADH_RY
-#define SRADH_RY 42
-#endif
-extern "C" __global__ void __launch_bounds__(256) orion_srad4h_f32_256(orion_kargs a)
+template <bool STATS>
+__device__ __forceinline__ void srad4h_body(const orion_kargs &a)
 {
-    ORION_PROBE(a);
     const int ys = a.row_begin + blockIdx.y * (8 * SRADH_RY) + threadIdx.y * SRADH_RY;
     if (ys >= a.row_end) return;
     const int base = blockIdx.x * 120;
     const bool cedge = base == 0 || base + 124 >= a.width;
     if (cedge)
-        srad_strip_h<true>(a, base, ys, min(ys + SRADH_RY, a.row_end));
+        srad_strip_h<true, STATS>(a, base, ys, min(ys + SRADH_RY, a.row_end));
     else
-        srad_strip_h<false>(a, base, ys, min(ys + SRADH_RY, a.row_end));
+        srad_strip_h<false, STATS>(a, base, ys, min(ys + SRADH_RY, a.row_end));
+}
+extern "C" __global__ void __launch_bounds__(256) orion_srad4h_f32_256(orion_kargs a)
+{
+    ORION_PROBE(a);
+    srad4h_body<false>(a);
+}
+// srad_f32hs: the same strips with the ROI statistics fused in -- q0sqr of the input from the
+// slots behind src, the output ROI's slots written behind dst (no statistics kernel per iteration).
+extern "C" __global__ void __launch_bounds__(256) orion_srad4hs_f32_256(orion_kargs a)
+{
+    ORION_PROBE(a);
+    srad4h_body<true>(a);
+}
+
+// Statistics slots of a grid J (the first iteration's input) in srad_f32hs's partition: one warp
+// per (strip, block) slot of the ROI, the same per-lane column ownership (lanes 1..30 of the
+// 128-column segment [120 b - 4, 120 b + 124)), rows in ascending order, the same xor tree -- so
+// the slots are exactly what a fused launch writing J would have stored.  grid = (nslots), 32
+// threads; a.src = J (width x height + the statistics area), fparam[1..4] = ROI.
+extern "C" __global__ void __launch_bounds__(32) orion_srad_stats_init(orion_kargs a)
+{
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    const SradRoi r = srad_roi(a);
+    const int lane = threadIdx.x;
+    const int k = blockIdx.x;
+    const int g = r.g1 + k / r.nb, b = r.b1 + k % r.nb;
+    const int W = a.width, H = a.height;
+    const int cx = 120 * b - 4 + 4 * lane;
+    const bool own = lane >= 1 && lane <= 30 && cx < W;
+    double s = 0.0, s2 = 0.0;
+    const int y0 = g * SRADH_RY, y1 = min(y0 + SRADH_RY, H);
+    for (int y = y0; y < y1; ++y) {
+        if (!own || y < r.r1 || y > r.r2) continue;
+        const float4 v = *reinterpret_cast<const float4 *>((const float *)a.src + (size_t)y * (size_t)W + cx);
+        srad_roi_acc(s, s2, v, cx, y, r, own);
+    }
+    srad_roi_store(s, s2, srad_stats_area(a.src, a, 0), g, b, r, lane);
 }

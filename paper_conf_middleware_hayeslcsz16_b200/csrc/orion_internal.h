@@ -66,6 +66,7 @@ struct KernelDef {
     int width_align;        // > 1: the image width must be a multiple of this
     int steps_per_launch;   // stencil steps one launch performs (0 / 1 = one)
     int fanout;             // 1: the kernel's epilogue honours orion_args.fanout (store_out)
+    int srad_stats;         // 1: SRAD with the ROI statistics fused (slots behind src / dst grids)
     int dyn_need() const
     {
         if (smem_bytes > 0) return smem_bytes;

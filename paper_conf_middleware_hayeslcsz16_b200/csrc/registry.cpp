@@ -81,6 +81,9 @@ static const KernelDef kKernels[] = {
     {"srad_f32", 256, "orion_srad4_f32_256", "srad", 32, 8, 124, 256, 2, K_SRAD, 0, 8 * 6 * 132 * 4},
     // srad, halo lanes: 120 x 336 tile, width % 4 == 0; 6-slot ring of 8 warps x 6 x 128 floats
     {"srad_f32h", 256, "orion_srad4h_f32_256", "srad", 32, 8, 120, 8 * 42, 2, K_SRAD, 0, 8 * 6 * 128 * 4, 4},
+    // the same with the ROI statistics fused: q0sqr from the slots behind src, the output ROI's
+    // slots written behind dst (no statistics kernel per iteration; whole grids)
+    {"srad_f32hs", 256, "orion_srad4hs_f32_256", "srad", 32, 8, 120, 8 * 42, 2, K_SRAD, 0, 8 * 6 * 128 * 4, 4, 0, 0, 1},
 };
 
 const KernelDef *find_kernel(const char *id, int threads)

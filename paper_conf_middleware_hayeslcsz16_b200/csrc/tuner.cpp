@@ -413,7 +413,8 @@ orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterat
     if (a->row_begin != 0 || a->row_end != a->height || a->src_row_begin != 0 || a->src_row_end != a->height ||
         a->dst_row_begin != 0 || a->width < 1 || a->height < 1)
         return fail(ORION_E_INVALID, "orion_tune_run_host: whole grids only (rows [0, height))");
-    if (!dev_aux || (!srad && !a->aux) || (srad && !roi))
+    const bool fused = srad && def.srad_stats;   // statistics slots travel behind the grids
+    if ((!dev_aux && !fused) || (!srad && !a->aux) || (srad && !roi))
         return fail(ORION_E_INVALID, "orion_tune_run_host: missing aux / roi");
     const size_t bytes = (size_t)a->width * (size_t)a->height * 4;
     const Driver &D = drv();
@@ -426,14 +427,19 @@ orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterat
         in_bytes += bytes;
     }
     void *cur = dev_a, *nxt = dev_b;
+    if (fused)
+        ORION_TRY(orion_srad_stats_init(t->v->device, cur, a->width, a->height, roi[0], roi[1], roi[2], roi[3],
+                                        stream));
     for (int it = 0; it < iterations; ++it) {
-        if (srad)
+        if (srad && !fused)
             ORION_TRY(orion_srad_roi_stats(t->v->device, cur, a->width, a->height, roi[0], roi[1], roi[2], roi[3],
                                            dev_aux, stream));
         orion_args da = *a;
         da.src = cur;
         da.dst = nxt;
         da.aux = dev_aux;
+        if (fused)
+            for (int i = 0; i < 4; ++i) da.fparam[1 + i] = (float)roi[i];
         ORION_TRY(orion_tune_step(t, &da, stream, nullptr));
         std::swap(cur, nxt);
     }

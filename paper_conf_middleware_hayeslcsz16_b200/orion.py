@@ -29,7 +29,7 @@ SELECT_FASTEST, SELECT_LOWEST_WITHIN_TOL = 0, 1
 
 HALO = {"knn_f4": 3, "knn_f4_p1": 3, "knn_f4_t16": 3, "nlm_f4": 6, "nlm_f4_w": 6, "nlm_f4_direct": 6,
         "nlm_f4_regheavy": 6, "hotspot_f32": 1, "hotspot2h_f32": 2, "hotspot4h_f32": 4, "srad_f32": 2,
-        "srad_f32h": 2, "srad_f32_tile": 2}
+        "srad_f32h": 2, "srad_f32hs": 2, "srad_f32_tile": 2}
 # stencil steps one launch advances (temporal blocking); every other kernel: 1
 STEPS_PER_LAUNCH = {"hotspot2h_f32": 2, "hotspot4h_f32": 4}
 KERNELS = tuple(HALO)
@@ -158,6 +158,7 @@ def lib() -> ctypes.CDLL:
                 "orion_generate_thermal": [I, V, V, I, I, ctypes.c_uint, V],
                 "orion_flush_l2": [I, V, ctypes.c_longlong, V],
                 "orion_srad_roi_stats": [I, V, I, I, I, I, I, I, V, V],
+                "orion_srad_stats_init": [I, V, I, I, I, I, I, I, V],
             }
             for name, args in sig.items():
                 f = getattr(L, name)
@@ -526,12 +527,29 @@ def generate_thermal(device: int, t0: int, power: int, width: int, height: int, 
                                         _s(stream)), "orion_generate_thermal")
 
 
-def srad_args(j_in: int, j_out: int, q0: int, width: int, height: int, lam: float | None = None) -> Args:
-    """Arguments of one "srad_f32" iteration; q0 = device address of the float q0sqr; lam
-    None = liborion's default (orion_default_params)."""
-    a = Args(j_in, j_out, q0, width, height, 0, height, 0, height, 0)
+# "srad_f32hs": floats of ROI statistics slots behind every grid it reads or writes (orion.h)
+SRAD_STATS_FLOATS = 256
+
+
+def srad_args(j_in: int, j_out: int, q0: int, width: int, height: int, lam: float | None = None,
+              roi=None) -> Args:
+    """Arguments of one SRAD iteration.  "srad_f32" / "srad_f32h" / "srad_f32_tile": q0 = device
+    address of the float q0sqr (orion_srad_roi_stats).  "srad_f32hs": q0 unused (0), roi =
+    (r1, r2, c1, c2) -- the statistics travel in the slots behind the grids.  lam None =
+    liborion's default (orion_default_params)."""
+    a = Args(j_in, j_out, q0 or None, width, height, 0, height, 0, height, 0)
     a.fparam[0] = default_params("srad_f32h")[0] if lam is None else lam
+    if roi is not None:
+        for i, v in enumerate(roi):
+            a.fparam[1 + i] = float(v)
     return a
+
+
+def srad_stats_init(device: int, j: int, width: int, height: int, roi, stream=None):
+    """orion_srad_stats_init: the statistics slots of grid j (the first "srad_f32hs" input)."""
+    r1, r2, c1, c2 = roi
+    _check(lib().orion_srad_stats_init(device, ctypes.c_void_p(j), width, height, r1, r2, c1, c2, _s(stream)),
+           "orion_srad_stats_init")
 
 
 def srad_roi_stats(device: int, j: int, width: int, height: int, roi, q0: int, stream=None):

@@ -30,7 +30,8 @@ def _run(kernel, t0, pw, iterations, roi=None):
     v, _ = O.build_all_levels(0, kernel, mode=O.REALISE_MIN_CARVEOUT)
     tuner = O.Tuner(v)
     hs, hout = _pinned(t0), torch.empty((H, W), dtype=torch.float32).pin_memory()
-    da, db = torch.empty((H, W), device="cuda"), torch.empty((H, W), device="cuda")
+    extra = O.SRAD_STATS_FLOATS if kernel == "srad_f32hs" else 0    # statistics slots behind the grids
+    da, db = torch.empty(H * W + extra, device="cuda"), torch.empty(H * W + extra, device="cuda")
     if kernel.startswith("srad"):
         aux = torch.empty(1, device="cuda")
         args = O.srad_args(hs.data_ptr(), hout.data_ptr(), 0, W, H)
@@ -55,11 +56,12 @@ def test_hotspot_run_host_bit_exact(dev, kernel, shape, launches, steps):
     assert h2d == 2 * W * H * 4 and d2h == W * H * 4
 
 
-def test_srad_run_host_vs_oracle(dev):
+@pytest.mark.parametrize("kernel", ["srad_f32", "srad_f32hs"])
+def test_srad_run_host_vs_oracle(dev, kernel):
     W, H = 260, 190
     t0, _ = synth.thermal_inputs(W, H, seed=6)
     roi = (0, 127, 0, 127)
-    out, h2d, d2h, _ = _run("srad_f32", t0, None, 10, roi)
+    out, h2d, d2h, _ = _run(kernel, t0, None, 10, roi)
     ref, _ = oracle.srad(t0.astype(np.float64), 10, 0.5, roi)
     assert np.max(np.abs(out - ref) / np.abs(ref)) < 1e-5
     assert h2d == W * H * 4 and d2h == W * H * 4

@@ -26,13 +26,18 @@ elif lev == "orig":
 else:
     li = int(lev) % len(v)
 if kernel.startswith("srad"):
-    a = torch.empty((H, W), device="cuda")
-    b = torch.empty((H, W), device="cuda")
+    extra = O.SRAD_STATS_FLOATS if kernel == "srad_f32hs" else 0
+    a = torch.empty(H * W + extra, device="cuda")
+    b = torch.empty(H * W + extra, device="cuda")
     p = torch.empty((H, W), device="cuda")
     q0 = torch.empty(1, device="cuda")
     O.generate_thermal(0, a.data_ptr(), p.data_ptr(), W, H, stream=sp)
-    O.srad_roi_stats(0, a.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
-    args = O.srad_args(a.data_ptr(), b.data_ptr(), q0.data_ptr(), W, H)
+    if extra:
+        O.srad_stats_init(0, a.data_ptr(), W, H, (0, 127, 0, 127), sp)
+        args = O.srad_args(a.data_ptr(), b.data_ptr(), 0, W, H, roi=(0, 127, 0, 127))
+    else:
+        O.srad_roi_stats(0, a.data_ptr(), W, H, (0, 127, 0, 127), q0.data_ptr(), sp)
+        args = O.srad_args(a.data_ptr(), b.data_ptr(), q0.data_ptr(), W, H)
 elif kernel.startswith("hotspot"):
     a = torch.empty((H, W), device="cuda")
     b = torch.empty((H, W), device="cuda")
