@@ -25,6 +25,22 @@ using namespace orion;
 
 namespace {
 
+// The ROI of a fused-statistics SRAD launch: fparam[1..4] = r1, r2, c1, c2 (inclusive, exact
+// integers), inside the grid, and few enough (strip, block) slots for the statistics area.
+orion_status check_srad_roi(int W, int H, const float *f, int strip_rows)
+{
+    int v[4];
+    for (int i = 0; i < 4; ++i) {
+        v[i] = (int)f[i];
+        if ((float)v[i] != f[i]) return fail(ORION_E_INVALID, "srad ROI: fparam[1..4] must be integers");
+    }
+    if (v[0] < 0 || v[0] > v[1] || v[1] >= H || v[2] < 0 || v[2] > v[3] || v[3] >= W)
+        return fail(ORION_E_INVALID, "srad ROI outside the grid");
+    const int slots = (v[1] / strip_rows - v[0] / strip_rows + 1) * (v[3] / 120 - v[2] / 120 + 1);
+    if (slots > ORION_SRAD_STAT_SLOTS) return fail(ORION_E_INVALID, "srad ROI spans too many statistics slots");
+    return ORION_OK;
+}
+
 int warps_of(const orion_device_limits &d, int T) { return (T + d.warp_size - 1) / d.warp_size; }
 
 // Translate the public argument block into the kernel's parameter block, checking that
@@ -36,8 +52,13 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
     if (a->width <= 0 || a->height <= 0 || a->row_begin < 0 || a->row_end > a->height || a->row_begin > a->row_end)
         return fail(ORION_E_INVALID, "orion_launch: bad image geometry");
     if (a->row_begin == a->row_end) return ORION_OK;
-    if (!a->src || !a->dst || ((def.kind == K_STENCIL || def.kind == K_SRAD) && !a->aux))
+    if (!a->src || !a->dst || ((def.kind == K_STENCIL || (def.kind == K_SRAD && !def.srad_stats)) && !a->aux))
         return fail(ORION_E_INVALID, "orion_launch: NULL buffer");
+    if (def.srad_stats) {
+        if (a->row_begin != 0 || a->row_end != a->height || a->src_row_begin != 0 || a->dst_row_begin != 0)
+            return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + ": whole grids only");
+        ORION_TRY(check_srad_roi(a->width, a->height, a->fparam + 1, def.tile_h / 8));
+    }
     const int need_lo = std::max(0, a->row_begin - def.halo);
     const int need_hi = std::min(a->height, a->row_end + def.halo);
     if (a->src_row_begin > need_lo || a->src_row_end < need_hi)
@@ -72,6 +93,9 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
         k->fparam[0] = (float)(-noise * 1.4426950408889634);
         k->fparam[1] = a->fparam[1];
         k->fparam[2] = a->fparam[2];
+        // the weight threshold as an exponent (w = 2^e, flushed to 0 below 2^-126)
+        const double wt = a->fparam[2];
+        k->fparam[3] = wt > 0.0 ? (float)std::log2(wt) : (wt == 0.0 ? -126.0f : -INFINITY);
         k->iparam0 = (int)std::floor((double)a->fparam[3] * 49.0) + 1;
     }
     return ORION_OK;
@@ -539,6 +563,35 @@ orion_status orion_flush_l2(int device, void *buf, long long bytes, void *stream
 }
 
 }  // extern "C"
+
+extern "C" orion_status orion_srad_stats_init(int device, void *J, int width, int height, int r1, int r2, int c1,
+                                              int c2, void *stream)
+{
+    if (!J || width <= 0 || height <= 0 || width % 4) return fail(ORION_E_INVALID, "orion_srad_stats_init: bad argument");
+    const KernelDef *def = find_kernel("srad_f32hs", 0);
+    orion_kargs k;
+    std::memset(&k, 0, sizeof k);
+    k.src = J;
+    k.width = width;
+    k.height = height;
+    k.row_end = height;
+    k.src_row_end = height;
+    k.fparam[1] = (float)r1;
+    k.fparam[2] = (float)r2;
+    k.fparam[3] = (float)c1;
+    k.fparam[4] = (float)c2;
+    ORION_TRY(check_srad_roi(width, height, k.fparam + 1, def->tile_h / 8));
+    const int rows = def->tile_h / 8;
+    const int slots = (r2 / rows - r1 / rows + 1) * (c2 / 120 - c1 / 120 + 1);
+    CUmodule m;
+    ORION_TRY(load_aux_module(device, "srad", &m));
+    CUfunction f;
+    ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_srad_stats_init"));
+    void *params[] = {&k};
+    ORION_TRY(launch_maybe_pdl(f, (unsigned)slots, 1, 32, 1, 0, (CUstream)stream, params));
+    g_launches.fetch_add(1);
+    return ORION_OK;
+}
 
 extern "C" orion_status orion_srad_roi_stats(int device, const void *J, int width, int height, int r1, int r2, int c1,
                                              int c2, void *q0, void *stream)
