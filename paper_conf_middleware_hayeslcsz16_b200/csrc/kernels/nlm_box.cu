@@ -170,17 +170,20 @@ struct Acc {
     unsigned cnt[(TH + 3) / 4];   // 4 x 8-bit counts per word (<= 49)
 };
 
-// [w > wthr] into row r's 8-bit count: FSETP + one predicated IADD of an immediate.
-ORION_DEVICE void count_above(Acc &A, int r, float w, float wthr)
+// [w > wthr] into row r's 8-bit count: FSETP + one predicated IADD of an immediate.  Decided on
+// the exponent: w = 2^e > wthr <=> e > log2(wthr) (ethr, host-computed), so the compare does not
+// wait for MUFU.EX2; the two tests differ only within ex2.approx's 2 ulp of the threshold, inside
+// the ambiguous-weight band (reading R-AMB).
+ORION_DEVICE void count_above(Acc &A, int r, float e, float ethr)
 {
-    if (w > wthr) A.cnt[r >> 2] += 1u << (8 * (r & 3));
+    if (e > ethr) A.cnt[r >> 2] += 1u << (8 * (r & 3));
 }
 
 // Phase B for one pair (i, j) whose H_o lives in hb: thread t = output column x0+t.  The
 // +o and -o vertical windows run packed (fp32x2), as do their exponent arguments and the
 // (r, g) / (b, weight) accumulations.
 ORION_DEVICE void phase_b(const float2 *prg, const float *pb, const float *hb, int t, int i, int j,
-                          float nl2, float wthr, Acc &A)
+                          float nl2, float ethr, Acc &A)
 {
     const float geo = geo_l2_rt(i, j);
     // x: D_o(x, y) = sum_n H_o(x, y+n) -- H column t+3, rows 3 .. TH+8
@@ -200,8 +203,8 @@ ORION_DEVICE void phase_b(const float2 *prg, const float *pb, const float *hb, i
         A.azs[r] = fma2(make_float2(wp, wp), make_float2(pb[pp], 1.0f), A.azs[r]);
         A.axy[r] = fma2(make_float2(wm, wm), prg[pm], A.axy[r]);
         A.azs[r] = fma2(make_float2(wm, wm), make_float2(pb[pm], 1.0f), A.azs[r]);
-        count_above(A, r, wp, wthr);
-        count_above(A, r, wm, wthr);
+        count_above(A, r, e.x, ethr);
+        count_above(A, r, e.y, ethr);
     }
 }
 
@@ -239,6 +242,7 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 
     const float nl2 = a.fparam[0];
     const float wthr = a.fparam[2];
+    const float ethr = a.fparam[3];          // log2(wthr)
     const int t = tid;
     Acc A;
     {
@@ -265,7 +269,7 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
 #pragma unroll 1
             for (int g = 0; g < 3; ++g) {
                 const int ig = vert ? i + g : i, jg = vert ? j1 : j1 + g;
-                phase_b(prg, pb, hs + g * HBUF, t, ig, jg, nl2, wthr, A);
+                phase_b(prg, pb, hs + g * HBUF, t, ig, jg, nl2, ethr, A);
             }
         }
         __syncthreads();

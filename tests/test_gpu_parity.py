@@ -351,3 +351,34 @@ def test_sweep_times_every_level(dev):
     O.generate_rgba(0, src.data_ptr(), W, H, stream=stream())
     ms = v.sweep(O.denoise_args("knn_f4", src.data_ptr(), dst.data_ptr(), W, H), stream(), rounds=3)
     assert len(ms) == len(v) and all(m > 0 for m in ms)
+
+
+@pytest.mark.parametrize("shape", [(1, 1), (5, 300), (300, 5), (33, 17), (129, 24), (128, 23)])
+@pytest.mark.parametrize("kernel", ["nlm_f4_w", "nlm_f4_regheavy"])
+def test_nlm_ragged_and_degenerate(dev, shape, kernel):
+    # degenerate frames (a single pixel, one-pixel-wide strips: every window and patch clamps onto
+    # the edge) and shapes one pixel past / exactly at a tile (128 x 23 for nlm_f4_w)
+    W, H = shape
+    img = synth.noisy_rgba(W, H, seed=11, sigma=0.13)
+    v, _ = variants(kernel)
+    outs = run_denoise(kernel, img, level=0) + run_denoise(kernel, img, level=len(v) - 1)
+    assert np.array_equal(outs[0], outs[1])
+    out, alt, amb = oracle.denoise("nlm", img)
+    check_vs_oracle(outs[0], out, alt, amb)
+
+
+def test_tune_step_empty_band_is_not_an_iteration(dev):
+    W = H = 64
+    v, _ = variants("nlm_f4_w")
+    src = torch.empty((H, W, 4), device="cuda")
+    dst = torch.empty((H, W, 4), device="cuda")
+    O.generate_rgba(0, src.data_ptr(), W, H, stream=stream())
+    t = O.Tuner(v)
+    n0 = O.launch_count()
+    r = t.step(O.denoise_args("nlm_f4_w", src.data_ptr(), dst.data_ptr(), W, H, 10, 10), stream())
+    assert (r.iteration, r.level_idx, r.phase) == (-1, -1, -1) and O.launch_count() == n0
+    assert all(x < 0 for x in t.tried())                   # nothing reached Fig. 9
+    r = t.step(O.denoise_args("nlm_f4_w", src.data_ptr(), dst.data_ptr(), W, H), stream())
+    assert r.iteration == 0 and r.phase == 0               # the first real iteration is iteration 0
+    ms = v.sweep(O.denoise_args("nlm_f4_w", src.data_ptr(), dst.data_ptr(), W, H, 7, 7), stream())
+    assert ms == [0.0] * len(v)                            # an empty sweep times nothing
