@@ -511,11 +511,18 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     step = 0
     explore_ms = []
     ran_levels = []
-    for _ in range(warmup):
+    settle_extra = 0
+    while True:
+        # W warm-up iterations, extended (if need be) until Fig. 9 has set the final kernel: the
+        # timed region measures the settled loop; exploration is charged in fig11's Orion-Select
+        if step >= warmup and (tuner.final()[0] >= 0 or settle_extra >= 500):
+            break
         r = tuner.step(step_args(step), sp)
         ran_levels.append(r.level_idx)
         if r.phase == 0 and r.ms >= 0:
             explore_ms.append(r.ms)
+        if step >= warmup:
+            settle_extra += 1
         step += 1
     torch.cuda.synchronize()
     if world > 1:
@@ -645,7 +652,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
             cpu = cpu_baseline(kernel, wl, cpu_seconds, all_cores=True)
         # Orion-Select (Fig. 11, P:L747-P:L755) = the tuned run INCLUDING its exploration: every
         # iteration charged the sweep time of the level it ran (one timing method for all bars)
-        horizon = ran_levels + [final] * steps
+        horizon = ran_levels + [final] * steps      # warm-up (incl. any extension) + timed iterations
         select_ms = sum(ms[i] for i in horizon) / len(horizon)
         lvl_rows = [{"k": lv[i].ctas_per_sm, "occ": lv[i].occupancy_permille / 1000, "reg_cap": lv[i].reg_cap,
                      "regs": infos[i].regs, "pad": lv[i].smem_pad_bytes, "carveout_kb": lv[i].carveout_kb,
@@ -677,7 +684,8 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
                       "final_occupancy": lv[final].occupancy_permille / 1000 if final >= 0 else None,
                       "iterations_to_final": iters_to_final, "explore_ms": explore_ms,
                       "explored_k": [lv[i].ctas_per_sm for i in ran_levels[:max(0, iters_to_final)]],
-                      "samples_per_level": args.samples, "async_timing": bool(args.async_timing)},
+                      "samples_per_level": args.samples, "async_timing": bool(args.async_timing),
+                      "warmup_extended_by": settle_extra},
             "sweep": {"rounds": rounds, "n_levels": nlev, "levels": lvl_rows, "best_k": lv[best].ctas_per_sm,
                       "ms_best": ms[best], "worst_k": lv[worst].ctas_per_sm, "ms_worst": ms[worst],
                       "maxocc_k": lv[kmax].ctas_per_sm, "ms_maxocc": ms[kmax],
@@ -904,8 +912,16 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
             ev[1].record(stream)
         stream.wait_stream(comm)
 
-    for _ in range(warmup):
-        one_step()
+    def all_settled():
+        ok = torch.tensor([1 if tuner.final()[0] >= 0 else 0], device=dev)
+        if world > 1:          # every rank runs the same number of steps (the exchange is collective)
+            dist.all_reduce(ok, op=dist.ReduceOp.MIN, group=group)
+        return bool(ok.item())
+
+    done = 0
+    while done < warmup or (done < warmup + 500 and not all_settled()):
+        one_step()                    # warm-up, extended until every rank's Fig. 9 has set its final kernel
+        done += 1
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier(group=group)

@@ -424,3 +424,10 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot4h_f32_256(orion_
     ORION_PROBE(a);
     hotspotS_body<4, HS_ROWS, 9>(a);
 }
+
+// EXPERIMENT (A/B): 128-row strips (half the halo re-reads, the same 0.93 wave efficiency at 8192^2)
+extern "C" __global__ void __launch_bounds__(256) orion_hotspot4h128_f32_256(orion_kargs a)
+{
+    ORION_PROBE(a);
+    hotspotS_body<4, 128, 9>(a);
+}
