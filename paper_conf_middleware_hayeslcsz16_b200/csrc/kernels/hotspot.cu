@@ -298,7 +298,8 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2h_f32_256(orion_
 // P segments by one elected lane, completing on per-slot mbarriers; edge column blocks kept
 // LDGSTS) measured 0.176 vs 0.157 ms per launch (three A/B pairs on one box), and a 12-slot TMA
 // ring 0.218 ms: at this granularity the per-row elect / expect_tx / try_wait / warp-sync cost
-// more than the 2 LDGSTS they replace.  Removed.
+// more than the 2 LDGSTS they replace.  Removed.  128-row strips (half the halo re-reads, the same
+// 0.93 wave efficiency at 8192^2) measured 0.163 vs 0.154 ms (three A/B pairs): not kept.
 #ifndef HS_ROWS
 #define HS_ROWS 64
 #endif
@@ -423,11 +424,4 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot4h_f32_256(orion_
 {
     ORION_PROBE(a);
     hotspotS_body<4, HS_ROWS, 9>(a);
-}
-
-// EXPERIMENT (A/B): 128-row strips (half the halo re-reads, the same 0.93 wave efficiency at 8192^2)
-extern "C" __global__ void __launch_bounds__(256) orion_hotspot4h128_f32_256(orion_kargs a)
-{
-    ORION_PROBE(a);
-    hotspotS_body<4, 128, 9>(a);
 }

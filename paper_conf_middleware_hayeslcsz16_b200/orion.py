@@ -28,10 +28,10 @@ DIR_DECREASING, DIR_INCREASING = -1, 1
 SELECT_FASTEST, SELECT_LOWEST_WITHIN_TOL = 0, 1
 
 HALO = {"knn_f4": 3, "knn_f4_p1": 3, "knn_f4_t16": 3, "nlm_f4": 6, "nlm_f4_w": 6, "nlm_f4_direct": 6,
-        "nlm_f4_regheavy": 6, "hotspot_f32": 1, "hotspot2h_f32": 2, "hotspot4h_f32": 4, "hotspot4h128_f32": 4, "srad_f32": 2,
+        "nlm_f4_regheavy": 6, "hotspot_f32": 1, "hotspot2h_f32": 2, "hotspot4h_f32": 4, "srad_f32": 2,
         "srad_f32h": 2, "srad_f32hs": 2, "srad_f32_tile": 2}
 # stencil steps one launch advances (temporal blocking); every other kernel: 1
-STEPS_PER_LAUNCH = {"hotspot2h_f32": 2, "hotspot4h_f32": 4, "hotspot4h128_f32": 4}
+STEPS_PER_LAUNCH = {"hotspot2h_f32": 2, "hotspot4h_f32": 4}
 KERNELS = tuple(HALO)
 
 
