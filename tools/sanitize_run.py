@@ -1,7 +1,7 @@
 """Small launches of every kernel family for compute-sanitizer (memcheck / racecheck /
 synccheck; SURVEY §4 layer 3 and §5): C1-sized images, ragged edges, every level of each
-kernel once, the SRAD statistics kernel, the generators, the fan-out epilogue and the
-hotspot / SRAD cp.async rings.  Usage: compute-sanitizer --tool T python tools/sanitize_run.py"""
+kernel once, the SRAD statistics kernels (separate and fused), the generators, the fan-out
+epilogue, row bands read from exactly-sized slabs, and the hotspot / SRAD cp.async rings.  Usage: compute-sanitizer --tool T python tools/sanitize_run.py"""
 import os
 import sys
 
@@ -26,7 +26,19 @@ for k in ("knn_f4", "knn_f4_p1", "knn_f4_t16", "nlm_f4", "nlm_f4_w", "nlm_f4_dir
         v.launch(i, a, sp)
     torch.cuda.synchronize()
     print("ok", k, flush=True)
-WT, HT = 132, 37                                  # width % 4 == 0 for hotspot2; srad takes any width
+# row bands read from exactly-sized input slabs (a band height that is not a multiple of the tile
+# height must not read past the slab: the C5 shard launch shape)
+for k, halo in (("nlm_f4_w", 6), ("nlm_f4", 6), ("knn_f4", 3), ("knn_f4_t16", 3), ("nlm_f4_regheavy", 6)):
+    v, _ = O.build_all_levels(0, k)
+    r0, r1 = 10, 33
+    s0, s1 = r0 - halo, r1 + halo
+    slab = torch.empty((s1 - s0, W, 4), device="cuda")
+    O.generate_rgba(0, slab.data_ptr(), W, H, s0, s1, sigma=0.13, stream=sp)
+    band = torch.empty((r1 - r0, W, 4), device="cuda")
+    v.launch(len(v) - 1, O.denoise_args(k, slab.data_ptr(), band.data_ptr(), W, H, r0, r1, s0, s1, r0), sp)
+    torch.cuda.synchronize()
+    print("ok band", k, flush=True)
+WT, HT = 132, 37                                  # width % 4 == 0 for the float4 strips; srad takes any width
 t0 = torch.empty((HT, WT), device="cuda")
 pw = torch.empty_like(t0)
 t1 = torch.empty_like(t0)
@@ -44,4 +56,16 @@ for k in ("hotspot_f32", "hotspot2h_f32", "hotspot4h_f32", "srad_f32", "srad_f32
             v.launch(i, a, sp)
     torch.cuda.synchronize()
     print("ok", k, flush=True)
+# SRAD with fused statistics: grids carry their statistics slots; the ROI spans two blocks
+fa = torch.zeros(HT * 252 + O.SRAD_STATS_FLOATS, device="cuda")
+fb = torch.zeros_like(fa)
+O.generate_thermal(0, fa.data_ptr(), pw.data_ptr(), 252, HT, stream=sp)
+roi = (2, 30, 100, 140)
+O.srad_stats_init(0, fa.data_ptr(), 252, HT, roi, sp)
+v, _ = O.build_all_levels(0, "srad_f32hs")
+for i in (0, len(v) - 1):
+    v.launch(i, O.srad_args(fa.data_ptr(), fb.data_ptr(), 0, 252, HT, roi=roi), sp)
+    fa, fb = fb, fa
+torch.cuda.synchronize()
+print("ok srad_f32hs", flush=True)
 print("sanitize run complete")
