@@ -192,6 +192,11 @@ def spawn(n: int, argv: list[str]) -> int:
     return subprocess.run(spawn_command(n, argv, free_port()), env=env).returncode
 
 
+def dist_initialized() -> bool:
+    import torch.distributed as dist
+    return dist.is_available() and dist.is_initialized()
+
+
 def backend_name() -> str:
     """ORION_BENCH_BACKEND=gloo only exists to exercise the multi-rank control flow on one GPU
     (ranks then share device local % device_count) or on CPU (--plumbing-check)."""
@@ -859,7 +864,9 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
     tuner = O.Tuner(variants, O.default_cfg(samples_per_level=args.samples))
     # the exchange: the kernels' fan-out stores into every rank's symmetric-memory image (compute
     # + gather in one kernel over NVLink), else chunked all-gathers overlapped with compute
-    mode, fan, fan_note = ("none" if world == 1 else mode_req), None, None
+    # P = 1: no exchange, unless the fan-out is requested explicitly (the symmetric-memory path
+    # exercised on one GPU over a one-rank NCCL group, see run_single)
+    mode, fan, fan_note = ("none" if world == 1 and mode_req != "fanout" else mode_req), None, None
     full = None
     if mode in ("auto", "fanout"):
         try:
@@ -990,7 +997,8 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
                        "collective": ("kernel fan-out stores into every rank's symmetric-memory image over NVLink "
                                       "+ device barrier" if mode == "fanout" else
                                       f"all_gather of {chunks} row chunks on a side stream, overlapped with the "
-                                      f"next chunk's kernel" if mode == "gather" else "none (P=1)"),
+                                      f"next chunk's kernel" if mode == "gather" else "none (P=1)")
+                       if world > 1 or mode == "fanout" else "none (P=1)",
                        "collective_note": fan_note, "l2": "4 GiB frame >> L2",
                        "parallelism": f"row-sharded x{world}", "backend": backend_name() if world > 1 else None},
             "compute_only": {"value": H * W * steps / (comp * 1e-3) / 1e6, "unit": "Mpix/s",
@@ -1028,6 +1036,11 @@ def run_single(args):
     wl = WORKLOADS[key]
     steps = args.steps or wl["steps"]
     if key == "c5":
+        if args.c5_mode == "fanout" and not dist_initialized():
+            # a one-rank NCCL group: the symmetric-memory fan-out path on one GPU
+            import torch.distributed as dist
+            dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{free_port()}", world_size=1, rank=0,
+                                    device_id=torch.device("cuda", local))
         line = measure_c5(args, world=1, rank=0, local=local, steps=steps, warmup=args.warmup, size=args.size,
                           mode_req=args.c5_mode, chunks_req=args.c5_chunks)
         print(json.dumps(line), flush=True)
