@@ -882,7 +882,7 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
     if mode == "gather":
         full = torch.empty((world * b.rows_per_rank, W, 4), device=dev)
     chunks = max(1, chunks_req) if mode == "gather" else 1
-    per = -(-b.rows // chunks) if b.rows else 0
+    plan = shard.chunk_plan(b, chunks)     # the same gathered rows on every rank
     comm = torch.cuda.Stream() if mode == "gather" else None
 
     def one_step(ev=None, recorded=None):
@@ -898,14 +898,11 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
             if ev is not None:
                 ev[1].record(stream)
             return
-        for c in range(chunks):
-            r0, r1 = min(b.rows, c * per), min(b.rows, (c + 1) * per)
-            if r0 >= r1:
-                continue
-            ca = O.denoise_args(kernel, src.data_ptr(), out.data_ptr(), W, H, b.row_begin + r0, b.row_begin + r1,
+        for r0, r1, k0, k1 in plan:
+            ca = O.denoise_args(kernel, src.data_ptr(), out.data_ptr(), W, H, b.row_begin + k0, b.row_begin + k1,
                                 b.src_begin, b.src_end, b.row_begin)
             ce = None
-            if recorded is not None:
+            if recorded is not None and k0 < k1:
                 ce = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                 ce[0].record(stream)
             tuner.step(ca, sp)
@@ -1132,7 +1129,11 @@ def run_plumbing_check(args):
     full = torch.empty((world * b.rows_per_rank, W, 4))
     t0 = time.perf_counter()
     if world > 1:
-        shard.gather_bands(out, full)
+        if args.c5_chunks > 1:   # the chunked gather of the C5 measurement (uneven last band included)
+            for r0, r1, _, _ in shard.chunk_plan(b, args.c5_chunks):
+                shard.gather_rows(out, full, b.rows_per_rank, r0, r1)
+        else:
+            shard.gather_bands(out, full)
     else:
         full = out
     dt = torch.tensor([time.perf_counter() - t0 + rank * 1e-3])

@@ -53,6 +53,20 @@ def band(rank: int, world: int, height: int, halo: int) -> Band:
     return Band(rank, world, height, per, r0, r1, max(0, r0 - halo), min(height, r1 + halo))
 
 
+def chunk_plan(b: Band, chunks: int):
+    """Row chunks of a band for the overlapped gather: [(r0, r1, k0, k1)] with [r0, r1) the band-relative
+    rows EVERY rank gathers (cut from the equal band height, so the collectives match across ranks
+    even when the last band is shorter) and [k0, k1) the rows of the image inside it (empty for the
+    last rank's padding rows)."""
+    per = -(-b.rows_per_rank // max(1, chunks))
+    plan = []
+    for c in range(max(1, chunks)):
+        r0, r1 = min(b.rows_per_rank, c * per), min(b.rows_per_rank, (c + 1) * per)
+        if r0 < r1:
+            plan.append((r0, r1, min(b.rows, r0), min(b.rows, r1)))
+    return plan
+
+
 def gather_rows(out_band, full_out, rows_per_rank: int, r0: int, r1: int, group=None):
     """all_gather rows [r0, r1) of every rank's band straight into their places in
     `full_out` (rank k's rows land at k * rows_per_rank + [r0, r1)).  Issue it on a side

@@ -47,8 +47,8 @@ def test_spawn_command_is_one_process_per_gpu(bench):
     assert cmd[-3:] == [os.path.join(ROOT, "bench.py"), "--steps", "3"]
 
 
-@pytest.mark.parametrize("n,height", [(2, 37), (3, 20), (1, 9)])
-def test_gpus_flag_spawns_ranks_gloo_plumbing(n, height):
+@pytest.mark.parametrize("n,height,chunks", [(2, 37, 1), (3, 20, 1), (1, 9, 1), (3, 37, 4), (2, 37, 3)])
+def test_gpus_flag_spawns_ranks_gloo_plumbing(n, height, chunks):
     # `bench.py --gpus N` without torchrun re-launches itself on N ranks; the plumbing check
     # (CPU, gloo: bands + halos, gather, max over ranks; the kernel replaced by a copy) must
     # print exactly ONE JSON line, from rank 0, with n_gpus = N and the gathered image intact.
@@ -58,7 +58,8 @@ def test_gpus_flag_spawns_ranks_gloo_plumbing(n, height):
     env = dict(os.environ, ORION_BENCH_BACKEND="gloo", OMP_NUM_THREADS="1")
     env.pop("WORLD_SIZE", None)
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", str(n), "--plumbing-check",
-                        "--size", str(height)], capture_output=True, text=True, env=env, timeout=300, cwd=ROOT)
+                        "--size", str(height), "--c5-chunks", str(chunks)], capture_output=True, text=True, env=env,
+                       timeout=300, cwd=ROOT)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, r.stdout

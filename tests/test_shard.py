@@ -104,3 +104,15 @@ def test_chunked_gather_places_rows(world, H, chunks):
         p.join(timeout=300)
         assert p.exitcode == 0
     assert np.array_equal(got, np.repeat(np.arange(H, dtype=np.float32)[:, None], 5, axis=1))
+
+
+@pytest.mark.parametrize("H,P,chunks", [(4096, 3, 4), (37, 3, 4), (16384, 8, 4), (5, 4, 3), (100, 7, 2)])
+def test_chunk_plan_is_the_same_on_every_rank(H, P, chunks):
+    # the gathered rows [r0, r1) must not depend on the rank (collectives match), and the image rows
+    # [k0, k1) of the chunks tile each band exactly
+    plans = [shard.chunk_plan(shard.band(r, P, H, 6), chunks) for r in range(P)]
+    assert all([(p[0], p[1]) for p in pl] == [(p[0], p[1]) for p in plans[0]] for pl in plans)
+    for r, pl in enumerate(plans):
+        b = shard.band(r, P, H, 6)
+        rows = [k for _, _, k0, k1 in pl for k in range(k0, k1)]
+        assert rows == list(range(b.rows))
