@@ -1021,6 +1021,184 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
     return rec
 
 
+# ---- C3 row-sharded: the thermal stencil with a halo exchange per launch ------------------------
+def measure_c3_sharded(args, *, world: int, rank: int, local: int, steps: int, warmup: int, group=None,
+                       size: int = 0, e2e: bool = True):
+    """The 8192^2 thermal stencil row-sharded over the `world` ranks (strong scaling; SURVEY 8(e)'s
+    NEXT item): each rank runs its tuner on its band (+ 4 halo rows per side) with `hotspot4h_f32`,
+    whose launches store their first / last 4 rows into the neighbours' next slabs (symmetric memory
+    over NVLink; fallback: an all-gather of the boundary rows); one device barrier per launch.
+    A step = one 4-step launch on every rank + the exchange."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_middleware_hayeslcsz16_b200 import orion as O
+    from paper_conf_middleware_hayeslcsz16_b200 import shard
+
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    sp = stream.cuda_stream
+    wl = WORKLOADS["c3"]
+    kernel = "hotspot4h_f32"
+    S = O.STEPS_PER_LAUNCH[kernel]
+    W = H = size or wl["W"]
+    bands = [shard.band(r, world, H, S) for r in range(world)]
+    b = bands[rank]
+    if world > 1 and min(x.rows for x in bands if x.rows) < S:
+        raise SystemExit("bench.py: C3 bands must hold at least 4 rows")
+    rows_max = max(x.src_rows for x in bands)
+    # initial grid and power map: the generator's whole grid, this rank's slab copied out (untimed)
+    full_t = torch.empty((H, W), device=dev)
+    full_p = torch.empty((H, W), device=dev)
+    O.generate_thermal(local, full_t.data_ptr(), full_p.data_ptr(), W, H, seed=1, stream=sp)
+    pw = full_p[b.src_begin:b.src_end].clone()
+    t0_slab = full_t[b.src_begin:b.src_end].clone()
+    del full_t, full_p
+    mode, note, slabs = "none", None, None
+    if world > 1:
+        try:
+            if backend_name() != "nccl":
+                raise RuntimeError("symmetric memory needs the nccl backend")
+            slabs = shard.SymmetricSlabs(rows_max, W, dev, group)
+            bufs = slabs.tensors
+            mode = "fanout"
+        except Exception as ex:
+            mode, note = "gather", f"symmetric memory unavailable ({type(ex).__name__}: {ex}); all-gather of halo rows"
+    if slabs is None:
+        bufs = [torch.empty((rows_max, W), device=dev) for _ in range(2)]
+    bufs[0][:b.src_rows].copy_(t0_slab)
+    variants, res = O.build_all_levels(local, kernel, mode=O.REALISE_MIN_CARVEOUT if args.realise == "min"
+                                       else O.REALISE_MAX_SMEM)
+    nlev = len(variants)
+    up, down = shard.halo_neighbours(rank, world, bands)
+
+    def launch_args(n):
+        cur, nxt = n % 2, (n + 1) % 2
+        a = O.hotspot_args(bufs[cur].data_ptr(), bufs[nxt].data_ptr(), pw.data_ptr(), W, H, b.row_begin, b.row_end,
+                           src_row_begin=b.src_begin, src_row_end=b.src_end, dst_row_begin=b.src_begin)
+        if mode == "fanout":
+            a = O.with_fanout(a, [shard.global_row_ptr(slabs.ptrs[nxt][up], bands[up], W) if up is not None else None,
+                                  shard.global_row_ptr(slabs.ptrs[nxt][down], bands[down], W)
+                                  if down is not None else None])
+        return a
+
+    ms = variants.sweep(launch_args(0), sp, rounds=max(3, args.rounds // 3))
+    # the sweep wrote slab 1 from slab 0 (and, in fan-out mode, halo rows of the neighbours' slab 1):
+    # restart from the initial grid
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier(group=group)
+    bufs[0][:b.src_rows].copy_(t0_slab)
+    tuner = O.Tuner(variants, O.default_cfg(samples_per_level=args.samples))
+    n = 0
+
+    def one_step(ev=None):
+        nonlocal n
+        tuner.step(launch_args(n), sp)
+        if ev is not None:
+            ev[1].record(stream)
+        if mode == "fanout":
+            slabs.barrier()                  # every rank's halo stores have landed
+        elif mode == "gather":
+            shard.exchange_halos_gather(bufs[(n + 1) % 2][:b.src_rows], b, bands, S, group)
+        n += 1
+
+    def all_settled():
+        ok = torch.tensor([1 if tuner.final()[0] >= 0 else 0], device=dev)
+        if world > 1:
+            dist.all_reduce(ok, op=dist.ReduceOp.MIN, group=group)
+        return bool(ok.item())
+
+    done = 0
+    while done < warmup or (done < warmup + 500 and not all_settled()):
+        one_step()
+        done += 1
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier(group=group)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+           torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    n0 = O.launch_count()
+    with ClockSampler(local) as clk:
+        for e in ev:
+            e[0].record(stream)
+            one_step(e)
+            e[2].record(stream)
+        torch.cuda.synchronize()
+        clk.mark_end()
+    launches = O.launch_count() - n0
+    tot = ev[0][0].elapsed_time(ev[-1][2])
+    comp = sum(e0.elapsed_time(e1) for e0, e1, _ in ev)
+    exch = sum(e1.elapsed_time(e2) for _, e1, e2 in ev)
+    # ---- end to end: pinned host slabs (T0 + P) -> device, 25 launches = 100 steps, band -> host ----
+    e2e_dt = 0.0
+    h2d = d2h = 0
+    n_e2e = 100 // S
+    if e2e:
+        h_t = t0_slab.cpu().pin_memory()
+        h_p = pw.cpu().pin_memory()
+        h_o = torch.empty((b.rows, W), pin_memory=True)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier(group=group)
+        t0 = time.perf_counter()
+        n = 0
+        bufs[0][:b.src_rows].copy_(h_t, non_blocking=True)
+        pw.copy_(h_p, non_blocking=True)
+        for _ in range(n_e2e):
+            one_step()
+        h_o.copy_(bufs[n % 2][b.row_begin - b.src_begin:b.row_end - b.src_begin], non_blocking=True)
+        torch.cuda.synchronize()
+        e2e_dt = time.perf_counter() - t0
+        h2d, d2h = 2 * b.src_rows * W * 4, b.rows * W * 4
+    t = torch.tensor([tot, comp, exch, e2e_dt], device=dev)
+    byts = torch.tensor([float(h2d), float(d2h)], device=dev, dtype=torch.float64)
+    final, it = tuner.final()
+    chosen = [variants.level(final).ctas_per_sm if final >= 0 else -1, it,
+              variants.level(min(range(nlev), key=lambda k: ms[k])).ctas_per_sm, b.row_begin, b.row_end]
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+        dist.all_reduce(byts, op=dist.ReduceOp.SUM, group=group)
+        allc = [None] * world
+        dist.all_gather_object(allc, chosen, group=group)
+    else:
+        allc = [chosen]
+    tot, comp, exch, e2e_dt = (float(x) for x in t.tolist())
+    rec = None
+    if rank == 0:
+        units = H * W * S
+        rec = {
+            "metric": METRIC, "value": units * steps / (tot * 1e-3) / 1e6, "unit": "Mcell-steps/s",
+            "n_gpus": world, "steps": steps, "warmup": warmup, "ms_per_step": tot / steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "thermal stencil 8192x8192 fp32 row-sharded, halo exchange per 4-step launch",
+                       "baseline_config_index": 2, "kernel": kernel, "width": W, "height": H,
+                       "rows_per_rank": b.rows_per_rank, "halo_rows": S,
+                       "exchange": ("kernel stores of the first / last 4 rows into the neighbours' symmetric-memory "
+                                    "slabs over NVLink + device barrier" if mode == "fanout" else
+                                    "all_gather of the boundary rows" if mode == "gather" else "none (P=1)"),
+                       "exchange_note": note, "parallelism": f"row-sharded x{world}",
+                       "backend": backend_name() if world > 1 else None, "l2": "grids (3 x 256 MiB / P) vs L2"},
+            "compute_only": {"value": units * steps / (comp * 1e-3) / 1e6, "unit": "Mcell-steps/s",
+                             "ms_per_step": comp / steps},
+            "exchange_ms_per_step": exch / steps,
+            "per_rank": [{"rank": r, "final_k": c[0], "iterations_to_final": c[1], "sweep_best_k": c[2],
+                          "rows": [c[3], c[4]]} for r, c in enumerate(allc)],
+            "sweep_rank0": [{"k": variants.level(i).ctas_per_sm, "ms": round(ms[i], 4)} for i in range(nlev)],
+            "gpu_launches": launches, "clocks": clk.summary(), "energy": clk.energy(steps),
+            "e2e": ({"value": units * n_e2e / e2e_dt / 1e6, "unit": "Mcell-steps/s",
+                     "h2d_bytes_per_step": float(byts[0]) / n_e2e, "d2h_bytes_per_step": float(byts[1]) / n_e2e,
+                     "steps": n_e2e, "api": "per rank: pinned host T0 + P slabs -> device, 25 tuned launches "
+                                            "(100 steps) with the halo exchange, own band -> pinned host"}
+                    if e2e else None),
+            "cpu_baseline": None,
+        }
+    tuner.close()
+    variants.close()
+    del bufs, slabs
+    torch.cuda.empty_cache()
+    return rec
+
+
 # ---- drivers ------------------------------------------------------------------------------------
 def run_single(args):
     """N = 1: the headline configuration and (unless --only) every other one as a sub-record."""
@@ -1088,19 +1266,22 @@ def run_multi(args):
     if args.gpus and args.gpus != world:
         raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}")
     local = init_dist(world, local)
-    steps = args.steps or WORKLOADS["c5"]["steps"]
+    if args.workload == "c3":      # the stencil row-sharded with a halo exchange per launch
+        measure, key, extra = measure_c3_sharded, "c3", {}
+    else:                          # C5: the NLM frame row-sharded + the output exchange
+        measure, key, extra = measure_c5, "c5", {"mode_req": args.c5_mode, "chunks_req": args.c5_chunks}
+    steps = args.steps or WORKLOADS[key]["steps"]
     anchor = None
     if not args.no_anchor:
         if rank == 0:
-            anchor = measure_c5(args, world=1, rank=0, local=local, steps=steps, warmup=3, size=args.size,
-                                e2e=False)
+            anchor = measure(args, world=1, rank=0, local=local, steps=steps, warmup=3, size=args.size, e2e=False)
         dist.barrier()
-    line = measure_c5(args, world=world, rank=rank, local=local, steps=steps, warmup=args.warmup, size=args.size,
-                      mode_req=args.c5_mode, chunks_req=args.c5_chunks)
+    line = measure(args, world=world, rank=rank, local=local, steps=steps, warmup=args.warmup, size=args.size,
+                   **extra)
     if rank == 0:
         if anchor is not None:
-            line["c5_p1_anchor"] = {k: anchor[k] for k in ("value", "ms_per_step", "compute_only", "per_rank",
-                                                           "roofline", "clocks")}
+            line[f"{key}_p1_anchor"] = {k: anchor[k] for k in ("value", "ms_per_step", "compute_only", "per_rank",
+                                                                "clocks")}
             line["speedup_vs_p1"] = line["value"] / anchor["value"]
         print(json.dumps(line), flush=True)
     dist.barrier()

@@ -200,9 +200,16 @@ void orion_variants_destroy(orion_variants *v);
  *             window taps), as in the SDK imageDenoising sample (reading R-O2).
  *  hotspot:   src = T (float), aux = power (same rows as src), dst = T'; fparam[0..4] =
  *             sdc (step/Cap), rx = 1/Rx, ry = 1/Ry, rz = 1/Rz, amb (reading R-O3/R-A15).
- *             src must hold rows row_begin-1 .. row_end (clamped).
+ *             src must hold rows row_begin-S .. row_end+S-1 (clamped; S = steps per launch).
+ *  halo exchange ("hotspot4h_f32", n_fanout = 2): a launch on a row band [row_begin, row_end)
+ *             of a row-sharded grid also stores its first 4 and last 4 output rows -- the rows the
+ *             neighbouring bands' next 4-step launch reads as halo -- into fanout[0] (upper
+ *             neighbour) and fanout[1] (lower neighbour): device pointers such that global row y
+ *             lands at fanout[f] + y * width (the neighbour's next input buffer, its own memory or
+ *             a peer's over NVLink); NULL at the grid's top / bottom edge.  n_fanout other than 0
+ *             or 2 -> ORION_E_INVALID.
  *  fan-out (every box-sum NLM kernel "nlm_f4*" except "nlm_f4_direct", every KNN kernel
- *             "knn_f4*"; not the stencils or "nlm_f4_regheavy"): every output
+ *             "knn_f4*"; not "nlm_f4_regheavy"): every output
  *             pixel is also stored into fanout[0 .. n_fanout) -- full width x height images
  *             (global row y at y * width), device pointers in this GPU's memory or a peer's
  *             reachable over NVLink (P2P / symmetric memory) -- so a row-sharded frame is

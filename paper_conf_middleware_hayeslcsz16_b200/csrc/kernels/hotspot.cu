@@ -402,6 +402,21 @@ __device__ __forceinline__ void hotspotS_strip(const orion_kargs &a, int ys, int
 #pragma unroll 1
     for (; q < nq; ++q) row(q, q % NB, S);
     cp_async_wait<0>();
+    if (a.nfan) {
+        // halo exchange of a row-sharded grid (off the hot loop): the band's first S and last S output
+        // rows -- the halos the neighbouring bands' next launch reads -- go from dst (written above
+        // by this same lane) into fan[0] / fan[1] (the upper / lower neighbour's next input, global
+        // row y at y * W; NULL at the grid's edge), over NVLink when those are peer buffers
+        const float *ob = (const float *)a.dst + (size_t)cx - (size_t)a.dst_row_begin * (size_t)W;
+        if (writer && a.fan[0])
+            for (int y = max(ys, a.row_begin); y < min(ye, a.row_begin + S); ++y)
+                *reinterpret_cast<float4 *>((float *)a.fan[0] + (size_t)y * (size_t)W + cx) =
+                    *reinterpret_cast<const float4 *>(ob + (size_t)y * (size_t)W);
+        if (writer && a.fan[1])
+            for (int y = max(ys, a.row_end - S); y < ye; ++y)
+                *reinterpret_cast<float4 *>((float *)a.fan[1] + (size_t)y * (size_t)W + cx) =
+                    *reinterpret_cast<const float4 *>(ob + (size_t)y * (size_t)W);
+    }
 }
 
 template <int S, int RY, int NB>

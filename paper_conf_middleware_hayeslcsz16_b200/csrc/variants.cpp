@@ -69,8 +69,14 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
                                          std::to_string(def.width_align) + " == 0");
     if (a->n_fanout < 0 || a->n_fanout > 8 || (a->n_fanout > 0 && !def.fanout))
         return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + ": bad n_fanout");
-    for (int f = 0; f < a->n_fanout; ++f)
-        if (!a->fanout[f]) return fail(ORION_E_INVALID, "orion_launch: NULL fanout buffer");
+    if (def.kind == K_STENCIL) {
+        // the halo exchange: exactly (upper, lower) neighbour buffers, NULL at the grid's edge
+        if (a->n_fanout != 0 && a->n_fanout != 2)
+            return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + ": n_fanout must be 0 or 2");
+    } else {
+        for (int f = 0; f < a->n_fanout; ++f)
+            if (!a->fanout[f]) return fail(ORION_E_INVALID, "orion_launch: NULL fanout buffer");
+    }
     for (int f = 0; f < a->n_fanout; ++f) k->fan[f] = a->fanout[f];
     k->nfan = a->n_fanout;
     k->src = a->src;

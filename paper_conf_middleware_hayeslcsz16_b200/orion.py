@@ -261,9 +261,13 @@ def default_params(kernel_id: str) -> tuple:
 
 
 def hotspot_args(t_in: int, t_out: int, power: int, width: int, height: int, row_begin: int = 0,
-                 row_end: int | None = None, consts=None) -> Args:
+                 row_end: int | None = None, consts=None, src_row_begin: int = 0, src_row_end: int | None = None,
+                 dst_row_begin: int = 0) -> Args:
+    """Arguments of one thermal-stencil launch.  Whole grid by default; a row band of a sharded
+    grid: t_in / power hold global rows [src_row_begin, src_row_end), t_out from dst_row_begin."""
     row_end = height if row_end is None else row_end
-    a = Args(t_in, t_out, power, width, height, row_begin, row_end, 0, height, 0)
+    src_row_end = height if src_row_end is None else src_row_end
+    a = Args(t_in, t_out, power, width, height, row_begin, row_end, src_row_begin, src_row_end, dst_row_begin)
     for i, x in enumerate(consts or default_params("hotspot_f32")[:5]):
         a.fparam[i] = x
     return a

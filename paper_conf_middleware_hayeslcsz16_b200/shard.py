@@ -119,3 +119,69 @@ class FanoutImage:
 
     def barrier(self):
         self.handle.barrier()
+
+
+# ---- the thermal stencil row-sharded with a per-launch halo exchange ------------------------------
+# Each rank holds its band of a W x H grid plus `halo` rows per side (two such slabs, ping-pong) and
+# the same slab of the power map.  A launch advancing `halo` steps writes the band into its next
+# slab and, through orion_args.fanout, its first / last `halo` rows into the neighbours' next slabs
+# (the kernel's halo exchange); one device barrier per launch orders those stores before any rank
+# reads them.  Host-side logic only: pointer arithmetic and the fallback exchange.
+
+def halo_neighbours(rank: int, world: int, bands):
+    """(upper, lower) neighbour ranks whose next slabs receive this band's first / last rows, or
+    None at the grid's edge (or when the neighbour's band is empty)."""
+    up = rank - 1 if rank > 0 and bands[rank - 1].rows else None
+    down = rank + 1 if rank + 1 < world and bands[rank + 1].rows else None
+    return up, down
+
+
+def global_row_ptr(base_ptr: int, b: Band, width: int, elem: int = 4) -> int:
+    """Address such that global row y of the slab starting at b.src_begin sits at ptr + y * width."""
+    return base_ptr - b.src_begin * width * elem
+
+
+def exchange_halos_gather(nxt, b: Band, bands, halo: int, group=None):
+    """Fallback halo exchange (no symmetric memory, e.g. gloo): every rank contributes its band's
+    first and last `halo` rows of `nxt` (a (b.src_rows, W) slab), all ranks gather them, and each
+    copies its neighbours' rows into its own halo rows -- the same rows the kernel's fan-out stores."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    W = nxt.shape[1]
+    mine = torch.zeros((2, halo, W), dtype=nxt.dtype, device=nxt.device)
+    if b.rows:
+        o = b.row_begin - b.src_begin
+        mine[0] = nxt[o:o + halo]
+        mine[1] = nxt[o + b.rows - halo:o + b.rows]
+    host = nxt.is_cuda and dist.get_backend(group) != "nccl"
+    src = mine.cpu() if host else mine
+    allr = [torch.empty_like(src) for _ in range(world)]
+    dist.all_gather(allr, src, group=group)
+    up, down = halo_neighbours(rank, world, bands)
+    if up is not None:           # rows [row_begin - halo, row_begin): the upper band's last rows
+        nxt[b.row_begin - halo - b.src_begin:b.row_begin - b.src_begin] = allr[up][1].to(nxt.device)
+    if down is not None:         # rows [row_end, row_end + halo): the lower band's first rows
+        nxt[b.row_end - b.src_begin:b.row_end + halo - b.src_begin] = allr[down][0].to(nxt.device)
+    return nxt
+
+
+class SymmetricSlabs:
+    """Two (rows x W) float32 slabs per rank in symmetric memory (every rank's addresses known):
+    the ping-pong grids of a row-sharded stencil whose kernels store halo rows into peers."""
+
+    def __init__(self, rows: int, width: int, device, group=None):
+        import torch
+        import torch.distributed as dist
+        import torch.distributed._symmetric_memory as symm_mem
+        self.tensors, self.handles, self.ptrs = [], [], []
+        for _ in range(2):
+            t = symm_mem.empty(rows, width, dtype=torch.float32, device=device)
+            h = symm_mem.rendezvous(t, group or dist.group.WORLD)
+            self.tensors.append(t)
+            self.handles.append(h)
+            self.ptrs.append([int(p) for p in h.buffer_ptrs])
+
+    def barrier(self):
+        self.handles[0].barrier()

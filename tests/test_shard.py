@@ -116,3 +116,48 @@ def test_chunk_plan_is_the_same_on_every_rank(H, P, chunks):
         b = shard.band(r, P, H, 6)
         rows = [k for _, _, k0, k1 in pl for k in range(k0, k1)]
         assert rows == list(range(b.rows))
+
+
+def _halo_worker(rank, world, port, H, W, halo, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    bands = [shard.band(r, world, H, halo) for r in range(world)]
+    b = bands[rank]
+    # this rank's next slab: its band rows hold the global row index, the halo rows -1 (not exchanged yet)
+    nxt = torch.full((b.src_rows, W), -1.0)
+    nxt[b.row_begin - b.src_begin:b.row_end - b.src_begin] = \
+        torch.arange(b.row_begin, b.row_end, dtype=torch.float32)[:, None] + torch.zeros(W)
+    shard.exchange_halos_gather(nxt, b, bands, halo)
+    q.put((rank, nxt.numpy()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,H,halo", [(2, 37, 4), (3, 40, 4), (4, 61, 4)])
+def test_stencil_halo_exchange_fallback(world, H, halo):
+    # the all-gather fallback of the C3 halo exchange (the kernels' fan-out stores do the same over
+    # NVLink): after it every slab holds the global rows [src_begin, src_end) -- its neighbours'
+    # boundary rows in its halo
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_halo_worker, args=(r, world, port, H, 6, halo, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = dict(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=300)
+        assert p.exitcode == 0
+    for r in range(world):
+        b = shard.band(r, world, H, halo)
+        want = np.repeat(np.arange(b.src_begin, b.src_end, dtype=np.float32)[:, None], 6, axis=1)
+        assert np.array_equal(got[r], want), r
+
+
+def test_global_row_pointer_and_neighbours():
+    bands = [shard.band(r, 4, 100, 4) for r in range(4)]
+    assert shard.halo_neighbours(0, 4, bands) == (None, 1)
+    assert shard.halo_neighbours(2, 4, bands) == (1, 3)
+    assert shard.halo_neighbours(3, 4, bands) == (2, None)
+    b = bands[2]                      # rows 50..75, slab from row 46
+    assert shard.global_row_ptr(1 << 40, b, 64) + 46 * 64 * 4 == 1 << 40
