@@ -89,3 +89,46 @@ def test_halo_fanout_argument_checks(v):
     a = O.hotspot_args(t.data_ptr(), t.data_ptr(), t.data_ptr(), 64, 16)
     with pytest.raises(O.OrionError):
         v.launch(0, O.with_fanout(a, [t.data_ptr()]), sp)            # the exchange takes (upper, lower)
+
+
+def test_symmetric_slabs_one_rank_nccl(v):
+    # shard.SymmetricSlabs (the C3 multi-GPU slabs) on a one-rank NCCL group: a band launch whose
+    # halo stores target the symmetric slabs' own addresses (as a neighbour's would over NVLink)
+    # leaves the same bits as plain buffers
+    import json
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import json, socket, torch, torch.distributed as dist
+import numpy as np, synth
+from paper_conf_middleware_hayeslcsz16_b200 import orion as O, shard
+s = socket.socket(); s.bind(("127.0.0.1", 0)); port = s.getsockname()[1]; s.close()
+torch.cuda.set_device(0)
+dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", world_size=1, rank=0,
+                        device_id=torch.device("cuda", 0))
+W, H = 256, 96
+t0, pw = synth.thermal_inputs(W, H, seed=3)
+v, _ = O.build_all_levels(0, "hotspot4h_f32")
+sl = shard.SymmetricSlabs(H, W, torch.device("cuda", 0))
+sl.tensors[0].copy_(torch.from_numpy(t0))
+p = torch.from_numpy(pw).cuda()
+b = shard.band(0, 1, H, 4)
+sp = torch.cuda.current_stream().cuda_stream
+for n in range(5):
+    cur, nxt = n % 2, (n + 1) % 2
+    a = O.hotspot_args(sl.tensors[cur].data_ptr(), sl.tensors[nxt].data_ptr(), p.data_ptr(), W, H)
+    # the halo stores of a band [0, H) land on the slab's own rows: a no-op by value
+    a = O.with_fanout(a, [shard.global_row_ptr(sl.ptrs[nxt][0], b, W), shard.global_row_ptr(sl.ptrs[nxt][0], b, W)])
+    v.launch(0, a, sp)
+    sl.barrier()
+torch.cuda.synchronize()
+import oracle
+print(json.dumps({"equal": bool(np.array_equal(sl.tensors[1].cpu().numpy(), oracle.hotspot(t0, pw, 20, precision="f32")))}))
+dist.destroy_process_group()
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600, cwd=root,
+                       env=dict(os.environ, PYTHONPATH=root))
+    assert r.returncode == 0, r.stderr[-3000:]
+    assert json.loads(r.stdout.strip().splitlines()[-1]) == {"equal": True}
