@@ -192,3 +192,14 @@ def test_every_header_entry_cites_its_passage():
         if not re.search(r"P:L|SURVEY|reading|Fig\.|Eq\.", com):
             missing.append(m.group(2))
     assert not missing, missing
+
+
+def test_set_pdl_switch_host_only():
+    prev = O.set_pdl(False)
+    try:
+        assert O.set_pdl(True) is False          # returns the setting it replaces
+        assert O.set_pdl(True) is True
+        import ctypes
+        assert O.lib().orion_set_pdl(2, None) == -1   # ORION_E_INVALID
+    finally:
+        O.set_pdl(prev)
