@@ -70,3 +70,24 @@ def test_gpus_flag_spawns_ranks_gloo_plumbing(n, height, chunks):
         rows = [b[:2] for b in d["bands"]]
         assert rows[0][0] == 0 and rows[-1][1] == height
         assert all(rows[k][1] == rows[k + 1][0] for k in range(n - 1))
+
+
+@pytest.mark.parametrize("gpus", [1, 2])
+def test_reference_arm_runs_the_oracle_on_rank0_only(gpus):
+    # --impl reference: the CPU oracle on a bounded sample of the headline workload, one JSON line
+    # from rank 0 (under --gpus 2 the other rank exits without work), e2e with no copies
+    import json
+    import subprocess
+    import sys
+    env = dict(os.environ, ORION_BENCH_BACKEND="gloo", OMP_NUM_THREADS="1")
+    env.pop("WORLD_SIZE", None)
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", str(gpus),
+                        "--steps", "1", "--warmup", "3"], capture_output=True, text=True, env=env, timeout=600,
+                       cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == gpus and d["value"] > 0
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["value"] == d["value"]
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["d2h_bytes_per_step"] == 0
