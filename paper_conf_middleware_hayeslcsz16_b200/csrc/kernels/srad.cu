@@ -43,9 +43,11 @@ ORION_DEVICE SradCell srad_coeff(float Jc, float N, float S, float Wv, float E, 
     const float g2 = __fmaf_rn(dE, dE, __fmaf_rn(dW, dW, __fmaf_rn(dS, dS, __fmul_rn(dN, dN))));
     const float dnw = __fadd_rn(dN, dW);
     const float sd = __fadd_rn(__fadd_rn(dnw, dS), dE);
-    const float num = __fmaf_rn(__fmul_rn(-0.0625f, sd), sd, __fmul_rn(0.5f, g2));
-    const float den = __fmaf_rn(0.25f, sd, Jc);
-    const float qsqr = __fmul_rn(num, rcp_approx(__fmul_rn(den, den)));
+    // 16*num and 4*den: power-of-two scalings commute with every rounding below, so
+    // qsqr = (16 num) * rcp(16 den^2) is bit-identical to num * rcp(den^2), one FMUL less
+    const float num16 = __fmaf_rn(-sd, sd, __fmul_rn(8.0f, g2));
+    const float den4 = __fmaf_rn(4.0f, Jc, sd);
+    const float qsqr = __fmul_rn(num16, rcp_approx(__fmul_rn(den4, den4)));
     const float c = rcp_approx(__fadd_rn(1.0f, __fmaf_rn(qsqr, iqden, nq)));
     SradCell r;
     r.c = __saturatef(c);
@@ -77,10 +79,10 @@ ORION_DEVICE SradPair srad_coeff2(float2 Jc, float2 N, float2 S, float2 dW, floa
     const float2 g2 = __ffma2_rn(dE, dE, __ffma2_rn(dW, dW, __ffma2_rn(dS, dS, __fmul2_rn(dN, dN))));
     const float2 dnw = __fadd2_rn(dN, dW);
     const float2 sd = __fadd2_rn(__fadd2_rn(dnw, dS), dE);
-    const float2 num = __ffma2_rn(__fmul2_rn(f2(-0.0625f), sd), sd, __fmul2_rn(f2(0.5f), g2));
-    const float2 den = __ffma2_rn(f2(0.25f), sd, Jc);
-    const float2 dd = __fmul2_rn(den, den);
-    const float2 qsqr = __fmul2_rn(num, make_float2(rcp_approx(dd.x), rcp_approx(dd.y)));
+    const float2 num16 = __ffma2_rn(neg(sd), sd, __fmul2_rn(f2(8.0f), g2));   // as srad_coeff
+    const float2 den4 = __ffma2_rn(f2(4.0f), Jc, sd);
+    const float2 dd = __fmul2_rn(den4, den4);
+    const float2 qsqr = __fmul2_rn(num16, make_float2(rcp_approx(dd.x), rcp_approx(dd.y)));
     const float2 t = __fadd2_rn(f2(1.0f), __ffma2_rn(qsqr, f2(iqden), f2(nq)));
     SradPair r;
     r.c = make_float2(__saturatef(rcp_approx(t.x)), __saturatef(rcp_approx(t.y)));
