@@ -7,7 +7,7 @@ OUT=gpurun_out; mkdir -p $OUT
 for i in $(seq 1 $N); do
   for k in "$@"; do
     python bench.py --workload $WL --only --kernel $k --rounds 5 --no-cpu-baseline --no-carveout-axis > $OUT/kab_last.log 2>&1
-    echo "$WL $k $(grep -o '"ms_per_step": [0-9.]*' $OUT/kab_last.log) $(grep -o '"ms_best": [0-9.]*' $OUT/kab_last.log | head -1)" >> $OUT/kernel_ab.txt
+    echo "$WL $k $(grep -o '"value": [0-9.]*' $OUT/kab_last.log | head -1) $(grep -o '"ms_per_step": [0-9.]*' $OUT/kab_last.log) $(grep -o '"ms_best": [0-9.]*' $OUT/kab_last.log | head -1)" >> $OUT/kernel_ab.txt
   done
 done
 cat $OUT/kernel_ab.txt
