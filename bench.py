@@ -480,13 +480,18 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
         for f, t in enumerate(srcs):
             O.generate_rgba(local, t.data_ptr(), W, H, seed=1 + f + 97 * rank, sigma=wl["sigma"], stream=sp)
 
-        def step_args(s):
+        def step_args(s, independent=True):
+            # consecutive frames live in their own buffers (nframes >= 2): each launch is
+            # independent of the stream's previous one (ORION_ARGS_INDEPENDENT), so with PDL a
+            # frame's CTAs start in the previous frame's last wave
             f = s % nframes
-            return O.denoise_args(kernel, srcs[f].data_ptr(), dsts[f].data_ptr(), W, H)
+            return O.denoise_args(kernel, srcs[f].data_ptr(), dsts[f].data_ptr(), W, H,
+                                  independent=independent and nframes > 1)
     torch.cuda.synchronize()
 
     # ---- exhaustive sweep (brute-force reference, Fig. 11 Orion-Max/Min) ------------------
-    sweep_args = step_args(0)
+    # (repeats one frame: not independent launches)
+    sweep_args = step_args(0) if is_stencil else step_args(0, independent=False)
     if is_stencil:
         state["a"], state["b"] = t_a, t_b
         if is_srad and not fused:

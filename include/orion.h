@@ -214,7 +214,18 @@ void orion_variants_destroy(orion_variants *v);
  *             (global row y at y * width), device pointers in this GPU's memory or a peer's
  *             reachable over NVLink (P2P / symmetric memory) -- so a row-sharded frame is
  *             gathered by the kernel's own epilogue as each tile completes (C5).  n_fanout = 0:
- *             no fan-out; > 8, or > 0 for other kernels -> ORION_E_INVALID. */
+ *             no fan-out; > 8, or > 0 for other kernels -> ORION_E_INVALID.
+ *  flags:     0, or ORION_ARGS_INDEPENDENT for a denoiser launch that reads nothing the stream's
+ *             previous kernel writes and writes nothing that kernel reads or writes (e.g. the
+ *             next frame of a stream of frames, each in its own buffers; one band after another
+ *             of orion_tune_split).  With programmatic dependent launch on (orion_set_pdl), the
+ *             kernel then does not wait for its predecessor: its CTAs fill the previous grid's
+ *             last wave (one frame per iteration, P:L605-P:L607, overlapped on the GPU).  The
+ *             caller asserts the independence; the result bits are the same.  Set on a
+ *             stencil / SRAD launch (each reads its predecessor's output), or any other bit ->
+ *             ORION_E_INVALID.  The host-buffer entry points (orion_tune_step_host,
+ *             orion_host_pipe_submit) launch after their own copies and ignore it. */
+#define ORION_ARGS_INDEPENDENT 1
 typedef struct {
     const void *src;
     void *dst;
@@ -226,6 +237,7 @@ typedef struct {
     float fparam[8];
     void *fanout[8];
     int n_fanout;
+    int flags;
 } orion_args;
 
 /* Launch variant `level_idx` (realising its occupancy level, P:L649, P:L757-P:L759) on

@@ -20,9 +20,11 @@ ORION_DEVICE bool orion_probe(const orion_kargs &a)
 {
     // programmatic dependent launch (orion_launch with ORION_PDL=1): let the stream's next grid
     // be scheduled now, and wait here until the previous grid has completed and its memory is
-    // visible -- before any load.  Both are no-ops for a normal launch.
+    // visible -- before any load -- unless the caller asserted the launch independent of it
+    // (ORION_ARGS_INDEPENDENT: the CTAs start in the previous grid's last wave).  Both are no-ops
+    // for a normal launch.
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    asm volatile("griddepcontrol.wait;" ::: "memory");
+    if (!a.nowait) asm volatile("griddepcontrol.wait;" ::: "memory");
     if (a.probe == nullptr) return false;
     if (threadIdx.x == 0 && threadIdx.y == 0) {
         unsigned smid;

@@ -19,6 +19,7 @@ typedef struct {
                                         (orion_probe in kernels/common.cuh)                        */
     void *fan[8];                    /* denoisers: extra full-image outputs (global row y at y*width), */
     int nfan;                        /* e.g. every rank's gather buffer over NVLink peer memory        */
+    int nowait;                      /* 1: ORION_ARGS_INDEPENDENT -- no griddepcontrol.wait (PDL)      */
 } orion_kargs;
 
 #endif

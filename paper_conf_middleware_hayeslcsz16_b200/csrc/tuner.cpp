@@ -392,6 +392,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
     da.src = dev_src;
     da.dst = dev_dst;
     da.aux = dev_aux;
+    da.flags = 0;                  // the launch follows this call's own copies
     ORION_TRY(orion_tune_step(t, &da, stream, out));
     const char *dptr = (const char *)dev_dst + (size_t)(a->row_begin - a->dst_row_begin) * row;
     ORION_CU(D.cuMemcpyDtoHAsync((char *)a->dst + (size_t)(a->row_begin - a->dst_row_begin) * row,
@@ -549,6 +550,7 @@ orion_status orion_host_pipe_submit(orion_host_pipe *p, const orion_args *a, ori
     da.src = (const void *)s.src;
     da.dst = (void *)s.dst;
     da.aux = (const void *)s.aux;
+    da.flags = 0;                  // the launch follows the pipe's copies and event waits
     da.dst_row_begin = a->row_begin;
     ORION_TRY(orion_tune_step(p->t, &da, p->s_comp, out));
     ORION_CU(D.cuEventRecord(s.ev_done, p->s_comp));

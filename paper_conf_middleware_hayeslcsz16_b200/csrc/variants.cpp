@@ -79,6 +79,11 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
     }
     for (int f = 0; f < a->n_fanout; ++f) k->fan[f] = a->fanout[f];
     k->nfan = a->n_fanout;
+    if (a->flags & ~ORION_ARGS_INDEPENDENT) return fail(ORION_E_INVALID, "orion_launch: unknown flags");
+    if ((a->flags & ORION_ARGS_INDEPENDENT) && (def.kind == K_STENCIL || def.kind == K_SRAD))
+        return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id +
+                                         ": a stencil launch reads its predecessor's output (not independent)");
+    k->nowait = (a->flags & ORION_ARGS_INDEPENDENT) ? 1 : 0;
     k->src = a->src;
     k->dst = a->dst;
     k->aux = a->aux;

@@ -77,7 +77,10 @@ class Args(ctypes.Structure):
                 ("row_begin", ctypes.c_int), ("row_end", ctypes.c_int),
                 ("src_row_begin", ctypes.c_int), ("src_row_end", ctypes.c_int),
                 ("dst_row_begin", ctypes.c_int), ("fparam", ctypes.c_float * 8),
-                ("fanout", ctypes.c_void_p * 8), ("n_fanout", ctypes.c_int)]
+                ("fanout", ctypes.c_void_p * 8), ("n_fanout", ctypes.c_int), ("flags", ctypes.c_int)]
+
+
+ARGS_INDEPENDENT = 1       # orion.h ORION_ARGS_INDEPENDENT
 
 
 def with_fanout(a: Args, ptrs) -> Args:
@@ -240,7 +243,10 @@ def compile_info(kernel_id: str, block_threads: int, reg_cap: int) -> dict:
 # ---- launch arguments ----------------------------------------------------------------------
 def denoise_args(kernel_id: str, src: int, dst: int, width: int, height: int, row_begin: int = 0,
                  row_end: int | None = None, src_row_begin: int = 0, src_row_end: int | None = None,
-                 dst_row_begin: int | None = None, params=None) -> Args:
+                 dst_row_begin: int | None = None, params=None, independent: bool = False) -> Args:
+    """Arguments of one denoiser launch.  independent: ORION_ARGS_INDEPENDENT -- the caller asserts
+    the launch touches nothing the stream's previous kernel writes (e.g. the next frame, in its own
+    buffers), so with PDL it need not wait for that kernel."""
     row_end = height if row_end is None else row_end
     src_row_end = height if src_row_end is None else src_row_end
     dst_row_begin = row_begin if dst_row_begin is None else dst_row_begin
@@ -248,6 +254,7 @@ def denoise_args(kernel_id: str, src: int, dst: int, width: int, height: int, ro
     a = Args(src, dst, None, width, height, row_begin, row_end, src_row_begin, src_row_end, dst_row_begin)
     for i, x in enumerate(p):
         a.fparam[i] = x
+    a.flags = ARGS_INDEPENDENT if independent else 0
     return a
 
 

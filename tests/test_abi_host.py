@@ -203,3 +203,30 @@ def test_set_pdl_switch_host_only():
         assert O.lib().orion_set_pdl(2, None) == -1   # ORION_E_INVALID
     finally:
         O.set_pdl(prev)
+
+
+def test_ctypes_structs_match_the_header_layout(tmp_path):
+    # the binding's ctypes mirrors (orion.py) against the C compiler's layout of include/orion.h
+    import ctypes
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    structs = {"orion_args": O.Args, "orion_tuner_cfg": O.TunerCfg, "orion_step_report": O.StepReport,
+               "orion_device_limits": O.DeviceLimits, "orion_kernel_resources": O.KernelResources,
+               "orion_level": O.Level}
+    src = ["#include <stdio.h>", "#include <stddef.h>", '#include "orion.h"', "int main(void) {"]
+    for cname, cls in structs.items():
+        src.append(f'printf("{cname} %zu\\n", sizeof({cname}));')
+        for f in cls._fields_:
+            src.append(f'printf("{cname}.{f[0]} %zu\\n", offsetof({cname}, {f[0]}));')
+    src += ["return 0; }"]
+    c = tmp_path / "layout.c"
+    c.write_text("\n".join(src))
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-I", os.path.join(root, "include"), str(c), "-o", str(exe)], check=True)
+    got = dict(l.rsplit(" ", 1) for l in subprocess.run([str(exe)], capture_output=True, text=True,
+                                                         check=True).stdout.split("\n") if l)
+    for cname, cls in structs.items():
+        assert int(got[cname]) == ctypes.sizeof(cls), cname
+        for f in cls._fields_:
+            assert int(got[f"{cname}.{f[0]}"]) == getattr(cls, f[0]).offset, (cname, f[0])
+    assert O.ARGS_INDEPENDENT == 1
