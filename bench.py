@@ -447,6 +447,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     kmax = nlev - 1
 
     # ---- inputs resident in HBM: a pool of frames larger than L2 -------------------------
+    chain = None
     frame_bytes = W * H * (4 if is_stencil else 16)
     nframes = max(2, math.ceil(2 * 126e6 / (2 * frame_bytes)) + 1)
     if is_stencil:
@@ -462,16 +463,20 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
         state = {"a": t_a, "b": t_b}
         q0 = torch.empty(1, device=dev)   # srad: the ROI statistic of the current iteration
 
-        def grid_args(src, dst):
+        # consecutive iterations overlapped tile by tile (orion_chain) where the family allows it;
+        # the sweep below repeats one launch and runs unchained
+        chain = O.Chain(variants, W, H) if kernel in O.CHAINABLE and not args.no_chain else None
+
+        def grid_args(src, dst, ch=None):
             if is_srad:
                 return O.srad_args(src.data_ptr(), dst.data_ptr(), 0 if fused else q0.data_ptr(), W, H,
-                                   roi=ROI if fused else None)
-            return O.hotspot_args(src.data_ptr(), dst.data_ptr(), pw.data_ptr(), W, H)
+                                   roi=ROI if fused else None, chain=ch)
+            return O.hotspot_args(src.data_ptr(), dst.data_ptr(), pw.data_ptr(), W, H, chain=ch)
 
         def step_args(s):
             if is_srad and not fused:   # the iteration's ROI statistics precede the tuned update kernel
                 O.srad_roi_stats(local, state["a"].data_ptr(), W, H, ROI, q0.data_ptr(), sp)
-            a = grid_args(state["a"], state["b"])
+            a = grid_args(state["a"], state["b"], chain)
             state["a"], state["b"] = state["b"], state["a"]
             return a
     else:
@@ -677,6 +682,10 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
                              "grids (3 x 256 MiB) > L2 (126 MB)",
                        "parallelism": f"dp{world} (independent frames per GPU)",
                        "cuda_graph": graph is not None,
+                       "overlap": ("orion_chain (tile-level waits between iterations)" if chain is not None else
+                                   "none (each iteration waits for the whole previous grid)") if is_stencil else
+                                  ("independent frames (ORION_ARGS_INDEPENDENT: no grid-wide wait)"
+                                   if nframes > 1 and graph is None else "none"),
                        "issue": "graph" if graph is not None else ("orion_tune_steps" if native_args is not None
                                                                    else "orion_tune_step per step")},
             "roofline": _roofline(kernel, wl, W * H, ms_step),      # bytes / instructions per cell or pixel per launch
@@ -712,6 +721,9 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
             "realise": "min_carveout" if realise == O.REALISE_MIN_CARVEOUT else "max_smem",
             "carveout_axis": caxis,
         }
+    torch.cuda.synchronize()
+    if chain is not None:
+        chain.close()
     tuner.close()
     variants.close()
     if graph_loop:
@@ -1363,6 +1375,8 @@ def main(argv=None):
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--sub-cpu-seconds", type=float, default=3.0)
     ap.add_argument("--no-energy", action="store_true", help="skip the NEXT-3 energy record")
+    ap.add_argument("--no-chain", action="store_true",
+                    help="stencils: launch every iteration grid-wide ordered (no orion_chain)")
     ap.add_argument("--no-anchor", action="store_true", help="N > 1: skip C5 at P = 1 on rank 0")
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
     ap.add_argument("--kernel", default="", help="override the headline workload's kernel id (same family)")

@@ -224,8 +224,11 @@ void orion_variants_destroy(orion_variants *v);
  *             caller asserts the independence; the result bits are the same.  Set on a
  *             stencil / SRAD launch (each reads its predecessor's output), or any other bit ->
  *             ORION_E_INVALID.  The host-buffer entry points (orion_tune_step_host,
- *             orion_host_pipe_submit) launch after their own copies and ignore it. */
+ *             orion_host_pipe_submit) launch after their own copies and ignore it.
+ *  chain:     NULL, or an orion_chain of this kernel family and grid (below): the launch is the
+ *             chain's next iteration and waits for the previous one tile by tile, not grid-wide. */
 #define ORION_ARGS_INDEPENDENT 1
+typedef struct orion_chain orion_chain;   /* opaque, library-owned: see orion_chain_create */
 typedef struct {
     const void *src;
     void *dst;
@@ -238,7 +241,34 @@ typedef struct {
     void *fanout[8];
     int n_fanout;
     int flags;
+    orion_chain *chain;   /* NULL, or the chain this launch continues (orion_chain_create) */
 } orion_args;
+
+/* ---- chains: consecutive stencil iterations overlapped tile by tile ----------------------
+ * A stencil iteration reads what the previous one wrote, so each launch normally waits for the
+ * whole previous grid (griddepcontrol.wait): the last, partial wave of every iteration leaves
+ * SMs idle.  A chain (one kernel family, one whole grid, one stream) replaces that wait by
+ * per-tile completion epochs in device memory: with programmatic dependent launch on, the CTA
+ * at tile (x, y) of iteration n+1 starts as soon as the tiles of iteration n whose output it
+ * reads or whose input it overwrites (the 3 x 3 neighbourhood: halos are smaller than a tile;
+ * for "srad_f32hs" also the ROI tiles that write the statistics slots) have completed, so
+ * iteration n+1 fills iteration n's last wave (the iterations of P:L605-P:L607, overlapped;
+ * the bits are unchanged).  Chainable: "hotspot4h_f32", "srad_f32hs".  Rules: every launch of
+ * the chain covers the whole grid (row_begin = 0, row_end = height, src / dst rows from 0),
+ * takes no flags or fan-out, goes to the same stream, and is not captured into a graph
+ * (orion_tuner_capture) or repeated by orion_sweep -- each gets ORION_E_INVALID.  Behind any
+ * other liborion kernel on the stream (or at the chain's first launch) a chained launch waits
+ * grid-wide as usual; kernels from outside liborion that use programmatic dependent launch
+ * themselves must not be enqueued between two launches of a chain.  A CTA that waits 4 s
+ * (a broken chain) traps instead of hanging. */
+/* Allocates the chain's tile flags (zeroed) for `v`'s kernel family and a width x height grid
+ * (the iterations of P:L605-P:L607 on one grid).  ORION_E_INVALID for a family without chains. */
+orion_status orion_chain_create(const orion_variants *v, int width, int height, orion_chain **out);
+/* Launches (iterations) enqueued on the chain so far, and its tile grid.  Any output may
+ * be NULL. */
+orion_status orion_chain_info(const orion_chain *c, unsigned *epoch, int *tiles_x, int *tiles_y);
+/* Frees the chain (after its launches -- the iterations of P:L605 -- have completed). */
+void orion_chain_destroy(orion_chain *c);
 
 /* Launch variant `level_idx` (realising its occupancy level, P:L649, P:L757-P:L759) on
  * `stream` (async).  An empty row range (row_begin == row_end) is a no-op returning ORION_OK.
@@ -370,7 +400,8 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
  *           once with orion_srad_stats_init before the first iteration)
  *   roi     srad only: {r1, r2, c1, c2} of the ROI statistics run before every iteration
  * Copies in, runs `iterations` orion_tune_step iterations on `stream` (hotspot2h_f32 advances
- * two time steps per iteration, hotspot4h_f32 four), copies the final grid out and synchronises the stream.
+ * two time steps per iteration, hotspot4h_f32 four; chainable families run them as one
+ * internal orion_chain), copies the final grid out and synchronises the stream.
  * Bytes copied are returned in *h2d_bytes / *d2h_bytes.  ORION_E_INVALID on other kernels,
  * partial row ranges or missing buffers. */
 orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterations, void *dev_a, void *dev_b,

@@ -23,7 +23,7 @@ ORION_DEVICE bool orion_probe(const orion_kargs &a)
     // visible -- before any load -- unless the caller asserted the launch independent of it
     // (ORION_ARGS_INDEPENDENT: the CTAs start in the previous grid's last wave).  Both are no-ops
     // for a normal launch.
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    if (!a.dep_late) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     if (!a.nowait) asm volatile("griddepcontrol.wait;" ::: "memory");
     if (a.probe == nullptr) return false;
     if (threadIdx.x == 0 && threadIdx.y == 0) {
@@ -44,6 +44,67 @@ ORION_DEVICE bool orion_probe(const orion_kargs &a)
 }
 #define ORION_PROBE(a) \
     if (orion_probe(a)) return
+
+// ---- orion_chain: tile-level dependencies between consecutive launches -------------------------
+// A chained launch (orion.h orion_chain) does not wait for the whole previous grid: its CTA at
+// tile (bx, by) waits only until the previous launch of the chain has completed the tiles whose
+// output it reads or whose input it overwrites -- the 3 x 3 neighbourhood (the stencil halos are
+// smaller than a tile) plus an optional extra rectangle (SRAD: the ROI tiles that write the
+// statistics slots) -- and publishes its own completion at the end.  Flags hold the epoch of the
+// last launch that completed the tile: wait for >= epoch-1, publish epoch (release / acquire at
+// GPU scope; the data written by other SMs is then read through L2: cp.async.cg / ld.global.cg).
+ORION_DEVICE unsigned chain_ld_acquire(const unsigned *p)
+{
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+ORION_DEVICE void chain_wait_tile(const orion_kargs &a, int x, int y, unsigned long long t0)
+{
+    const unsigned *f = a.chain + (size_t)y * gridDim.x + x;
+    const unsigned need = a.chain_epoch - 1u;
+    while (chain_ld_acquire(f) < need) {
+        __nanosleep(200);
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        if (t - t0 > 4000000000ull) __trap();   // 4 s: a broken chain (misuse) fails loudly, never hangs
+    }
+}
+// Called by every thread of the CTA (contains a barrier).  ex0 > ex1: no extra rectangle.  The
+// lanes of warp 0 poll one tile each (k < 9: the 3 x 3 neighbourhood, then the extra rectangle),
+// so a CTA pays one flag round trip, not one per tile.
+ORION_DEVICE void chain_wait(const orion_kargs &a, int ex0, int ex1, int ey0, int ey1)
+{
+    if (threadIdx.y == 0) {
+        unsigned long long t0;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        const int gx = gridDim.x, gy = gridDim.y;
+        const int ew = ex1 >= ex0 ? ex1 - ex0 + 1 : 0, eh = ey1 >= ey0 ? ey1 - ey0 + 1 : 0;
+        for (int k = threadIdx.x; k < 9 + ew * eh; k += 32) {
+            int x, y;
+            if (k < 9) {
+                x = (int)blockIdx.x + k % 3 - 1;
+                y = (int)blockIdx.y + k / 3 - 1;
+            } else {
+                x = ex0 + (k - 9) % ew;
+                y = ey0 + (k - 9) / ew;
+            }
+            if (x >= 0 && x < gx && y >= 0 && y < gy) chain_wait_tile(a, x, y, t0);
+        }
+        __syncwarp();
+    }
+    __syncthreads();
+}
+// Called by every thread of the CTA after its last global access (contains a barrier).
+ORION_DEVICE void chain_signal(const orion_kargs &a)
+{
+    __syncthreads();
+    if (threadIdx.x == 0 && threadIdx.y == 0) {
+        __threadfence();
+        unsigned *f = a.chain + (size_t)blockIdx.y * gridDim.x + blockIdx.x;
+        asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(f), "r"(a.chain_epoch) : "memory");
+    }
+}
 
 ORION_DEVICE int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
 

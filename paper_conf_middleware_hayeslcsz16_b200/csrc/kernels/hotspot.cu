@@ -419,18 +419,25 @@ __device__ __forceinline__ void hotspotS_strip(const orion_kargs &a, int ys, int
     }
 }
 
+// A chained launch (orion_chain) waits for the previous launch's 3 x 3 neighbourhood of tiles --
+// every tile whose output rows / columns this CTA's strips read (halo S <= 4 < the 120 x 512
+// tile) or whose input this CTA's output overwrites (ping-pong) -- instead of the whole grid.
 template <int S, int RY, int NB>
 __device__ __forceinline__ void hotspotS_body(const orion_kargs &a)
 {
+    const bool chained = a.chain != nullptr;
+    if (chained) chain_wait(a, 1, 0, 1, 0);
     const int ys = a.row_begin + (blockIdx.y * 8 + threadIdx.y) * RY;
-    if (ys >= a.row_end) return;
-    const int ye = min(ys + RY, a.row_end);
-    const bool redge = ys - S < 0 || ye - 1 + S > a.height - 1;
-    const bool cedge = blockIdx.x == 0 || (int)blockIdx.x * 120 + 124 >= a.width;
-    if (!redge && !cedge)
-        hotspotS_strip<S, NB, false, false>(a, ys, ye);
-    else
-        hotspotS_strip<S, NB, true, true>(a, ys, ye);
+    if (ys < a.row_end) {
+        const int ye = min(ys + RY, a.row_end);
+        const bool redge = ys - S < 0 || ye - 1 + S > a.height - 1;
+        const bool cedge = blockIdx.x == 0 || (int)blockIdx.x * 120 + 124 >= a.width;
+        if (!redge && !cedge)
+            hotspotS_strip<S, NB, false, false>(a, ys, ye);
+        else
+            hotspotS_strip<S, NB, true, true>(a, ys, ye);
+    }
+    if (chained) chain_signal(a);
 }
 
 // T = 256 threads (32 x 8 warps): 120 output columns x 8 strips of HS_ROWS rows per CTA; 4 steps

@@ -150,9 +150,9 @@ ORION_DEVICE double *srad_stats_area(const void *grid, const orion_kargs &a, int
 ORION_DEVICE float srad_q0_from_slots(const double *slots, const SradRoi &r, int lane)
 {
     double s = 0.0, s2 = 0.0;
-    for (int k = lane; k < r.nslots; k += 32) {
-        s += slots[2 * k];
-        s2 += slots[2 * k + 1];
+    for (int k = lane; k < r.nslots; k += 32) {     // through L2 (written by other SMs, see chain_wait)
+        s += __ldcg(slots + 2 * k);
+        s2 += __ldcg(slots + 2 * k + 1);
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
@@ -544,7 +544,8 @@ constexpr int SRADH_SLOT = 128;   // floats per ring slot: the warp's 128 column
 }  // namespace
 
 template <bool CEDGE, bool STATS = false>
-__device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int ys, int ye)
+__device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int ys, int ye,
+                                             const SradConsts *pre = nullptr)
 {
     const int W = a.width, H = a.height;
     const int lane = threadIdx.x;
@@ -557,7 +558,9 @@ __device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int
     const float *J = (const float *)a.src - (size_t)a.src_row_begin * (size_t)W + cxl;   // row 0, own columns
     float *Jo = (float *)a.dst + (size_t)cx - (size_t)a.dst_row_begin * (size_t)W;
 
-    auto load = [&](int y) { return __ldg(reinterpret_cast<const float4 *>(J + (size_t)y * (size_t)W)); };
+    // rows written by the previous launch (possibly still running on other SMs for a chained
+    // launch, orion_chain): read through L2
+    auto load = [&](int y) { return __ldcg(reinterpret_cast<const float4 *>(J + (size_t)y * (size_t)W)); };
     auto coeff_row = [&](const float4 &N, const float4 &T, const float4 &S) {
         float Wv = __shfl_up_sync(0xffffffffu, T.w, 1);
         float Ev = __shfl_down_sync(0xffffffffu, T.x, 1);
@@ -602,8 +605,9 @@ __device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int
         srad_commit();
     }
     if (STATS)   // the input's q0sqr from its statistics slots, while the ring rows are in flight
-        kc = srad_consts_q0(srad_q0_from_slots(srad_stats_area(a.src, a, a.src_row_begin), srad_roi(a), lane),
-                            a.fparam[0]);
+        kc = pre ? *pre
+                 : srad_consts_q0(srad_q0_from_slots(srad_stats_area(a.src, a, a.src_row_begin), srad_roi(a), lane),
+                                  a.fparam[0]);
     float4 j0 = load(ys), j1 = load(min(ys + 1, H - 1)), j2;
     CRow<4> c0 = coeff_row(load(max(ys - 1, 0)), j0, j1), c1;
     auto row = [&](int q, float *sl_read, float *sl_issue, const float4 &N, const float4 &T, float4 &S,
@@ -655,17 +659,34 @@ __device__ __forceinline__ void srad_strip_h(const orion_kargs &a, int base, int
 
 // T = 256 threads (32 x 8 warps), output tile 120 x (8 * SRADH_RY); width % 4 == 0.  42-row
 // strips: a multiple of the 6-row loop body (no remainder iterations), 25 x 69 CTAs at 8192^2.
+// A chained srad_f32hs launch (orion_chain) waits for the previous launch's 3 x 3 neighbourhood
+// of tiles and for its ROI tiles (the writers of the statistics slots it reduces); every warp
+// then reduces the slots, and only after that does the CTA let the next launch be scheduled
+// (griddepcontrol.launch_dependents, dep_late): a later launch's ROI warps overwrite the slots
+// behind this launch's input only once every CTA of this launch has read them.
 template <bool STATS>
 __device__ __forceinline__ void srad4h_body(const orion_kargs &a)
 {
+    const bool chained = STATS && a.chain != nullptr;
+    SradConsts pre;
+    if (chained) {
+        const SradRoi r = srad_roi(a);
+        chain_wait(a, r.c1 / 120, r.c2 / 120, r.r1 / (8 * SRADH_RY), r.r2 / (8 * SRADH_RY));
+        pre = srad_consts_q0(srad_q0_from_slots(srad_stats_area(a.src, a, a.src_row_begin), r, threadIdx.x),
+                             a.fparam[0]);
+        __syncthreads();
+        asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    }
     const int ys = a.row_begin + blockIdx.y * (8 * SRADH_RY) + threadIdx.y * SRADH_RY;
-    if (ys >= a.row_end) return;
-    const int base = blockIdx.x * 120;
-    const bool cedge = base == 0 || base + 124 >= a.width;
-    if (cedge)
-        srad_strip_h<true, STATS>(a, base, ys, min(ys + SRADH_RY, a.row_end));
-    else
-        srad_strip_h<false, STATS>(a, base, ys, min(ys + SRADH_RY, a.row_end));
+    if (ys < a.row_end) {
+        const int base = blockIdx.x * 120;
+        const bool cedge = base == 0 || base + 124 >= a.width;
+        if (cedge)
+            srad_strip_h<true, STATS>(a, base, ys, min(ys + SRADH_RY, a.row_end), chained ? &pre : nullptr);
+        else
+            srad_strip_h<false, STATS>(a, base, ys, min(ys + SRADH_RY, a.row_end), chained ? &pre : nullptr);
+    }
+    if (chained) chain_signal(a);
 }
 extern "C" __global__ void __launch_bounds__(256) orion_srad4h_f32_256(orion_kargs a)
 {

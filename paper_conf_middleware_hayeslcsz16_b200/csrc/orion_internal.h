@@ -29,6 +29,11 @@ extern std::atomic<long long> g_launches;
 // Set while orion_tuner_capture records a graph: launches inside it are plain (no PDL attribute).
 extern thread_local bool t_capturing;
 
+// The last kernel liborion enqueued on a stream: its orion_chain (tag) or nullptr for any other
+// kernel.  A chained launch skips the grid-wide wait only behind its own chain's previous launch.
+void note_stream_launch(CUstream s, const void *tag);
+const void *last_stream_tag(CUstream s);
+
 // Makes the primary context of `device` current on the calling thread (retaining it).
 orion_status ensure_context(int device);
 
@@ -67,6 +72,7 @@ struct KernelDef {
     int steps_per_launch;   // stencil steps one launch performs (0 / 1 = one)
     int fanout;             // 1: the kernel's epilogue honours orion_args.fanout (store_out)
     int srad_stats;         // 1: SRAD with the ROI statistics fused (slots behind src / dst grids)
+    int chain;              // 1: honours orion_args.chain (tile-level waits between launches)
     int dyn_need() const
     {
         if (smem_bytes > 0) return smem_bytes;
@@ -92,6 +98,16 @@ orion_status load_aux_module(int device, const char *module, CUmodule *out);
 }  // namespace orion
 
 // Opaque handles.
+// A chain of launches of one kernel family over one whole grid on one stream (orion.h).
+struct orion_chain {
+    int device = 0;
+    const orion::KernelDef *def = nullptr;
+    int width = 0, height = 0, gx = 0, gy = 0;
+    CUdeviceptr flags = 0;          // gy x gx epochs of the last completed launch per tile
+    unsigned epoch = 0;             // launches enqueued so far
+    CUstream stream = nullptr;
+    bool stream_set = false;
+};
 struct orion_variants {
     int device = 0;
     const orion::KernelDef *def = nullptr;

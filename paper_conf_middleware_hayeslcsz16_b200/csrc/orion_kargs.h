@@ -19,7 +19,13 @@ typedef struct {
                                         (orion_probe in kernels/common.cuh)                        */
     void *fan[8];                    /* denoisers: extra full-image outputs (global row y at y*width), */
     int nfan;                        /* e.g. every rank's gather buffer over NVLink peer memory        */
-    int nowait;                      /* 1: ORION_ARGS_INDEPENDENT -- no griddepcontrol.wait (PDL)      */
+    int nowait;                      /* 1: no griddepcontrol.wait (ORION_ARGS_INDEPENDENT, or a chained
+                                        launch whose predecessor is the same chain's previous launch) */
+    int dep_late;                    /* 1: the kernel issues griddepcontrol.launch_dependents itself,
+                                        later than at entry (chained srad_f32hs: after its slot reads) */
+    unsigned *chain;                 /* orion_chain tile flags (gridDim.y x gridDim.x); NULL: none     */
+    unsigned chain_epoch;            /* this launch's epoch; it waits for epoch-1 on the tiles it reads */
+    int chain_pad;
 } orion_kargs;
 
 #endif

@@ -73,9 +73,10 @@ static const KernelDef kKernels[] = {
     {"hotspot2h_f32", 256, "orion_hotspot2h_f32_256", "hotspot", 32, 8, 120, 256, 2, K_STENCIL, 0, 8 * 6 * 256 * 4, 4, 2},
     // four steps per launch, whole halo lanes: the same 120-column warps walking 64-row strips as
     // a 4-stage register pipeline; 9-slot ring of 8 warps x 9 x 256 floats; reads 4 rows beyond;
-    // fan-out = the halo exchange of a row-sharded grid (first / last 4 rows to the neighbours)
+    // fan-out = the halo exchange of a row-sharded grid (first / last 4 rows to the neighbours);
+    // chainable (orion_chain: tile-level waits between consecutive launches)
     {"hotspot4h_f32", 256, "orion_hotspot4h_f32_256", "hotspot", 32, 8, 120, 512, 4, K_STENCIL, 0, 8 * 9 * 256 * 4, 4, 4,
-     1},
+     1, 0, 1},
     // srad: J tile (32+3)^2 + coefficient tile (32+1)^2 floats; reads 2 rows below the tile
     {"srad_f32_tile", 256, "orion_srad_f32_256", "srad", 32, 8, 32, 32, 2, K_SRAD, 0, (35 * 35 + 33 * 33) * 4},
     // srad, register-sliding: 124 x 128 tile; float4 lanes (width % 4 == 0) or scalar lanes;
@@ -84,8 +85,9 @@ static const KernelDef kKernels[] = {
     // srad, halo lanes: 120 x 336 tile, width % 4 == 0; 6-slot ring of 8 warps x 6 x 128 floats
     {"srad_f32h", 256, "orion_srad4h_f32_256", "srad", 32, 8, 120, 8 * 42, 2, K_SRAD, 0, 8 * 6 * 128 * 4, 4},
     // the same with the ROI statistics fused: q0sqr from the slots behind src, the output ROI's
-    // slots written behind dst (no statistics kernel per iteration; whole grids)
-    {"srad_f32hs", 256, "orion_srad4hs_f32_256", "srad", 32, 8, 120, 8 * 42, 2, K_SRAD, 0, 8 * 6 * 128 * 4, 4, 0, 0, 1},
+    // slots written behind dst (no statistics kernel per iteration; whole grids); chainable
+    {"srad_f32hs", 256, "orion_srad4hs_f32_256", "srad", 32, 8, 120, 8 * 42, 2, K_SRAD, 0, 8 * 6 * 128 * 4, 4, 0, 0, 1,
+     1},
 };
 
 const KernelDef *find_kernel(const char *id, int threads)

@@ -393,6 +393,7 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
     da.dst = dev_dst;
     da.aux = dev_aux;
     da.flags = 0;                  // the launch follows this call's own copies
+    da.chain = nullptr;
     ORION_TRY(orion_tune_step(t, &da, stream, out));
     const char *dptr = (const char *)dev_dst + (size_t)(a->row_begin - a->dst_row_begin) * row;
     ORION_CU(D.cuMemcpyDtoHAsync((char *)a->dst + (size_t)(a->row_begin - a->dst_row_begin) * row,
@@ -431,6 +432,22 @@ orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterat
     if (fused)
         ORION_TRY(orion_srad_stats_init(t->v->device, cur, a->width, a->height, roi[0], roi[1], roi[2], roi[3],
                                         stream));
+    // chainable families: the iterations overlap tile by tile (orion_chain); the chain is freed
+    // only after the stream has drained, on every path
+    struct ChainGuard {
+        orion_chain *c = nullptr;
+        CUstream s = nullptr;
+        ~ChainGuard()
+        {
+            if (c) {
+                drv().cuStreamSynchronize(s);
+                orion_chain_destroy(c);
+            }
+        }
+    } chain;
+    chain.s = s;
+    if (def.chain && a->n_fanout == 0 && a->flags == 0)
+        ORION_TRY(orion_chain_create(t->v, a->width, a->height, &chain.c));
     for (int it = 0; it < iterations; ++it) {
         if (srad && !fused)
             ORION_TRY(orion_srad_roi_stats(t->v->device, cur, a->width, a->height, roi[0], roi[1], roi[2], roi[3],
@@ -439,6 +456,7 @@ orion_status orion_tune_run_host(orion_tuner *t, const orion_args *a, int iterat
         da.src = cur;
         da.dst = nxt;
         da.aux = dev_aux;
+        da.chain = chain.c;
         if (fused)
             for (int i = 0; i < 4; ++i) da.fparam[1 + i] = (float)roi[i];
         ORION_TRY(orion_tune_step(t, &da, stream, nullptr));
@@ -551,6 +569,7 @@ orion_status orion_host_pipe_submit(orion_host_pipe *p, const orion_args *a, ori
     da.dst = (void *)s.dst;
     da.aux = (const void *)s.aux;
     da.flags = 0;                  // the launch follows the pipe's copies and event waits
+    da.chain = nullptr;
     da.dst_row_begin = a->row_begin;
     ORION_TRY(orion_tune_step(p->t, &da, p->s_comp, out));
     ORION_CU(D.cuEventRecord(s.ev_done, p->s_comp));

@@ -14,6 +14,8 @@
 #include <cmath>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
+#include <unordered_map>
 #include <string>
 #include <vector>
 
@@ -22,6 +24,22 @@
 #include "orion_internal.h"
 
 using namespace orion;
+
+// The last kernel liborion enqueued per stream (orion_internal.h).
+static std::mutex g_tag_mu;
+static std::unordered_map<CUstream, const void *> g_stream_tag;
+
+void orion::note_stream_launch(CUstream s, const void *tag)
+{
+    std::lock_guard<std::mutex> lk(g_tag_mu);
+    g_stream_tag[s] = tag;
+}
+const void *orion::last_stream_tag(CUstream s)
+{
+    std::lock_guard<std::mutex> lk(g_tag_mu);
+    auto it = g_stream_tag.find(s);
+    return it == g_stream_tag.end() ? nullptr : it->second;
+}
 
 namespace {
 
@@ -84,6 +102,18 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
         return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id +
                                          ": a stencil launch reads its predecessor's output (not independent)");
     k->nowait = (a->flags & ORION_ARGS_INDEPENDENT) ? 1 : 0;
+    if (a->chain) {
+        const orion_chain *c = a->chain;
+        if (!def.chain || c->def != &def)
+            return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + ": chain of another kernel family");
+        if (a->width != c->width || a->height != c->height || a->row_begin != 0 || a->row_end != a->height ||
+            a->src_row_begin != 0 || a->src_row_end != a->height || a->dst_row_begin != 0)
+            return fail(ORION_E_INVALID, "orion_launch: a chained launch covers the chain's whole grid");
+        if (a->flags || a->n_fanout)
+            return fail(ORION_E_INVALID, "orion_launch: a chained launch takes no flags / fan-out");
+        if (t_capturing)
+            return fail(ORION_E_INVALID, "orion_launch: chained launches cannot be captured (epochs advance per launch)");
+    }
     k->src = a->src;
     k->dst = a->dst;
     k->aux = a->aux;
@@ -144,8 +174,9 @@ static int pdl_enabled_setting()
 // orion_srad_stats) for its predecessor's completion before touching memory, so results are
 // unchanged.
 static orion_status launch_maybe_pdl(CUfunction fn, unsigned gx, unsigned gy, unsigned bx, unsigned by,
-                                     unsigned smem, CUstream s, void **params)
+                                     unsigned smem, CUstream s, void **params, const void *tag = nullptr)
 {
+    note_stream_launch(s, tag);
     if (!pdl_enabled()) {
         ORION_CU(drv().cuLaunchKernel(fn, gx, gy, 1, bx, by, 1, smem, s, params, nullptr));
         return ORION_OK;
@@ -171,14 +202,15 @@ static orion_status launch_maybe_pdl(CUfunction fn, unsigned gx, unsigned gy, un
 }
 
 
-orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const orion_kargs &k, CUstream s)
+orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const orion_kargs &k, CUstream s,
+                       const void *tag = nullptr)
 {
     const int rows = k.row_end - k.row_begin;
     if (rows <= 0) return ORION_OK;
     const unsigned gx = (unsigned)((k.width + def.tile_w - 1) / def.tile_w);
     const unsigned gy = (unsigned)((rows + def.tile_h - 1) / def.tile_h);
     void *params[] = {const_cast<orion_kargs *>(&k)};
-    ORION_TRY(launch_maybe_pdl(fn, gx, gy, (unsigned)def.bx, (unsigned)def.by, (unsigned)dyn_bytes, s, params));
+    ORION_TRY(launch_maybe_pdl(fn, gx, gy, (unsigned)def.bx, (unsigned)def.by, (unsigned)dyn_bytes, s, params, tag));
     g_launches.fetch_add(1);
     return ORION_OK;
 }
@@ -213,6 +245,7 @@ orion_status measure_residency(const orion_variants &v, const KernelDef &def, CU
     k.probe = reinterpret_cast<unsigned *>(buf.p);
     void *params[] = {&k};
     const unsigned grid = (unsigned)(v.dev.sm_count * v.dev.max_blocks_per_sm);
+    note_stream_launch(nullptr, nullptr);
     ORION_CU(D.cuLaunchKernel(fn, grid, 1, 1, (unsigned)def.bx, (unsigned)def.by, 1, (unsigned)dyn_bytes, nullptr,
                               params, nullptr));
     ORION_CU(D.cuCtxSynchronize());
@@ -372,7 +405,62 @@ orion_status orion_launch(orion_variants *v, int i, const orion_args *a, void *s
     if (a->row_begin == a->row_end) return ORION_OK;
     ORION_TRY(ensure_context(v->device));
     const auto &w = v->vars[i];
-    return launch_fn(*v->def, w.fn, w.dyn_bytes, k, (CUstream)stream);
+    orion_chain *c = a->chain;
+    if (!c) return launch_fn(*v->def, w.fn, w.dyn_bytes, k, (CUstream)stream);
+    if (c->device != v->device) return fail(ORION_E_INVALID, "orion_launch: chain of another device");
+    if (c->stream_set && c->stream != (CUstream)stream)
+        return fail(ORION_E_INVALID, "orion_launch: a chain's launches go to one stream");
+    k.chain = (unsigned *)c->flags;
+    k.chain_epoch = c->epoch + 1;
+    // tile-level waits replace the grid-wide wait only right behind this chain's previous launch;
+    // behind any other kernel of liborion (or the chain's first launch) the launch waits as usual
+    k.nowait = (c->epoch > 0 && last_stream_tag((CUstream)stream) == (const void *)c) ? 1 : 0;
+    k.dep_late = v->def->srad_stats ? 1 : 0;
+    ORION_TRY(launch_fn(*v->def, w.fn, w.dyn_bytes, k, (CUstream)stream, c));
+    c->epoch += 1;
+    c->stream = (CUstream)stream;
+    c->stream_set = true;
+    return ORION_OK;
+}
+
+orion_status orion_chain_create(const orion_variants *v, int width, int height, orion_chain **out)
+{
+    if (!v || !out || width <= 0 || height <= 0) return fail(ORION_E_INVALID, "orion_chain_create: bad argument");
+    *out = nullptr;
+    if (!v->def->chain)
+        return fail(ORION_E_INVALID, std::string("orion_chain_create: ") + v->def->id + " does not take a chain");
+    ORION_TRY(ensure_context(v->device));
+    std::unique_ptr<orion_chain> c(new orion_chain());
+    c->device = v->device;
+    c->def = v->def;
+    c->width = width;
+    c->height = height;
+    c->gx = (width + v->def->tile_w - 1) / v->def->tile_w;
+    c->gy = (height + v->def->tile_h - 1) / v->def->tile_h;
+    const size_t bytes = (size_t)c->gx * (size_t)c->gy * sizeof(unsigned);
+    if (drv().cuMemAlloc(&c->flags, bytes) != CUDA_SUCCESS) return fail(ORION_E_CUDA, "cuMemAlloc (chain flags)");
+    if (drv().cuMemsetD32(c->flags, 0u, bytes / sizeof(unsigned)) != CUDA_SUCCESS) {
+        drv().cuMemFree(c->flags);
+        return fail(ORION_E_CUDA, "cuMemsetD32 (chain flags)");
+    }
+    *out = c.release();
+    return ORION_OK;
+}
+
+void orion_chain_destroy(orion_chain *c)
+{
+    if (!c) return;
+    if (drv().ok && c->flags && ensure_context(c->device) == ORION_OK) drv().cuMemFree(c->flags);
+    delete c;
+}
+
+orion_status orion_chain_info(const orion_chain *c, unsigned *epoch, int *tiles_x, int *tiles_y)
+{
+    if (!c) return fail(ORION_E_INVALID, "orion_chain_info: NULL");
+    if (epoch) *epoch = c->epoch;
+    if (tiles_x) *tiles_x = c->gx;
+    if (tiles_y) *tiles_y = c->gy;
+    return ORION_OK;
 }
 
 orion_status orion_default_params(const char *kernel_id, float *fparam, int n)
@@ -431,6 +519,7 @@ orion_status orion_set_pdl(int on, int *previous)
 orion_status orion_sweep(orion_variants *v, const orion_args *a, void *stream, int rounds, float *ms_median)
 {
     if (!v || !a || rounds <= 0 || !ms_median) return fail(ORION_E_INVALID, "orion_sweep: bad argument");
+    if (a->chain) return fail(ORION_E_INVALID, "orion_sweep: repeats one launch -- time it without a chain");
     orion_kargs k;
     ORION_TRY(make_kargs(*v->def, a, &k));
     if (a->row_begin == a->row_end) {     // nothing to time: an empty launch is a no-op at every level
@@ -536,6 +625,7 @@ orion_status orion_generate_rgba(int device, void *dst, int W, int H, int row_be
     const float s = (float)(std::sqrt(3.0) * (double)sigma);
     unsigned long long sd = seed;
     void *params[] = {&dst, &W, &H, &row_begin, &row_end, &sd, (void *)&s, &bx};
+    note_stream_launch((CUstream)stream, nullptr);
     ORION_CU(drv().cuLaunchKernel(f, (unsigned)((W + 255) / 256), (unsigned)(row_end - row_begin), 1, 256, 1, 1, 0,
                                   (CUstream)stream, params, nullptr));
     g_launches.fetch_add(1);
@@ -552,6 +642,7 @@ orion_status orion_generate_thermal(int device, void *t0, void *pw, int W, int H
     ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_gen_thermal"));
     unsigned long long sd = seed;
     void *params[] = {&t0, &pw, &W, &H, &sd};
+    note_stream_launch((CUstream)stream, nullptr);
     ORION_CU(drv().cuLaunchKernel(f, (unsigned)((W + 255) / 256), (unsigned)H, 1, 256, 1, 1, 0, (CUstream)stream,
                                   params, nullptr));
     g_launches.fetch_add(1);
@@ -568,6 +659,7 @@ orion_status orion_flush_l2(int device, void *buf, long long bytes, void *stream
     size_t n = (size_t)(bytes / 16);
     float val = 0.0f;
     void *params[] = {&buf, &n, &val};
+    note_stream_launch((CUstream)stream, nullptr);
     ORION_CU(drv().cuLaunchKernel(f, 148 * 8, 1, 1, 256, 1, 1, 0, (CUstream)stream, params, nullptr));
     g_launches.fetch_add(1);
     return ORION_OK;

@@ -33,6 +33,8 @@ HALO = {"knn_f4": 3, "knn_f4_p1": 3, "knn_f4_t16": 3, "nlm_f4": 6, "nlm_f4_w": 6
 # stencil steps one launch advances (temporal blocking); every other kernel: 1
 STEPS_PER_LAUNCH = {"hotspot2h_f32": 2, "hotspot4h_f32": 4}
 KERNELS = tuple(HALO)
+# families whose launches take an orion_chain (tile-level waits between iterations)
+CHAINABLE = ("hotspot4h_f32", "srad_f32hs")
 
 
 class OrionError(RuntimeError):
@@ -77,7 +79,8 @@ class Args(ctypes.Structure):
                 ("row_begin", ctypes.c_int), ("row_end", ctypes.c_int),
                 ("src_row_begin", ctypes.c_int), ("src_row_end", ctypes.c_int),
                 ("dst_row_begin", ctypes.c_int), ("fparam", ctypes.c_float * 8),
-                ("fanout", ctypes.c_void_p * 8), ("n_fanout", ctypes.c_int), ("flags", ctypes.c_int)]
+                ("fanout", ctypes.c_void_p * 8), ("n_fanout", ctypes.c_int), ("flags", ctypes.c_int),
+                ("chain", ctypes.c_void_p)]
 
 
 ARGS_INDEPENDENT = 1       # orion.h ORION_ARGS_INDEPENDENT
@@ -162,13 +165,15 @@ def lib() -> ctypes.CDLL:
                 "orion_flush_l2": [I, V, ctypes.c_longlong, V],
                 "orion_srad_roi_stats": [I, V, I, I, I, I, I, I, V, V],
                 "orion_srad_stats_init": [I, V, I, I, I, I, I, I, V],
+                "orion_chain_create": [V, I, I, P(V)],
+                "orion_chain_info": [V, P(ctypes.c_uint), P(I), P(I)],
             }
             for name, args in sig.items():
                 f = getattr(L, name)
                 f.argtypes = args
                 f.restype = ctypes.c_int
             for name in ("orion_variants_destroy", "orion_tuner_destroy", "orion_host_pipe_destroy",
-                         "orion_graph_destroy"):
+                         "orion_graph_destroy", "orion_chain_destroy"):
                 getattr(L, name).argtypes = [V]
                 getattr(L, name).restype = None
             L.orion_status_str.restype = ctypes.c_char_p
@@ -269,14 +274,16 @@ def default_params(kernel_id: str) -> tuple:
 
 def hotspot_args(t_in: int, t_out: int, power: int, width: int, height: int, row_begin: int = 0,
                  row_end: int | None = None, consts=None, src_row_begin: int = 0, src_row_end: int | None = None,
-                 dst_row_begin: int = 0) -> Args:
+                 dst_row_begin: int = 0, chain: "Chain | None" = None) -> Args:
     """Arguments of one thermal-stencil launch.  Whole grid by default; a row band of a sharded
-    grid: t_in / power hold global rows [src_row_begin, src_row_end), t_out from dst_row_begin."""
+    grid: t_in / power hold global rows [src_row_begin, src_row_end), t_out from dst_row_begin.
+    chain: the orion_chain this whole-grid launch continues (tile-level waits, orion.h)."""
     row_end = height if row_end is None else row_end
     src_row_end = height if src_row_end is None else src_row_end
     a = Args(t_in, t_out, power, width, height, row_begin, row_end, src_row_begin, src_row_end, dst_row_begin)
     for i, x in enumerate(consts or default_params("hotspot_f32")[:5]):
         a.fparam[i] = x
+    a.chain = chain.h if chain is not None else None
     return a
 
 
@@ -543,7 +550,7 @@ SRAD_STATS_FLOATS = 256
 
 
 def srad_args(j_in: int, j_out: int, q0: int, width: int, height: int, lam: float | None = None,
-              roi=None) -> Args:
+              roi=None, chain: "Chain | None" = None) -> Args:
     """Arguments of one SRAD iteration.  "srad_f32" / "srad_f32h" / "srad_f32_tile": q0 = device
     address of the float q0sqr (orion_srad_roi_stats).  "srad_f32hs": q0 unused (0), roi =
     (r1, r2, c1, c2) -- the statistics travel in the slots behind the grids.  lam None =
@@ -553,7 +560,34 @@ def srad_args(j_in: int, j_out: int, q0: int, width: int, height: int, lam: floa
     if roi is not None:
         for i, v in enumerate(roi):
             a.fparam[1 + i] = float(v)
+    a.chain = chain.h if chain is not None else None
     return a
+
+
+class Chain:
+    """orion_chain: consecutive whole-grid launches of one stencil family on one stream, each
+    waiting for the previous one tile by tile (orion.h).  Pass it to hotspot_args / srad_args."""
+
+    def __init__(self, variants: "Variants", width: int, height: int):
+        self.h = ctypes.c_void_p()
+        _check(lib().orion_chain_create(variants.h, width, height, ctypes.byref(self.h)), "orion_chain_create")
+
+    def info(self) -> tuple[int, int, int]:
+        """(launches so far, tiles_x, tiles_y)."""
+        e, x, y = ctypes.c_uint(), ctypes.c_int(), ctypes.c_int()
+        _check(lib().orion_chain_info(self.h, ctypes.byref(e), ctypes.byref(x), ctypes.byref(y)), "orion_chain_info")
+        return e.value, x.value, y.value
+
+    def close(self):
+        if self.h:
+            lib().orion_chain_destroy(self.h)
+            self.h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 def srad_stats_init(device: int, j: int, width: int, height: int, roi, stream=None):

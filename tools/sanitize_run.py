@@ -1,7 +1,8 @@
 """Small launches of every kernel family for compute-sanitizer (memcheck / racecheck /
 synccheck; SURVEY §4 layer 3 and §5): C1-sized images, ragged edges, every level of each
 kernel once, the SRAD statistics kernels (separate and fused), the generators, the fan-out
-epilogue, row bands read from exactly-sized slabs, and the hotspot / SRAD cp.async rings.  Usage: compute-sanitizer --tool T python tools/sanitize_run.py"""
+epilogue, row bands read from exactly-sized slabs, the hotspot / SRAD cp.async rings and
+chained iterations (orion_chain).  Usage: compute-sanitizer --tool T python tools/sanitize_run.py"""
 import os
 import sys
 
@@ -68,4 +69,29 @@ for i in (0, len(v) - 1):
     fa, fb = fb, fa
 torch.cuda.synchronize()
 print("ok srad_f32hs", flush=True)
+# chained iterations (orion_chain: tile flags polled / published across launches), several tiles
+# in both directions; every level once
+WC, HC = 252, 1100
+ca = torch.zeros(HC * WC + O.SRAD_STATS_FLOATS, device="cuda")
+cb = torch.zeros_like(ca)
+cp = torch.empty((HC, WC), device="cuda")
+O.generate_thermal(0, ca.data_ptr(), cp.data_ptr(), WC, HC, stream=sp)
+v, _ = O.build_all_levels(0, "hotspot4h_f32")
+ch = O.Chain(v, WC, HC)
+for i in list(range(len(v))) * 2:
+    v.launch(i, O.hotspot_args(ca.data_ptr(), cb.data_ptr(), cp.data_ptr(), WC, HC, chain=ch), sp)
+    ca, cb = cb, ca
+torch.cuda.synchronize()
+ch.close()
+print("ok chained hotspot4h_f32", flush=True)
+roi = (300, 700, 100, 200)
+O.srad_stats_init(0, ca.data_ptr(), WC, HC, roi, sp)
+v, _ = O.build_all_levels(0, "srad_f32hs")
+ch = O.Chain(v, WC, HC)
+for i in list(range(len(v))) * 2:
+    v.launch(i, O.srad_args(ca.data_ptr(), cb.data_ptr(), 0, WC, HC, roi=roi, chain=ch), sp)
+    ca, cb = cb, ca
+torch.cuda.synchronize()
+ch.close()
+print("ok chained srad_f32hs", flush=True)
 print("sanitize run complete")
