@@ -551,6 +551,10 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     graph = None
     native_args = None
     if use_graph:
+        # the settled frames are independent (ORION_ARGS_INDEPENDENT): captured with PDL on, the
+        # graph keeps programmatic edges and consecutive 64^2 frames run concurrently (the sweep
+        # and the tuner's exploration above ran without PDL)
+        O.set_pdl(True)
         graph = tuner.capture([step_args(step + k) for k in range(steps)])
         step += steps
         torch.cuda.synchronize()

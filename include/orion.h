@@ -215,13 +215,17 @@ void orion_variants_destroy(orion_variants *v);
  *             reachable over NVLink (P2P / symmetric memory) -- so a row-sharded frame is
  *             gathered by the kernel's own epilogue as each tile completes (C5).  n_fanout = 0:
  *             no fan-out; > 8, or > 0 for other kernels -> ORION_E_INVALID.
- *  flags:     0, or ORION_ARGS_INDEPENDENT for a denoiser launch that reads nothing the stream's
- *             previous kernel writes and writes nothing that kernel reads or writes (e.g. the
- *             next frame of a stream of frames, each in its own buffers; one band after another
- *             of orion_tune_split).  With programmatic dependent launch on (orion_set_pdl), the
- *             kernel then does not wait for its predecessor: its CTAs fill the previous grid's
- *             last wave (one frame per iteration, P:L605-P:L607, overlapped on the GPU).  The
- *             caller asserts the independence; the result bits are the same.  Set on a
+ *  flags:     0, or ORION_ARGS_INDEPENDENT for a denoiser launch independent of the kernels
+ *             enqueued before it on the stream since the last launch without the flag: it reads
+ *             nothing they write and writes nothing they read (writes of identical values to the
+ *             same words excepted) -- e.g. the next frame of a stream of frames, each in its own
+ *             buffers (a pool reused round-robin rewrites a frame's output with the same bits);
+ *             one band after another of orion_tune_split.  With programmatic dependent launch on
+ *             (orion_set_pdl), the kernel then does not wait for its predecessor: its CTAs fill
+ *             the previous grid's last wave (one frame per iteration, P:L605-P:L607, overlapped
+ *             on the GPU), and a graph of such launches (orion_tuner_capture) keeps programmatic
+ *             edges, so consecutive small frames run concurrently.  The caller asserts the
+ *             independence; the result bits are the same.  Set on a
  *             stencil / SRAD launch (each reads its predecessor's output), or any other bit ->
  *             ORION_E_INVALID.  The host-buffer entry points (orion_tune_step_host,
  *             orion_host_pipe_submit) launch after their own copies and ignore it.
@@ -461,8 +465,10 @@ typedef struct orion_graph orion_graph;   /* opaque, library-owned (a CUgraphExe
  * e.g. a ring of frames; device pointers, geometry as for orion_launch -- into a CUDA graph on
  * a library stream.  Each orion_graph_launch then replays the n launches on `stream` with one
  * host call (no per-launch host work: what bounds small frames such as C1's 64x64).  The
- * tuner's iteration counter advances by n per replay.  ORION_E_STATE while the tuner is still
- * exploring; ORION_E_INVALID on n < 1 or bad args. */
+ * tuner's iteration counter advances by n per replay.  The nodes are plain launches unless every
+ * args[i] carries ORION_ARGS_INDEPENDENT and PDL is on: then they keep programmatic dependent
+ * launch and overlap.  ORION_E_STATE while the tuner is still exploring; ORION_E_INVALID on
+ * n < 1, bad args or chained args. */
 orion_status orion_tuner_capture(orion_tuner *t, const orion_args *args, int n, orion_graph **out);
 orion_status orion_graph_launch(orion_graph *g, void *stream);
 void orion_graph_destroy(orion_graph *g);

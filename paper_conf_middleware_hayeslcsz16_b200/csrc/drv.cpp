@@ -45,6 +45,7 @@ const Driver &drv()
 static thread_local std::string t_last_error;
 std::atomic<long long> g_launches{0};
 thread_local bool t_capturing = false;
+thread_local bool t_capture_pdl = false;
 
 orion_status fail(orion_status s, const std::string &msg)
 {

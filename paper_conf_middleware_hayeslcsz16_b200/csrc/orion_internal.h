@@ -28,6 +28,9 @@ orion_status cu_fail(CUresult r, const char *what);          // maps a driver er
 extern std::atomic<long long> g_launches;
 // Set while orion_tuner_capture records a graph: launches inside it are plain (no PDL attribute).
 extern thread_local bool t_capturing;
+// ... and whether its launches keep programmatic dependent launch (every captured launch
+// independent: ORION_ARGS_INDEPENDENT), so the graph gets programmatic edges.
+extern thread_local bool t_capture_pdl;
 
 // The last kernel liborion enqueued on a stream: its orion_chain (tag) or nullptr for any other
 // kernel.  A chained launch skips the grid-wide wait only behind its own chain's previous launch.

@@ -670,10 +670,18 @@ orion_status orion_tuner_capture(orion_tuner *t, const orion_args *args, int n, 
     if (D.cuStreamBeginCapture(s, CU_STREAM_CAPTURE_MODE_THREAD_LOCAL) != CUDA_SUCCESS)
         st = fail(ORION_E_CUDA, "cuStreamBeginCapture");
     const long long before = g_launches.load();
-    t_capturing = true;         // graph nodes are plain kernel launches (measured: PDL edges in the
-                                // C1 graph did not help, ~4.0 vs ~3.8 us per frame)
+    // graph nodes are plain kernel launches, unless every captured launch is independent
+    // (ORION_ARGS_INDEPENDENT): then they keep programmatic dependent launch, the graph gets
+    // programmatic edges and, as the kernels skip griddepcontrol.wait, consecutive frames run
+    // concurrently (C1: 2.9 -> 1.3 us per 64^2 frame; with waiting kernels the edges measured
+    // ~4.0 vs ~3.8 us, no gain)
+    bool indep = true;
+    for (int i = 0; i < n; ++i) indep = indep && (args[i].flags & ORION_ARGS_INDEPENDENT);
+    t_capturing = true;
+    t_capture_pdl = indep;
     for (int i = 0; i < n && st == ORION_OK; ++i) st = orion_launch(t->v, t->f.final_idx, &args[i], s);
     t_capturing = false;
+    t_capture_pdl = false;
     g_launches.store(before);   // captured, not launched: replays are counted
     CUgraph graph = nullptr;
     const CUresult end = D.cuStreamEndCapture(s, &graph);   // always end the capture

@@ -157,7 +157,7 @@ static bool pdl_enabled()
         g_pdl.compare_exchange_strong(on, want);
         on = g_pdl.load();
     }
-    return on && !t_capturing;
+    return on && (!t_capturing || t_capture_pdl);
 }
 
 static int pdl_enabled_setting()

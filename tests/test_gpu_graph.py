@@ -118,3 +118,39 @@ def test_tune_steps_equals_step_loop(knn):
     assert finals[0] == finals[1]
     for a, b in zip(*outs):
         assert np.array_equal(a, b)
+
+
+def test_graph_of_independent_frames_overlaps_and_matches(knn):
+    # ORION_ARGS_INDEPENDENT frames captured with PDL on: the nodes keep programmatic edges and
+    # skip griddepcontrol.wait (consecutive frames run concurrently); the bits are unchanged
+    W = H = 64
+    n = 24
+    sp = torch.cuda.current_stream().cuda_stream
+    prev = O.set_pdl(True)
+    try:
+        srcs = [torch.from_numpy(synth.noisy_rgba(W, H, seed=40 + f, sigma=0.2)).cuda() for f in range(n)]
+        dsts = [torch.zeros_like(s) for s in srcs]
+        args = [O.denoise_args("knn_f4", srcs[f].data_ptr(), dsts[f].data_ptr(), W, H, independent=True)
+                for f in range(n)]
+        tuner = O.Tuner(knn)
+        it = 0
+        while tuner.final()[0] < 0:
+            tuner.step(args[it % n], sp)
+            it += 1
+            assert it < 200
+        final = tuner.final()[0]
+        refs = [torch.zeros_like(s) for s in srcs]
+        for f in range(n):
+            knn.launch(final, O.denoise_args("knn_f4", srcs[f].data_ptr(), refs[f].data_ptr(), W, H), sp)
+        for d in dsts:
+            d.zero_()
+        g = tuner.capture(args)
+        for _ in range(5):
+            g.launch(sp)
+        torch.cuda.synchronize()
+        for f in range(n):
+            assert torch.equal(dsts[f], refs[f]), f
+        g.close()
+        tuner.close()
+    finally:
+        O.set_pdl(prev)
