@@ -299,9 +299,11 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2h_f32_256(orion_
 // LDGSTS) measured 0.176 vs 0.157 ms per launch (three A/B pairs on one box), and a 12-slot TMA
 // ring 0.218 ms: at this granularity the per-row elect / expect_tx / try_wait / warp-sync cost
 // more than the 2 LDGSTS they replace.  Removed.  128-row strips (half the halo re-reads, the same
-// 0.93 wave efficiency at 8192^2) measured 0.163 vs 0.154 ms (three A/B pairs): not kept.
+// 0.93 wave efficiency at 8192^2) measured 0.163 vs 0.154 ms (three A/B pairs) with grid-wide waits
+// between launches; with chained launches (orion_chain: no idle last wave) they measure 0.1401-
+// 0.1412 vs 0.1421-0.1436 ms for 64-row strips (three A/B rounds on one box): kept.
 #ifndef HS_ROWS
-#define HS_ROWS 64
+#define HS_ROWS 128
 #endif
 namespace {
 constexpr int HS_SLOT = 256;                // floats: T0 row segment (128) + P row segment (128)

@@ -71,11 +71,11 @@ static const KernelDef kKernels[] = {
     // two steps per launch (temporal blocking) with whole halo lanes: 120 output columns per warp, 6-slot ring of
     // 8 warps x 6 x 256 floats
     {"hotspot2h_f32", 256, "orion_hotspot2h_f32_256", "hotspot", 32, 8, 120, 256, 2, K_STENCIL, 0, 8 * 6 * 256 * 4, 4, 2},
-    // four steps per launch, whole halo lanes: the same 120-column warps walking 64-row strips as
+    // four steps per launch, whole halo lanes: the same 120-column warps walking 128-row strips as
     // a 4-stage register pipeline; 9-slot ring of 8 warps x 9 x 256 floats; reads 4 rows beyond;
     // fan-out = the halo exchange of a row-sharded grid (first / last 4 rows to the neighbours);
     // chainable (orion_chain: tile-level waits between consecutive launches)
-    {"hotspot4h_f32", 256, "orion_hotspot4h_f32_256", "hotspot", 32, 8, 120, 512, 4, K_STENCIL, 0, 8 * 9 * 256 * 4, 4, 4,
+    {"hotspot4h_f32", 256, "orion_hotspot4h_f32_256", "hotspot", 32, 8, 120, 1024, 4, K_STENCIL, 0, 8 * 9 * 256 * 4, 4, 4,
      1, 0, 1},
     // srad: J tile (32+3)^2 + coefficient tile (32+1)^2 floats; reads 2 rows below the tile
     {"srad_f32_tile", 256, "orion_srad_f32_256", "srad", 32, 8, 32, 32, 2, K_SRAD, 0, (35 * 35 + 33 * 33) * 4},
