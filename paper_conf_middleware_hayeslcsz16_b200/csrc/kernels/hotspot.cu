@@ -301,7 +301,8 @@ extern "C" __global__ void __launch_bounds__(256) orion_hotspot2h_f32_256(orion_
 // more than the 2 LDGSTS they replace.  Removed.  128-row strips (half the halo re-reads, the same
 // 0.93 wave efficiency at 8192^2) measured 0.163 vs 0.154 ms (three A/B pairs) with grid-wide waits
 // between launches; with chained launches (orion_chain: no idle last wave) they measure 0.1401-
-// 0.1412 vs 0.1421-0.1436 ms for 64-row strips (three A/B rounds on one box): kept.
+// 0.1412 vs 0.1421-0.1436 ms for 64-row strips (three A/B rounds on one box): kept.  256-row strips
+// (276 CTAs, less than one wave of 296 slots) chained: 0.158 vs 0.1405 ms (three A/B pairs).
 #ifndef HS_ROWS
 #define HS_ROWS 128
 #endif
