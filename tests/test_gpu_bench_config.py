@@ -11,6 +11,11 @@ dependent launch and issue mode as the timed loops --
   crops whose 100-cell margin holds the dependency cone.
 * SRAD: the 8192^2 grid, 3 chained `srad_f32hs` iterations (statistics fused) through the tuner
   against O5 (double) over the WHOLE grid, <= 1e-5 relative.
+* C1: 64^2 KNN frames (`knn_f4_t16`) tuned without PDL, then the settled iterations of 48
+  independent frames captured as one CUDA graph WITH programmatic edges (consecutive frames run
+  concurrently) and replayed: every frame against the double oracle.
+* C4: two independent 4096^2 frames of `nlm_f4_regheavy` through the tuner (its 16-level ladder
+  explored); one whole frame against the double oracle.
 """
 import numpy as np
 import pytest
@@ -152,4 +157,68 @@ def test_srad_chained_tuned_whole_grid(dev):
     ref, _ = oracle.srad(j0.astype(np.float64), iters, 0.5, ROI)
     rel = np.abs(g - ref) / np.abs(ref)
     assert rel.max() < 1e-5, (levels, float(rel.max()))
+    v.close()
+
+
+def test_c1_graph_of_independent_frames_vs_oracle(dev):
+    W = H = 64
+    n = 48
+    v, _ = O.build_all_levels(0, "knn_f4_t16", mode=O.REALISE_MIN_CARVEOUT)
+    imgs = [synth.noisy_rgba(W, H, seed=1 + f, sigma=0.2) for f in range(n)]
+    srcs = [torch.from_numpy(im).cuda() for im in imgs]
+    dsts = [torch.full_like(s, float("nan")) for s in srcs]
+    args = [O.denoise_args("knn_f4_t16", srcs[f].data_ptr(), dsts[f].data_ptr(), W, H, independent=True)
+            for f in range(n)]
+    prev = O.set_pdl(False)                  # bench.py: the sweep and the exploration run without PDL
+    try:
+        t = bench_tuner(v)
+        s = 0
+        while s < 20 or t.final()[0] < 0:
+            t.step(args[s % n], sp())
+            s += 1
+            assert s < 400
+        torch.cuda.synchronize()
+        for d in dsts:
+            d.fill_(float("nan"))
+        O.set_pdl(True)                      # the timed graph keeps programmatic edges
+        g = t.capture(args)
+        for _ in range(3):
+            g.launch(sp())
+        torch.cuda.synchronize()
+        g.close()
+        t.close()
+    finally:
+        O.set_pdl(prev)
+    res = oracle_par.map_threads(lambda im: oracle.denoise("knn", im), imgs)
+    for f in range(n):
+        out, alt, amb = res[f]
+        g_ = dsts[f].cpu().numpy()
+        e = np.abs(g_[..., :3].astype(np.float64) - out).max(-1)
+        ok = (e <= 1e-5) | (amb & (np.abs(g_[..., :3].astype(np.float64) - alt).max(-1) <= 1e-5))
+        assert ok.all(), (f, int((~ok).sum()), float(e.max()))
+        assert (g_[..., 3] == 0).all(), f
+    v.close()
+
+
+def test_c4_independent_frames_through_the_tuner_vs_oracle(dev):
+    W = H = 4096
+    v, _ = O.build_all_levels(0, "nlm_f4_regheavy", mode=O.REALISE_MIN_CARVEOUT)
+    srcs = [torch.empty((H, W, 4), device="cuda") for _ in range(2)]
+    dsts = [torch.full((H, W, 4), float("nan"), device="cuda") for _ in range(2)]
+    for f, t_ in enumerate(srcs):
+        O.generate_rgba(0, t_.data_ptr(), W, H, seed=1 + f, sigma=0.13, stream=sp())
+    t = bench_tuner(v)
+    s = 0
+    while s < 4 or t.final()[0] < 0:
+        t.step(O.denoise_args("nlm_f4_regheavy", srcs[s % 2].data_ptr(), dsts[s % 2].data_ptr(), W, H,
+                              independent=True), sp())
+        s += 1
+        assert s < 60
+    t.step(O.denoise_args("nlm_f4_regheavy", srcs[0].data_ptr(), dsts[0].data_ptr(), W, H, independent=True), sp())
+    torch.cuda.synchronize()
+    g = dsts[0].cpu().numpy()
+    img = synth.noisy_rgba(W, H, seed=1, sigma=0.13)
+    out, alt, amb = oracle_par.denoise_rows("nlm", img, H, 0, 0, H)
+    check(g, out, alt, amb, "C4 frames through the tuner, frame 0 (whole)")
+    t.close()
     v.close()
