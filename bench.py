@@ -78,6 +78,10 @@ def load_peaks():
     return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
+# throttle reasons that void a timed region (re-measured once); sw_power_cap is kept and noted
+THROTTLE_REJECT = {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "hw_power_brake_slowdown"}
+
+
 class ClockSampler:
     """nvidia-smi-equivalent sampling (NVML) of SM clock + throttle reasons during the timed
     region, and the board energy counter over it.  Call ``mark_end()`` right after the closing
@@ -561,21 +565,36 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     elif native:
         native_args = [step_args(step + k) for k in range(steps)]
         step += steps
-    torch.cuda.nvtx.range_push("timed")   # the launch list (ncu --nvtx-include "timed/") covers only this
-    with ClockSampler(local) as clk:
-        e0.record(stream)
-        if graph is not None:
-            graph.launch(sp)
-        elif native_args is not None:
-            tuner.steps(native_args, sp)
-        else:
-            for _ in range(steps):
-                tuner.step(step_args(step), sp)
-                step += 1
-        e1.record(stream)
+    remeasured = None
+    for attempt in range(2):
+        n_launch0 = O.launch_count()
+        torch.cuda.nvtx.range_push("timed")   # the launch list (ncu --nvtx-include "timed/") covers only this
+        with ClockSampler(local) as clk:
+            e0.record(stream)
+            if graph is not None:
+                graph.launch(sp)
+            elif native_args is not None:
+                tuner.steps(native_args, sp)
+            else:
+                for _ in range(steps):
+                    tuner.step(step_args(step), sp)
+                    step += 1
+            e1.record(stream)
+            torch.cuda.synchronize()
+            clk.mark_end()
+        torch.cuda.nvtx.range_pop()
+        # a timed region that saw a hardware / thermal slowdown is not a measurement: measure it
+        # once more (the same K steps), and keep what the second run saw
+        bad = sorted(THROTTLE_REJECT & set(clk.summary()["reasons"]))
+        flag = torch.tensor([1 if bad else 0], device=dev)
+        if world > 1:
+            dist.all_reduce(flag, op=dist.ReduceOp.MAX)
+        if not int(flag.item()) or attempt == 1:
+            break
+        remeasured = {"first_run_reasons": bad}
         torch.cuda.synchronize()
-        clk.mark_end()
-    torch.cuda.nvtx.range_pop()
+        if world > 1:
+            dist.barrier()
     if graph is not None:
         graph.close()
     launches = O.launch_count() - n_launch0
@@ -693,7 +712,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
                        "issue": "graph" if graph is not None else ("orion_tune_steps" if native_args is not None
                                                                    else "orion_tune_step per step")},
             "roofline": _roofline(kernel, wl, W * H, ms_step),      # bytes / instructions per cell or pixel per launch
-            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk.summary(),
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": dict(clk.summary(), remeasured=remeasured),
             "energy": clk.energy(steps), "select_mode": select,
             "resources": {"final_regs": infos[final].regs if final >= 0 else None,
                           "natural_regs": res.regs_per_thread,
@@ -950,17 +969,28 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier(group=group)
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
-           torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
-    recorded = [] if mode == "gather" else None
-    n0 = O.launch_count()
-    with ClockSampler(local) as clk:
-        for e in ev:
-            e[0].record(stream)
-            one_step(e, recorded)
-            e[2].record(stream)
-        torch.cuda.synchronize()
-        clk.mark_end()
+    remeasured = None
+    for attempt in range(2):
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+               torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+        recorded = [] if mode == "gather" else None
+        n0 = O.launch_count()
+        with ClockSampler(local) as clk:
+            for e in ev:
+                e[0].record(stream)
+                one_step(e, recorded)
+                e[2].record(stream)
+            torch.cuda.synchronize()
+            clk.mark_end()
+        bad = sorted(THROTTLE_REJECT & set(clk.summary()["reasons"]))   # a slowed-down region: once more
+        flag = torch.tensor([1 if bad else 0], device=dev)
+        if world > 1:
+            dist.all_reduce(flag, op=dist.ReduceOp.MAX, group=group)
+        if not int(flag.item()) or attempt == 1:
+            break
+        remeasured = {"first_run_reasons": bad}
+        if world > 1:
+            dist.barrier(group=group)
     launches = O.launch_count() - n0
     tot = ev[0][0].elapsed_time(ev[-1][2])
     if recorded is not None:
@@ -1027,7 +1057,7 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
                           "rows": [c[3], c[4]]} for r, c in enumerate(allc)],
             "sweep_rank0": [{"k": variants.level(i).ctas_per_sm, "ms": round(ms[i], 4)} for i in range(nlev)],
             "regret_rank0": (ms[final] / min(ms) - 1.0) if final >= 0 else None,
-            "gpu_launches": launches, "clocks": clk.summary(), "energy": clk.energy(steps),
+            "gpu_launches": launches, "clocks": dict(clk.summary(), remeasured=remeasured), "energy": clk.energy(steps),
             "e2e": ({"value": H * W * e2e_rec[3] / e2e_dt / 1e6, "unit": "Mpix/s",
                      "h2d_bytes_per_step": float(byts[0]), "d2h_bytes_per_step": float(byts[1]),
                      "steps": e2e_rec[3],
