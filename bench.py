@@ -45,8 +45,11 @@ METRIC = "tuned Mpix/s vs max-occupancy build; tuner regret vs exhaustive level 
 WORKLOADS = {
     # KNN: 49 taps x (3 FSUB + FMUL + 2 FFMA distance, 1 FFMA exponent, 3 FFMA + 1 FADD
     # accumulate, 1 compare) + ~10 for the blend
-    "c1": dict(kernel="knn_f4_t16", W=64, H=64, sigma=0.2, unit="Mpix/s", name="imageDenoising KNN 64x64 RGBA r=3",
-               insts=49 * 12 + 10, bytes=32, steps=3000, cfg_index=0),
+    # C1's 64x64 frames run as batches (orion_args.batch: B frames per launch, one batch per
+    # tuner iteration and per step) through the tile kernel with 256-thread CTAs; --c1-batch 1
+    # restores one frame per step (use --kernel knn_f4_t16, the small-frame kernel, then)
+    "c1": dict(kernel="knn_f4", threads=256, batch=256, W=64, H=64, sigma=0.2, unit="Mpix/s",
+               name="imageDenoising KNN 64x64 RGBA r=3", insts=49 * 12 + 10, bytes=32, steps=300, cfg_index=0),
     # NLM box-sum + symmetric pairs, per pixel and offset pair: 1 difference (6), 1 horizontal
     # and 2 vertical blocked 7-sums (4 each), 2 x (1 FFMA exponent + 3 FFMA + 1 FADD + 1 compare)
     "c2": dict(kernel="nlm_f4_w", W=2048, H=2048, sigma=0.13, unit="Mpix/s", name="imageDenoising NLM 2048x2048 RGBA",
@@ -429,6 +432,8 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     sp = stream.cuda_stream
     wl = WORKLOADS[key]
     kernel, W, H = kernel or wl["kernel"], wl["W"], wl["H"]
+    batch = max(1, args.c1_batch if key == "c1" and args.c1_batch > 0 else wl.get("batch", 1))
+    threads = wl.get("threads", 0) if kernel == wl["kernel"] else 0
     is_srad = kernel.startswith("srad_f32")
     is_stencil = kernel.startswith("hotspot") or is_srad
     fused = kernel == "srad_f32hs"
@@ -441,7 +446,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     # ---- multi-version binary: probe -> levels -> build (offline, untimed) ----------------
     t_build = time.perf_counter()
     realise = O.REALISE_MIN_CARVEOUT if args.realise == "min" else O.REALISE_MAX_SMEM
-    variants, res = O.build_all_levels(local, kernel, mode=realise)
+    variants, res = O.build_all_levels(local, kernel, block_threads=threads, mode=realise)
     t_build = time.perf_counter() - t_build
     nlev = len(variants)
     lv = [variants.level(i) for i in range(nlev)]
@@ -453,7 +458,8 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     # ---- inputs resident in HBM: a pool of frames larger than L2 -------------------------
     chain = None
     frame_bytes = W * H * (4 if is_stencil else 16)
-    nframes = max(2, math.ceil(2 * 126e6 / (2 * frame_bytes)) + 1)
+    # frames (or, batched, batches of frames) in the pool: inputs + outputs larger than L2
+    nframes = max(2, math.ceil(2 * 126e6 / (2 * frame_bytes * batch)) + 1)
     if is_stencil:
         nframes = 1
         # srad_f32hs: the ROI statistics slots travel behind each grid
@@ -484,18 +490,22 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
             state["a"], state["b"] = state["b"], state["a"]
             return a
     else:
-        srcs = [torch.empty((H, W, 4), device=dev) for _ in range(nframes)]
-        dsts = [torch.empty((H, W, 4), device=dev) for _ in range(nframes)]
+        shape = (batch, H, W, 4) if batch > 1 else (H, W, 4)
+        srcs = [torch.empty(shape, device=dev) for _ in range(nframes)]
+        dsts = [torch.empty(shape, device=dev) for _ in range(nframes)]
         for f, t in enumerate(srcs):
-            O.generate_rgba(local, t.data_ptr(), W, H, seed=1 + f + 97 * rank, sigma=wl["sigma"], stream=sp)
+            for b_ in range(batch):
+                fr = t[b_] if batch > 1 else t
+                O.generate_rgba(local, fr.data_ptr(), W, H, seed=1 + f * batch + b_ + 97 * rank, sigma=wl["sigma"],
+                                stream=sp)
 
         def step_args(s, independent=True):
-            # consecutive frames live in their own buffers (nframes >= 2): each launch is
+            # consecutive frames (batches) live in their own buffers (nframes >= 2): each launch is
             # independent of the stream's previous one (ORION_ARGS_INDEPENDENT), so with PDL a
             # frame's CTAs start in the previous frame's last wave
             f = s % nframes
             return O.denoise_args(kernel, srcs[f].data_ptr(), dsts[f].data_ptr(), W, H,
-                                  independent=independent and nframes > 1)
+                                  independent=independent and nframes > 1, batch=batch)
     torch.cuda.synchronize()
 
     # ---- exhaustive sweep (brute-force reference, Fig. 11 Orion-Max/Min) ------------------
@@ -608,7 +618,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
         total_ms = float(t.item())
     final, iters_to_final = tuner.final()
     spl = O.STEPS_PER_LAUNCH.get(kernel, 1)                # stencil steps per launch (temporal blocking)
-    units_per_step = W * H * spl
+    units_per_step = W * H * spl * batch
     value = world * units_per_step * steps / (total_ms * 1e-3) / 1e6
     ms_step = total_ms / steps
     t_final = ms[final] if final >= 0 else float("nan")
@@ -619,10 +629,11 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
         # copies the result device->host; H2D(n+1) / kernel(n) / D2H(n-1) overlap on the pipe's
         # three streams.  The synchronous orion_tune_step_host is reported beside it.
         host_in = [srcs[f].cpu().pin_memory() for f in range(2)]
-        host_out = [torch.empty((H, W, 4)).pin_memory() for _ in range(2)]
-        has = [O.denoise_args(kernel, host_in[f].data_ptr(), host_out[f].data_ptr(), W, H) for f in range(2)]
-        n_e2e = max(4, min(steps, 60 if frame_bytes > 1 << 20 else 2000))
-        pipe = O.HostPipe(tuner, W, H, depth=3)
+        host_out = [torch.empty(srcs[0].shape).pin_memory() for _ in range(2)]
+        has = [O.denoise_args(kernel, host_in[f].data_ptr(), host_out[f].data_ptr(), W, H, batch=batch)
+               for f in range(2)]
+        n_e2e = max(4, min(steps, 60 if frame_bytes * batch > 1 << 20 else 2000))
+        pipe = O.HostPipe(tuner, W, H * batch, depth=3)
         for f in range(2):
             pipe.submit(has[f])                                                    # warm
         pipe.drain()
@@ -645,9 +656,9 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
             t = torch.tensor([dt, dt_sync], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             dt, dt_sync = (float(x) for x in t.tolist())
-        e2e = {"value": world * W * H * n_e2e / dt / 1e6, "unit": wl["unit"], "h2d_bytes_per_step": hi,
+        e2e = {"value": world * W * H * batch * n_e2e / dt / 1e6, "unit": wl["unit"], "h2d_bytes_per_step": hi,
                "d2h_bytes_per_step": ho, "steps": n_e2e, "api": "orion_host_pipe (depth 3, pinned host frames)",
-               "sync_api_value": world * W * H * n_sync / dt_sync / 1e6}
+               "sync_api_value": world * W * H * batch * n_sync / dt_sync / 1e6}
         del host_in, host_out
     else:
         # a whole run per job (orion_tune_run_host): host grids -> device, the config's 100
@@ -700,7 +711,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
             "warmup": warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": wl["name"], "baseline_config_index": wl["cfg_index"], "kernel": kernel,
-                       "block_threads": res.block_threads, "width": W, "height": H, "frames_in_pool": nframes,
+                       "block_threads": res.block_threads, "width": W, "height": H, "frames_per_step": batch, "frames_in_pool": nframes * batch,
                        "l2": "inputs larger than L2: rotating pool of frames" if not is_stencil else
                              "grids (3 x 256 MiB) > L2 (126 MB)",
                        "parallelism": f"dp{world} (independent frames per GPU)",
@@ -711,7 +722,7 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
                                    if nframes > 1 and graph is None else "none"),
                        "issue": "graph" if graph is not None else ("orion_tune_steps" if native_args is not None
                                                                    else "orion_tune_step per step")},
-            "roofline": _roofline(kernel, wl, W * H, ms_step),      # bytes / instructions per cell or pixel per launch
+            "roofline": _roofline(kernel, wl, W * H * batch, ms_step),      # bytes / instructions per cell or pixel per launch
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": dict(clk.summary(), remeasured=remeasured),
             "energy": clk.energy(steps), "select_mode": select,
             "resources": {"final_regs": infos[final].regs if final >= 0 else None,
@@ -772,7 +783,9 @@ def measure_energy(key: str, args, kernel: str, local: int = 0, window_s: float 
     fused = kernel == "srad_f32hs"
     realise = O.REALISE_MIN_CARVEOUT if args.realise == "min" else O.REALISE_MAX_SMEM
     pdl_prev = O.set_pdl(False)          # every level below is replayed as a CUDA graph (plain launches)
-    v, res = O.build_all_levels(local, kernel, mode=realise)
+    batch = wl.get("batch", 1) if kernel == wl["kernel"] else 1
+    v, res = O.build_all_levels(local, kernel, block_threads=wl.get("threads", 0) if kernel == wl["kernel"] else 0,
+                                mode=realise)
     n = len(v)
     if is_stencil:
         extra = O.SRAD_STATS_FLOATS if fused else 0
@@ -794,12 +807,16 @@ def measure_energy(key: str, args, kernel: str, local: int = 0, window_s: float 
             args_pp = [O.hotspot_args(a_.data_ptr(), b_.data_ptr(), p_.data_ptr(), W, H),
                        O.hotspot_args(b_.data_ptr(), a_.data_ptr(), p_.data_ptr(), W, H)]
     else:
-        nfr = max(2, math.ceil(2 * 126e6 / (2 * W * H * 16)) + 1)
-        srcs = [torch.empty((H, W, 4), device="cuda") for _ in range(nfr)]
-        dsts = [torch.empty((H, W, 4), device="cuda") for _ in range(nfr)]
+        nfr = max(2, math.ceil(2 * 126e6 / (2 * W * H * 16 * batch)) + 1)
+        shape = (batch, H, W, 4) if batch > 1 else (H, W, 4)
+        srcs = [torch.empty(shape, device="cuda") for _ in range(nfr)]
+        dsts = [torch.empty(shape, device="cuda") for _ in range(nfr)]
         for f, t in enumerate(srcs):
-            O.generate_rgba(local, t.data_ptr(), W, H, seed=1 + f, sigma=wl["sigma"], stream=sp)
-        args_pp = [O.denoise_args(kernel, srcs[f].data_ptr(), dsts[f].data_ptr(), W, H) for f in range(nfr)]
+            for b_ in range(batch):
+                O.generate_rgba(local, (t[b_] if batch > 1 else t).data_ptr(), W, H, seed=1 + f * batch + b_,
+                                sigma=wl["sigma"], stream=sp)
+        args_pp = [O.denoise_args(kernel, srcs[f].data_ptr(), dsts[f].data_ptr(), W, H, batch=batch)
+                   for f in range(nfr)]
     torch.cuda.synchronize()
     ms = v.sweep(args_pp[0], sp, rounds=args.rounds)
 
@@ -1298,7 +1315,7 @@ def run_single(args):
         line["configs"] = subs
         if not args.no_energy:
             nx = {}
-            for sub, kern in (("c2", "nlm_f4_w"), ("srad", "srad_f32hs"), ("c3", "hotspot_f32"), ("c1", "knn_f4_t16"),
+            for sub, kern in (("c2", "nlm_f4_w"), ("srad", "srad_f32hs"), ("c3", "hotspot_f32"), ("c1", "knn_f4"),
                               ("c4", "nlm_f4_regheavy")):
                 try:
                     nx[f"{sub}:{kern}"] = measure_energy(sub, args, kern, local=local)
@@ -1414,6 +1431,8 @@ def main(argv=None):
     ap.add_argument("--no-anchor", action="store_true", help="N > 1: skip C5 at P = 1 on rank 0")
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
     ap.add_argument("--kernel", default="", help="override the headline workload's kernel id (same family)")
+    ap.add_argument("--c1-batch", type=int, default=0,
+                    help="C1: 64x64 frames per launch / step (0: the workload's default, 256; 1: one frame)")
     ap.add_argument("--c5-chunks", type=int, default=4, help="C5: row chunks per band whose all-gathers overlap compute")
     ap.add_argument("--c5-mode", default="auto", choices=("auto", "fanout", "gather"),
                     help="C5 exchange: kernel fan-out into symmetric memory (auto: when available) or all-gather")

@@ -230,7 +230,16 @@ void orion_variants_destroy(orion_variants *v);
  *             ORION_E_INVALID.  The host-buffer entry points (orion_tune_step_host,
  *             orion_host_pipe_submit) launch after their own copies and ignore it.
  *  chain:     NULL, or an orion_chain of this kernel family and grid (below): the launch is the
- *             chain's next iteration and waits for the previous one tile by tile, not grid-wide. */
+ *             chain's next iteration and waits for the previous one tile by tile, not grid-wide.
+ *  batch:     0 or 1: one frame.  B > 1 (denoisers only, up to 65535): B whole frames of
+ *             width x height pixels, stacked in src and in dst (frame f at f * width * height),
+ *             filtered by one launch (grid z = frame) -- the small frames of configuration C1
+ *             (BASELINE.json configs[0]) one batch per iteration of the tuner, whose
+ *             work-normalised timing counts all B frames.  Requires row_begin =
+ *             src_row_begin = dst_row_begin = 0 and row_end = src_row_end = height, no fan-out,
+ *             no chain; otherwise ORION_E_INVALID.  The host-buffer entry points
+ *             (orion_tune_step_host, orion_host_pipe_submit) copy the B frames as one block each
+ *             way (a pipe needs max_rows >= B * height). */
 #define ORION_ARGS_INDEPENDENT 1
 typedef struct orion_chain orion_chain;   /* opaque, library-owned: see orion_chain_create */
 typedef struct {
@@ -246,6 +255,7 @@ typedef struct {
     int n_fanout;
     int flags;
     orion_chain *chain;   /* NULL, or the chain this launch continues (orion_chain_create) */
+    int batch;            /* 0 / 1: one frame; B > 1: B whole frames in one launch (below)     */
 } orion_args;
 
 /* ---- chains: consecutive stencil iterations overlapped tile by tile ----------------------

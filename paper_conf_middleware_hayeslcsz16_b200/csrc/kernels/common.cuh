@@ -108,6 +108,13 @@ ORION_DEVICE void chain_signal(const orion_kargs &a)
 
 ORION_DEVICE int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
 
+// Frame of a batched denoiser launch (orion_args.batch: gridDim.z whole width x height frames
+// stacked in src / dst): the pixel offset of this CTA's frame (0 for a single frame).
+ORION_DEVICE size_t frame_px(const orion_kargs &a)
+{
+    return (size_t)blockIdx.z * (size_t)a.width * (size_t)a.height;
+}
+
 // Row of the input slab a staged tile reads for global row gy: clamp-to-edge in GLOBAL
 // coordinates (the definition), then into the rows the slab holds.  The second clamp never
 // changes a row that a stored output depends on (the host guarantees the slab covers
@@ -132,7 +139,7 @@ ORION_DEVICE float dist2(float4 a, float4 b)
 template <int TW, int TH, int NT>
 ORION_DEVICE void load_tile_clamped(float4 *tile, const orion_kargs &a, int gx0, int gy0)
 {
-    const float4 *src = (const float4 *)a.src;
+    const float4 *src = (const float4 *)a.src + frame_px(a);
     const int W = a.width;
     const int tid = threadIdx.y * blockDim.x + threadIdx.x;
     for (int idx = tid; idx < TW * TH; idx += NT) {
@@ -167,7 +174,7 @@ ORION_DEVICE void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: 
 // Output pixel (x, y) (global row y) into dst (rows from dst_row_begin).
 ORION_DEVICE void store_out(const orion_kargs &a, int x, int y, float4 o)
 {
-    ((float4 *)a.dst)[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = o;
+    ((float4 *)a.dst)[frame_px(a) + (size_t)(y - a.dst_row_begin) * (size_t)a.width + x] = o;
 }
 
 // Fan-out of this thread's output column x, rows [y0, y1) (already in dst, written by this

@@ -102,7 +102,7 @@ __device__ __forceinline__ void knn_tap_split_body(const orion_kargs &a)
     const int y = a.row_begin + blockIdx.y;
     const int W = a.width, H = a.height;
     const int xc = min(x, W - 1);
-    const float4 *src = (const float4 *)a.src - (size_t)a.src_row_begin * (size_t)W;
+    const float4 *src = (const float4 *)a.src + frame_px(a) - (size_t)a.src_row_begin * (size_t)W;
     const float nl2 = a.fparam[0];
     const float wthr = a.fparam[2];
     const float4 c00 = __ldg(src + (size_t)y * (size_t)W + xc);

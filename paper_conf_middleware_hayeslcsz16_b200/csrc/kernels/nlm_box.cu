@@ -226,7 +226,7 @@ __device__ __forceinline__ void nlm_box_body(const orion_kargs &a)
     const int y0 = a.row_begin + blockIdx.y * TH;
     {   // stage the planar tile (clamp-to-edge in global coords): per pixel one 8-byte (r, g)
         // and one 4-byte b cp.async, all of the thread's copies in flight at once
-        const float4 *src = (const float4 *)a.src;
+        const float4 *src = (const float4 *)a.src + frame_px(a);
 #pragma unroll 4
         for (int idx = tid; idx < PC * PR; idx += NT) {
             const int ty = idx / PC, tx = idx - ty * PC;

@@ -71,7 +71,7 @@ __device__ __forceinline__ void nlm_direct_body(const orion_kargs &a)
     }
     const int x = x0 + threadIdx.x, y = y0 + threadIdx.y;
     if (x < a.width && y < a.row_end)
-        ((float4 *)a.dst)[(size_t)(y - a.dst_row_begin) * (size_t)a.width + x] =
+        ((float4 *)a.dst)[frame_px(a) + (size_t)(y - a.dst_row_begin) * (size_t)a.width + x] =
             lerp_out(c00, ax, ay, az, sw, cnt, a);
 }
 

@@ -25,7 +25,7 @@ typedef struct {
                                         later than at entry (chained srad_f32hs: after its slot reads) */
     unsigned *chain;                 /* orion_chain tile flags (gridDim.y x gridDim.x); NULL: none     */
     unsigned chain_epoch;            /* this launch's epoch; it waits for epoch-1 on the tiles it reads */
-    int chain_pad;
+    int batch;                       /* frames of a batched denoiser launch (gridDim.z); 1 otherwise    */
 } orion_kargs;
 
 #endif

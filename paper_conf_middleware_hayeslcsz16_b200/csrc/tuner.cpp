@@ -265,7 +265,8 @@ orion_status orion_tune_step(orion_tuner *t, const orion_args *a, void *stream, 
     Fig9 &f = t->f;
     CUstream s = (CUstream)stream;
     const Driver &D = drv();
-    const double work = (double)(a->row_end - a->row_begin) * (double)a->width;
+    // output elements of the iteration (every frame of a batch, orion_args.batch)
+    const double work = (double)(a->row_end - a->row_begin) * (double)a->width * (double)(a->batch > 1 ? a->batch : 1);
     if (a->row_begin == a->row_end && a->width > 0 && a->row_begin >= 0 && a->row_end <= a->height) {
         // an empty band is not an iteration: nothing is launched, timed or fed to Fig. 9 (a
         // zero-work sample would be in other units than ns per output element)
@@ -375,8 +376,10 @@ orion_status orion_tune_step_host(orion_tuner *t, const orion_args *a, void *dev
     if (def.kind == K_SRAD) return fail(ORION_E_INVALID, "orion_tune_step_host: not available for srad");
     const size_t elem = def.kind == K_STENCIL ? 4 : 16;
     const size_t row = (size_t)a->width * elem;
-    const size_t in_bytes = (size_t)(a->src_row_end - a->src_row_begin) * row;
-    const size_t out_bytes = (size_t)(a->row_end - a->row_begin) * row;
+    // a batch (orion_args.batch, whole frames) is copied as one block of B frames each way
+    const size_t nb = a->batch > 1 ? (size_t)a->batch : 1;
+    const size_t in_bytes = (size_t)(a->src_row_end - a->src_row_begin) * row * nb;
+    const size_t out_bytes = (size_t)(a->row_end - a->row_begin) * row * nb;
     if (a->src_row_end < a->src_row_begin || (def.kind == K_STENCIL && (!dev_aux || !a->aux)))
         return fail(ORION_E_INVALID, "orion_tune_step_host: bad argument");
     const Driver &D = drv();
@@ -544,8 +547,14 @@ orion_status orion_host_pipe_submit(orion_host_pipe *p, const orion_args *a, ori
                                     long long *h2d, long long *d2h)
 {
     if (!p || !a || !a->src || !a->dst) return fail(ORION_E_INVALID, "orion_host_pipe_submit: NULL");
-    const int in_rows = a->src_row_end - a->src_row_begin;
-    const int out_rows = a->row_end - a->row_begin;
+    // a batch (orion_args.batch, whole frames) occupies B frames' rows of a slot
+    const int nb = a->batch > 1 ? a->batch : 1;
+    const long long in_rows_ll = (long long)(a->src_row_end - a->src_row_begin) * nb;
+    const long long out_rows_ll = (long long)(a->row_end - a->row_begin) * nb;
+    if (in_rows_ll > p->max_rows || out_rows_ll > p->max_rows)
+        return fail(ORION_E_INVALID, "orion_host_pipe_submit: frame does not fit the pipe");
+    const int in_rows = (int)in_rows_ll;
+    const int out_rows = (int)out_rows_ll;
     if (a->width != p->width || in_rows < 0 || in_rows > p->max_rows || out_rows < 0 || out_rows > p->max_rows ||
         a->dst_row_begin > a->row_begin || (p->t->v->def->kind == K_STENCIL && !a->aux))
         return fail(ORION_E_INVALID, "orion_host_pipe_submit: frame does not fit the pipe");

@@ -102,6 +102,16 @@ orion_status make_kargs(const KernelDef &def, const orion_args *a, orion_kargs *
         return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id +
                                          ": a stencil launch reads its predecessor's output (not independent)");
     k->nowait = (a->flags & ORION_ARGS_INDEPENDENT) ? 1 : 0;
+    k->batch = 1;
+    if (a->batch < 0 || a->batch > 65535) return fail(ORION_E_INVALID, "orion_launch: batch out of range");
+    if (a->batch > 1) {
+        if (def.kind == K_STENCIL || def.kind == K_SRAD)
+            return fail(ORION_E_INVALID, std::string("orion_launch: ") + def.id + ": batches are for the denoisers");
+        if (a->row_begin != 0 || a->row_end != a->height || a->src_row_begin != 0 || a->src_row_end != a->height ||
+            a->dst_row_begin != 0 || a->n_fanout || a->chain)
+            return fail(ORION_E_INVALID, "orion_launch: a batch holds whole frames (no bands, fan-out or chain)");
+        k->batch = a->batch;
+    }
     if (a->chain) {
         const orion_chain *c = a->chain;
         if (!def.chain || c->def != &def)
@@ -173,12 +183,12 @@ static int pdl_enabled_setting()
 // kernel of the stream drains; every kernel waits (griddepcontrol.wait, kernels/common.cuh and
 // orion_srad_stats) for its predecessor's completion before touching memory, so results are
 // unchanged.
-static orion_status launch_maybe_pdl(CUfunction fn, unsigned gx, unsigned gy, unsigned bx, unsigned by,
+static orion_status launch_maybe_pdl(CUfunction fn, unsigned gx, unsigned gy, unsigned gz, unsigned bx, unsigned by,
                                      unsigned smem, CUstream s, void **params, const void *tag = nullptr)
 {
     note_stream_launch(s, tag);
     if (!pdl_enabled()) {
-        ORION_CU(drv().cuLaunchKernel(fn, gx, gy, 1, bx, by, 1, smem, s, params, nullptr));
+        ORION_CU(drv().cuLaunchKernel(fn, gx, gy, gz, bx, by, 1, smem, s, params, nullptr));
         return ORION_OK;
     }
     CUlaunchAttribute attr;
@@ -189,7 +199,7 @@ static orion_status launch_maybe_pdl(CUfunction fn, unsigned gx, unsigned gy, un
     std::memset(&cfg, 0, sizeof cfg);
     cfg.gridDimX = gx;
     cfg.gridDimY = gy;
-    cfg.gridDimZ = 1;
+    cfg.gridDimZ = gz;
     cfg.blockDimX = bx;
     cfg.blockDimY = by;
     cfg.blockDimZ = 1;
@@ -210,7 +220,8 @@ orion_status launch_fn(const KernelDef &def, CUfunction fn, int dyn_bytes, const
     const unsigned gx = (unsigned)((k.width + def.tile_w - 1) / def.tile_w);
     const unsigned gy = (unsigned)((rows + def.tile_h - 1) / def.tile_h);
     void *params[] = {const_cast<orion_kargs *>(&k)};
-    ORION_TRY(launch_maybe_pdl(fn, gx, gy, (unsigned)def.bx, (unsigned)def.by, (unsigned)dyn_bytes, s, params, tag));
+    const unsigned gz = (unsigned)(k.batch > 1 ? k.batch : 1);    // frames of a batched launch
+    ORION_TRY(launch_maybe_pdl(fn, gx, gy, gz, (unsigned)def.bx, (unsigned)def.by, (unsigned)dyn_bytes, s, params, tag));
     g_launches.fetch_add(1);
     return ORION_OK;
 }
@@ -691,7 +702,7 @@ extern "C" orion_status orion_srad_stats_init(int device, void *J, int width, in
     CUfunction f;
     ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_srad_stats_init"));
     void *params[] = {&k};
-    ORION_TRY(launch_maybe_pdl(f, (unsigned)slots, 1, 32, 1, 0, (CUstream)stream, params));
+    ORION_TRY(launch_maybe_pdl(f, (unsigned)slots, 1, 1, 32, 1, 0, (CUstream)stream, params));
     g_launches.fetch_add(1);
     return ORION_OK;
 }
@@ -707,7 +718,7 @@ extern "C" orion_status orion_srad_roi_stats(int device, const void *J, int widt
     CUfunction f;
     ORION_CU(drv().cuModuleGetFunction(&f, m, "orion_srad_stats"));
     void *params[] = {&J, &width, &r1, &r2, &c1, &c2, &q0};
-    ORION_TRY(launch_maybe_pdl(f, 1, 1, 1024, 1, 0, (CUstream)stream, params));
+    ORION_TRY(launch_maybe_pdl(f, 1, 1, 1, 1024, 1, 0, (CUstream)stream, params));
     g_launches.fetch_add(1);
     return ORION_OK;
 }

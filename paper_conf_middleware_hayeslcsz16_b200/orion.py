@@ -80,7 +80,7 @@ class Args(ctypes.Structure):
                 ("src_row_begin", ctypes.c_int), ("src_row_end", ctypes.c_int),
                 ("dst_row_begin", ctypes.c_int), ("fparam", ctypes.c_float * 8),
                 ("fanout", ctypes.c_void_p * 8), ("n_fanout", ctypes.c_int), ("flags", ctypes.c_int),
-                ("chain", ctypes.c_void_p)]
+                ("chain", ctypes.c_void_p), ("batch", ctypes.c_int)]
 
 
 ARGS_INDEPENDENT = 1       # orion.h ORION_ARGS_INDEPENDENT
@@ -248,10 +248,11 @@ def compile_info(kernel_id: str, block_threads: int, reg_cap: int) -> dict:
 # ---- launch arguments ----------------------------------------------------------------------
 def denoise_args(kernel_id: str, src: int, dst: int, width: int, height: int, row_begin: int = 0,
                  row_end: int | None = None, src_row_begin: int = 0, src_row_end: int | None = None,
-                 dst_row_begin: int | None = None, params=None, independent: bool = False) -> Args:
+                 dst_row_begin: int | None = None, params=None, independent: bool = False, batch: int = 1) -> Args:
     """Arguments of one denoiser launch.  independent: ORION_ARGS_INDEPENDENT -- the caller asserts
     the launch touches nothing the stream's previous kernel writes (e.g. the next frame, in its own
-    buffers), so with PDL it need not wait for that kernel."""
+    buffers), so with PDL it need not wait for that kernel.  batch: B > 1 whole frames stacked in
+    src / dst (frame f at f * width * height pixels), one launch."""
     row_end = height if row_end is None else row_end
     src_row_end = height if src_row_end is None else src_row_end
     dst_row_begin = row_begin if dst_row_begin is None else dst_row_begin
@@ -260,6 +261,7 @@ def denoise_args(kernel_id: str, src: int, dst: int, width: int, height: int, ro
     for i, x in enumerate(p):
         a.fparam[i] = x
     a.flags = ARGS_INDEPENDENT if independent else 0
+    a.batch = batch
     return a
 
 

@@ -1,6 +1,6 @@
 """Launch ONE kernel variant once on a synthetic frame (for ncu --set full captures).
 
-usage: python tools/ncu_one.py KERNEL LEVEL W H [THREADS] [REPEAT]
+usage: python tools/ncu_one.py KERNEL LEVEL W H [THREADS] [REPEAT] [BATCH]
   LEVEL = index into the level list (-1 = max occupancy, 'orig' = natural build, 'best' = the
   sweep's fastest level, 'all' = every level once, in order).  Levels are realised as bench.py realises them (MIN_CARVEOUT).
 """
@@ -15,6 +15,7 @@ from paper_conf_middleware_hayeslcsz16_b200 import orion as O  # noqa: E402
 kernel, lev, W, H = sys.argv[1], sys.argv[2], int(sys.argv[3]), int(sys.argv[4])
 threads = int(sys.argv[5]) if len(sys.argv) > 5 else 0
 repeat = int(sys.argv[6]) if len(sys.argv) > 6 else 1
+batch = int(sys.argv[7]) if len(sys.argv) > 7 else 1     # frames per launch (orion_args.batch)
 torch.cuda.set_device(0)
 sp = torch.cuda.current_stream().cuda_stream
 mode = O.REALISE_MAX_SMEM if os.environ.get("ORION_REALISE") == "max" else O.REALISE_MIN_CARVEOUT
@@ -45,10 +46,11 @@ elif kernel.startswith("hotspot"):
     O.generate_thermal(0, a.data_ptr(), p.data_ptr(), W, H, stream=sp)
     args = O.hotspot_args(a.data_ptr(), b.data_ptr(), p.data_ptr(), W, H)
 else:
-    a = torch.empty((H, W, 4), device="cuda")
-    b = torch.empty((H, W, 4), device="cuda")
-    O.generate_rgba(0, a.data_ptr(), W, H, sigma=0.13, stream=sp)
-    args = O.denoise_args(kernel, a.data_ptr(), b.data_ptr(), W, H)
+    a = torch.empty((batch, H, W, 4), device="cuda")
+    b = torch.empty((batch, H, W, 4), device="cuda")
+    for f in range(batch):
+        O.generate_rgba(0, a[f].data_ptr(), W, H, seed=1 + f, sigma=0.13, stream=sp)
+    args = O.denoise_args(kernel, a.data_ptr(), b.data_ptr(), W, H, batch=batch)
 torch.cuda.synchronize()
 if lev == "best":   # the exhaustive sweep's fastest level (what the tuner should settle on)
     ms = v.sweep(args, sp, rounds=5)
