@@ -11,9 +11,9 @@ dependent launch and issue mode as the timed loops --
   crops whose 100-cell margin holds the dependency cone.
 * SRAD: the 8192^2 grid, 3 chained `srad_f32hs` iterations (statistics fused) through the tuner
   against O5 (double) over the WHOLE grid, <= 1e-5 relative.
-* C1: 64^2 KNN frames (`knn_f4_t16`) tuned without PDL, then the settled iterations of 48
-  independent frames captured as one CUDA graph WITH programmatic edges (consecutive frames run
-  concurrently) and replayed: every frame against the double oracle.
+* C1: batches of 64 64^2 KNN frames (orion_args.batch; `knn_f4`, 256-thread CTAs) tuned without
+  PDL, then the settled iterations of 6 independent batches captured as one CUDA graph WITH
+  programmatic edges and replayed: all 384 frames against the double oracle.
 * C4: two independent 4096^2 frames of `nlm_f4_regheavy` through the tuner (its 16-level ladder
   explored); one whole frame against the double oracle.
 """
@@ -160,26 +160,28 @@ def test_srad_chained_tuned_whole_grid(dev):
     v.close()
 
 
-def test_c1_graph_of_independent_frames_vs_oracle(dev):
+def test_c1_graph_of_independent_batches_vs_oracle(dev):
+    # bench.py's C1: batches of 64x64 frames (orion_args.batch) through knn_f4 with 256-thread CTAs,
+    # tuned without PDL, then the settled iterations captured as a CUDA graph with programmatic
+    # edges and replayed; every frame of every batch against the double oracle
     W = H = 64
-    n = 48
-    v, _ = O.build_all_levels(0, "knn_f4_t16", mode=O.REALISE_MIN_CARVEOUT)
-    imgs = [synth.noisy_rgba(W, H, seed=1 + f, sigma=0.2) for f in range(n)]
-    srcs = [torch.from_numpy(im).cuda() for im in imgs]
-    dsts = [torch.full_like(s, float("nan")) for s in srcs]
-    args = [O.denoise_args("knn_f4_t16", srcs[f].data_ptr(), dsts[f].data_ptr(), W, H, independent=True)
-            for f in range(n)]
+    B, nb = 64, 6
+    v, _ = O.build_all_levels(0, "knn_f4", 256, mode=O.REALISE_MIN_CARVEOUT)
+    imgs = np.stack([synth.noisy_rgba(W, H, seed=1 + f, sigma=0.2) for f in range(B * nb)])
+    src = torch.from_numpy(imgs).cuda().view(nb, B, H, W, 4)
+    dst = torch.full_like(src, float("nan"))
+    args = [O.denoise_args("knn_f4", src[b].data_ptr(), dst[b].data_ptr(), W, H, independent=True, batch=B)
+            for b in range(nb)]
     prev = O.set_pdl(False)                  # bench.py: the sweep and the exploration run without PDL
     try:
         t = bench_tuner(v)
         s = 0
-        while s < 20 or t.final()[0] < 0:
-            t.step(args[s % n], sp())
+        while s < 12 or t.final()[0] < 0:
+            t.step(args[s % nb], sp())
             s += 1
             assert s < 400
         torch.cuda.synchronize()
-        for d in dsts:
-            d.fill_(float("nan"))
+        dst.fill_(float("nan"))
         O.set_pdl(True)                      # the timed graph keeps programmatic edges
         g = t.capture(args)
         for _ in range(3):
@@ -189,10 +191,11 @@ def test_c1_graph_of_independent_frames_vs_oracle(dev):
         t.close()
     finally:
         O.set_pdl(prev)
-    res = oracle_par.map_threads(lambda im: oracle.denoise("knn", im), imgs)
-    for f in range(n):
+    res = oracle_par.map_threads(lambda im: oracle.denoise("knn", im), list(imgs))
+    got = dst.view(B * nb, H, W, 4).cpu().numpy()
+    for f in range(B * nb):
         out, alt, amb = res[f]
-        g_ = dsts[f].cpu().numpy()
+        g_ = got[f]
         e = np.abs(g_[..., :3].astype(np.float64) - out).max(-1)
         ok = (e <= 1e-5) | (amb & (np.abs(g_[..., :3].astype(np.float64) - alt).max(-1) <= 1e-5))
         assert ok.all(), (f, int((~ok).sum()), float(e.max()))
