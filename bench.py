@@ -46,7 +46,7 @@ WORKLOADS = {
     # KNN: 49 taps x (3 FSUB + FMUL + 2 FFMA distance, 1 FFMA exponent, 3 FFMA + 1 FADD
     # accumulate, 1 compare) + ~10 for the blend
     # C1's 64x64 frames run as batches (orion_args.batch: B frames per launch, one batch per
-    # tuner iteration and per step) through the tile kernel with 256-thread CTAs; --c1-batch 1
+    # tuner iteration and per step) through the tile kernel with 256-thread CTAs; --batch 1
     # restores one frame per step (use --kernel knn_f4_t16, the small-frame kernel, then)
     "c1": dict(kernel="knn_f4", threads=256, batch=256, W=64, H=64, sigma=0.2, unit="Mpix/s",
                name="imageDenoising KNN 64x64 RGBA r=3", insts=49 * 12 + 10, bytes=32, steps=300, cfg_index=0),
@@ -70,6 +70,10 @@ WORKLOADS = {
 }
 SUB_RECORDS = ("c1", "c3", "c4", "srad", "c5")
 ROI = (0, 127, 0, 127)     # SRAD's ROI statistics window (reading R-SRAD: Rodinia's default)
+
+
+def is_stencil_id(kernel: str) -> bool:
+    return kernel.startswith("hotspot") or kernel.startswith("srad")
 
 
 def load_peaks():
@@ -432,7 +436,11 @@ def measure_single(key: str, args, *, steps: int, warmup: int, rounds: int, cpu_
     sp = stream.cuda_stream
     wl = WORKLOADS[key]
     kernel, W, H = kernel or wl["kernel"], wl["W"], wl["H"]
-    batch = max(1, args.c1_batch if key == "c1" and args.c1_batch > 0 else wl.get("batch", 1))
+    # frames per launch / step (orion_args.batch): --batch for the headline workload, else the
+    # workload's default (C1: 256)
+    batch = max(1, args.batch if args.batch > 0 and key == args.workload else wl.get("batch", 1))
+    if is_stencil_id(kernel):
+        batch = 1
     threads = wl.get("threads", 0) if kernel == wl["kernel"] else 0
     is_srad = kernel.startswith("srad_f32")
     is_stencil = kernel.startswith("hotspot") or is_srad
@@ -1431,8 +1439,9 @@ def main(argv=None):
     ap.add_argument("--no-anchor", action="store_true", help="N > 1: skip C5 at P = 1 on rank 0")
     ap.add_argument("--size", type=int, default=0, help="override the C5 image side (tests)")
     ap.add_argument("--kernel", default="", help="override the headline workload's kernel id (same family)")
-    ap.add_argument("--c1-batch", type=int, default=0,
-                    help="C1: 64x64 frames per launch / step (0: the workload's default, 256; 1: one frame)")
+    ap.add_argument("--batch", type=int, default=0,
+                    help="denoisers: frames per launch / step of the headline workload (0: the workload's default "
+                         "-- C1 256, the others 1)")
     ap.add_argument("--c5-chunks", type=int, default=4, help="C5: row chunks per band whose all-gathers overlap compute")
     ap.add_argument("--c5-mode", default="auto", choices=("auto", "fanout", "gather"),
                     help="C5 exchange: kernel fan-out into symmetric memory (auto: when available) or all-gather")
