@@ -132,7 +132,8 @@ orion_status orion_ctas_per_sm_carveout(const orion_device_limits *dev, int bloc
  * ptxas (the "original" build).  Kernel ids (the paper's benchmarks, Table 2 P:L725-
  * P:L739; their math per readings R-O2, R-O3, R-SRAD):
  *   imageDenoising KNN: "knn_f4" (T = 128 / 256 / 64), "knn_f4_p1" (one pixel per
- *       thread, same bits), "knn_f4_t16" (the 49 taps of a pixel over 16 lanes; the C1 default);
+ *       thread, same bits), "knn_f4_t16" (the 49 taps of a pixel over 16 lanes: single small frames; C1 runs batches
+ *       of frames through "knn_f4" at T = 256);
  *   imageDenoising NLM: "nlm_f4_w" (box sums + symmetric pairs, 3 pairs per pass,
  *       128-column tiles; the C2 / C5 default), "nlm_f4" (same, 122-column tiles),
  *       "nlm_f4_direct" (the direct 2401-term definition, cross-check form), "nlm_f4_regheavy"
