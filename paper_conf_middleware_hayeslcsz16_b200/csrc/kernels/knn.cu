@@ -16,6 +16,18 @@
 #define KNN_R 3
 #define KNN_A 49
 
+// The exponent of a tap's weight, w = 2^e: e = d * (-Noise log2 e) + geo_ij with d = |c - c00|^2 =
+// (dr^2 + dg^2) + db^2 -- the (r, g) difference and squares packed (FADD2, FMUL2), a sum of
+// non-negative terms 3 roundings deep (reading R-NLM-FP).  nrg / nb: the negated centre colour.
+ORION_DEVICE float knn_tap_exponent(float4 c, float2 nrg, float nb, float nl2, float geo)
+{
+    const float2 drg = __fadd2_rn(make_float2(c.x, c.y), nrg);
+    const float2 q = __fmul2_rn(drg, drg);
+    const float db = __fadd_rn(c.z, nb);
+    const float d = __fmaf_rn(db, db, __fadd_rn(q.x, q.y));
+    return __fmaf_rn(d, nl2, geo);
+}
+
 template <int BX, int BY, int PY>
 __device__ __forceinline__ void knn_body(const orion_kargs &a)
 {
@@ -29,15 +41,22 @@ __device__ __forceinline__ void knn_body(const orion_kargs &a)
 
     const int tx = threadIdx.x, ty = threadIdx.y;
     const float nl2 = a.fparam[0];
-    const float wthr = a.fparam[2];
 
+    const float ethr = a.fparam[3];          // log2(wthr): [w > wthr] decided on the exponent
+
+    // packed fp32x2 taps (FADD2 / FMUL2 / FFMA2, two IEEE .rn operations each): the (r, g)
+    // difference, its squares, and the accumulations (w r, w g) and (w b, w) in pairs
     float4 c00[PY];
-    float ax[PY], ay[PY], az[PY], sw[PY];
+    float2 nrg[PY];                          // -(r, g) of the centre pixel
+    float nb[PY];
+    float2 axy[PY], azs[PY];                 // (sum w r, sum w g), (sum w b, sum w)
     int cnt[PY];
 #pragma unroll
     for (int p = 0; p < PY; ++p) {
         c00[p] = tile[(ty * PY + p + KNN_R) * TW + tx + KNN_R];
-        ax[p] = ay[p] = az[p] = sw[p] = 0.0f;
+        nrg[p] = make_float2(-c00[p].x, -c00[p].y);
+        nb[p] = -c00[p].z;
+        axy[p] = azs[p] = make_float2(0.0f, 0.0f);
         cnt[p] = 0;
     }
 #pragma unroll
@@ -50,13 +69,11 @@ __device__ __forceinline__ void knn_body(const orion_kargs &a)
                 const int i = r - KNN_R - p;          // row offset of this tap for pixel p
                 if (i < -KNN_R || i > KNN_R) continue; // resolved at compile time
                 const int j = jj - KNN_R;
-                const float d = dist2(c, c00[p]);
-                const float w = ex2(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
-                ax[p] = __fmaf_rn(w, c.x, ax[p]);
-                ay[p] = __fmaf_rn(w, c.y, ay[p]);
-                az[p] = __fmaf_rn(w, c.z, az[p]);
-                sw[p] = __fadd_rn(sw[p], w);
-                cnt[p] += (w > wthr);
+                const float e = knn_tap_exponent(c, nrg[p], nb[p], nl2, geo_l2_rt(i, j));
+                const float w = ex2(e);
+                axy[p] = __ffma2_rn(make_float2(w, w), make_float2(c.x, c.y), axy[p]);
+                azs[p] = __ffma2_rn(make_float2(w, w), make_float2(c.z, 1.0f), azs[p]);
+                cnt[p] += (e > ethr);
             }
         }
     }
@@ -65,7 +82,7 @@ __device__ __forceinline__ void knn_body(const orion_kargs &a)
 #pragma unroll
     for (int p = 0; p < PY; ++p) {
         const int y = y0 + ty * PY + p;
-        if (y < a.row_end) store_out(a, x, y, lerp_out(c00[p], ax[p], ay[p], az[p], sw[p], cnt[p], a));
+        if (y < a.row_end) store_out(a, x, y, lerp_out(c00[p], axy[p].x, axy[p].y, azs[p].x, azs[p].y, cnt[p], a));
     }
     fanout_column(a, x, y0 + ty * PY, min(y0 + ty * PY + PY, a.row_end));
 }
@@ -104,8 +121,10 @@ __device__ __forceinline__ void knn_tap_split_body(const orion_kargs &a)
     const int xc = min(x, W - 1);
     const float4 *src = (const float4 *)a.src + frame_px(a) - (size_t)a.src_row_begin * (size_t)W;
     const float nl2 = a.fparam[0];
-    const float wthr = a.fparam[2];
     const float4 c00 = __ldg(src + (size_t)y * (size_t)W + xc);
+    const float2 nrg = make_float2(-c00.x, -c00.y);
+    const float nb = -c00.z;
+    const float ethr = a.fparam[3];
     float ax = 0.0f, ay = 0.0f, az = 0.0f, sw = 0.0f;
     int cnt = 0;
 #pragma unroll
@@ -115,13 +134,13 @@ __device__ __forceinline__ void knn_tap_split_body(const orion_kargs &a)
         const int i = k / 7 - KNN_R, j = k % 7 - KNN_R;
         const int gy = clampi(y + i, 0, H - 1), gx = clampi(xc + j, 0, W - 1);
         const float4 c = __ldg(src + (size_t)gy * (size_t)W + gx);
-        const float d = dist2(c, c00);
-        const float w = ex2(__fmaf_rn(d, nl2, geo_l2_rt(i, j)));
+        const float e = knn_tap_exponent(c, nrg, nb, nl2, geo_l2_rt(i, j));
+        const float w = ex2(e);
         ax = __fmaf_rn(w, c.x, ax);
         ay = __fmaf_rn(w, c.y, ay);
         az = __fmaf_rn(w, c.z, az);
         sw = __fadd_rn(sw, w);
-        cnt += (w > wthr);
+        cnt += (e > ethr);
     }
 #pragma unroll
     for (int o = LP / 2; o > 0; o >>= 1) {
