@@ -46,16 +46,15 @@ __device__ __forceinline__ void knn_body(const orion_kargs &a)
 
     // packed fp32x2 taps (FADD2 / FMUL2 / FFMA2, two IEEE .rn operations each): the (r, g)
     // difference, its squares, and the accumulations (w r, w g) and (w b, w) in pairs
-    float4 c00[PY];
-    float2 nrg[PY];                          // -(r, g) of the centre pixel
-    float nb[PY];
+    float2 nrg[PY];                          // -(r, g) of the centre pixel (the centre itself is
+    float nb[PY];                            //  read again from the tile for the blend)
     float2 axy[PY], azs[PY];                 // (sum w r, sum w g), (sum w b, sum w)
     int cnt[PY];
 #pragma unroll
     for (int p = 0; p < PY; ++p) {
-        c00[p] = tile[(ty * PY + p + KNN_R) * TW + tx + KNN_R];
-        nrg[p] = make_float2(-c00[p].x, -c00[p].y);
-        nb[p] = -c00[p].z;
+        const float4 c00 = tile[(ty * PY + p + KNN_R) * TW + tx + KNN_R];
+        nrg[p] = make_float2(-c00.x, -c00.y);
+        nb[p] = -c00.z;
         axy[p] = azs[p] = make_float2(0.0f, 0.0f);
         cnt[p] = 0;
     }
@@ -82,7 +81,8 @@ __device__ __forceinline__ void knn_body(const orion_kargs &a)
 #pragma unroll
     for (int p = 0; p < PY; ++p) {
         const int y = y0 + ty * PY + p;
-        if (y < a.row_end) store_out(a, x, y, lerp_out(c00[p], axy[p].x, axy[p].y, azs[p].x, azs[p].y, cnt[p], a));
+        const float4 c00 = tile[(ty * PY + p + KNN_R) * TW + tx + KNN_R];
+        if (y < a.row_end) store_out(a, x, y, lerp_out(c00, axy[p].x, axy[p].y, azs[p].x, azs[p].y, cnt[p], a));
     }
     fanout_column(a, x, y0 + ty * PY, min(y0 + ty * PY + PY, a.row_end));
 }
