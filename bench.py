@@ -929,9 +929,9 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
     tuner = O.Tuner(variants, O.default_cfg(samples_per_level=args.samples))
     # the exchange: the kernels' fan-out stores into every rank's symmetric-memory image (compute
     # + gather in one kernel over NVLink), else chunked all-gathers overlapped with compute
-    # P = 1: no exchange, unless the fan-out is requested explicitly (the symmetric-memory path
+    # P = 1: no exchange, unless the fan-out or the gather is requested explicitly (either path
     # exercised on one GPU over a one-rank NCCL group, see run_single)
-    mode, fan, fan_note = ("none" if world == 1 and mode_req != "fanout" else mode_req), None, None
+    mode, fan, fan_note = ("none" if world == 1 and mode_req not in ("fanout", "gather") else mode_req), None, None
     full = None
     if mode in ("auto", "fanout"):
         try:
@@ -1071,9 +1071,10 @@ def measure_c5(args, *, world: int, rank: int, local: int, steps: int, warmup: i
                                       "+ device barrier" if mode == "fanout" else
                                       f"all_gather of {chunks} row chunks on a side stream, overlapped with the "
                                       f"next chunk's kernel" if mode == "gather" else "none (P=1)")
-                       if world > 1 or mode == "fanout" else "none (P=1)",
+                       if world > 1 or mode in ("fanout", "gather") else "none (P=1)",
                        "collective_note": fan_note, "l2": "4 GiB frame >> L2",
-                       "parallelism": f"row-sharded x{world}", "backend": backend_name() if world > 1 else None},
+                       "parallelism": f"row-sharded x{world}",
+                       "backend": backend_name() if world > 1 or mode != "none" else None},
             "compute_only": {"value": H * W * steps / (comp * 1e-3) / 1e6, "unit": "Mpix/s",
                              "ms_per_step": comp / steps},
             "exchange_ms_per_step": gat / steps,
@@ -1287,8 +1288,9 @@ def run_single(args):
     wl = WORKLOADS[key]
     steps = args.steps or wl["steps"]
     if key == "c5":
-        if args.c5_mode == "fanout" and not dist_initialized():
-            # a one-rank NCCL group: the symmetric-memory fan-out path on one GPU
+        if args.c5_mode in ("fanout", "gather") and not dist_initialized():
+            # a one-rank NCCL group: the symmetric-memory fan-out path, or the chunked NCCL
+            # all-gather overlapped with compute, exercised on one GPU
             import torch.distributed as dist
             dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{free_port()}", world_size=1, rank=0,
                                     device_id=torch.device("cuda", local))

@@ -118,3 +118,20 @@ def test_bench_c5_fanout_path_one_gpu(dev):
     assert "fan-out" in d["config"]["collective"] and d["n_gpus"] == 1
     assert d["value"] > 0 and d["compute_only"]["value"] > 0 and d["e2e"]["value"] > 0
     assert d["per_rank"][0]["final_k"] >= 1
+
+
+def test_bench_c5_gather_path_one_gpu(dev):
+    # bench.py's C5 with the chunked NCCL all-gather requested on one GPU (a one-rank NCCL group):
+    # row chunks computed as kernel-split iterations, each chunk's all-gather on a side stream
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--workload", "c5", "--only", "--size", "2048",
+                        "--c5-mode", "gather", "--steps", "3", "--warmup", "3", "--rounds", "3"],
+                       capture_output=True, text=True, timeout=900, cwd=root)
+    assert r.returncode == 0, r.stderr[-3000:]
+    d = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
+    assert "all_gather" in d["config"]["collective"] and d["n_gpus"] == 1, d["config"]
+    assert d["value"] > 0 and d["compute_only"]["value"] > 0 and d["e2e"]["value"] > 0
