@@ -1,7 +1,7 @@
 """Per-level ncu evidence (SURVEY 8(d) "ncu evidence per level"): profile one launch of every
 occupancy level of a kernel with a small metric set and write a table to profiles/.
 
-On the GPU box:   python tools/ncu_levels.py run KERNEL W H [THREADS]   -> gpurun_out/levels_KERNEL.csv
+On the GPU box:   python tools/ncu_levels.py run KERNEL W H [THREADS] [BATCH]   -> gpurun_out/levels_KERNEL.csv
 Here:             python tools/ncu_levels.py summarise KERNEL ROUND     -> profiles/ncu_levels_ROUND_KERNEL.txt
 """
 import csv
@@ -31,10 +31,10 @@ SHORT = ["us", "regs", "lim_reg", "lim_smem", "occ_theo%", "occ_ach%", "local_ld
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def run(kernel, W, H, threads="0"):
+def run(kernel, W, H, threads="0", batch="1"):
     out = os.path.join(ROOT, "gpurun_out", f"levels_{kernel}.csv")
     cmd = ["ncu", "--clock-control", "none", "--nvtx", "--nvtx-include", "measure/", "--csv", "--metrics", ",".join(METRICS), "-k", "regex:orion_",
-           "--log-file", out, sys.executable, os.path.join(ROOT, "tools", "ncu_one.py"), kernel, "all", W, H, threads]
+           "--log-file", out, sys.executable, os.path.join(ROOT, "tools", "ncu_one.py"), kernel, "all", W, H, threads, "1", batch]
     subprocess.run(cmd, check=True)
 
 
